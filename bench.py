@@ -1,0 +1,549 @@
+#!/usr/bin/env python
+"""bench.py — Gist stash-time encode/decode throughput on B200 (driver contract).
+
+A "step" is one pass of the whole hot path over one minibatch of synthetic stashed feature
+maps: every stash site of the network is encoded in forward order (a1 Binarize + a2 MaxPool
+argmax for ReLU->Pool sites, a4 SSDC for ReLU/Pool->Conv sites, a6 DPR for the rest) and
+decoded in backward order (a3 fused pool+ReLU backward, a5 SSDC decode, a7 DPR decode).
+
+Metric (BASELINE.json): fp32 feature-map GB/s = (fp32 bytes of every stashed map encoded +
+fp32 bytes of every map decoded) / step time, i.e. 8 bytes per stashed element per step.
+Default workload: C3, VGG16-shaped stash sites, batch 64 per GPU, SSDC at 80% sparsity
+("over 80%"), DPR-fp16 (VGG16 needs FP16).  Inputs (3.9 GB per GPU) exceed
+the 126 MB L2, so no explicit flush is needed between steps.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl gist|reference] [--config C3]
+  torchrun --nproc-per-node N bench.py --gpus N ...     (one rank per GPU, NCCL)
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import workloads as WL  # noqa: E402
+
+CONFIG_INDEX = {"C1": 1, "C2": 2, "C3": 3, "C4": 4, "C5o": 5, "C5n": 6}
+FALLBACK_HBM_GBS = 6650.0  # B200_PROFILING.md fallback, used only if MEASURED_PEAKS.json is absent
+
+
+def baseline_metric() -> str:
+    with open(os.path.join(ROOT, "BASELINE.json")) as f:
+        return json.load(f)["metric"]
+
+
+def hbm_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+# --------------------------------------------------------------------------------- sites
+def pool_out(chw, g):
+    c, h, w = chw
+    kh, kw, sh, sw, ph, pw, cm = g
+
+    def dim(i, k, s, p):
+        span = i + 2 * p - k
+        o = (span + (s - 1 if cm else 0)) // s + 1
+        if cm and (o - 1) * s >= i + p:
+            o -= 1
+        return o
+    return (c, dim(h, kh, sh, ph), dim(w, kw, sw, pw))
+
+
+def words(n, per):
+    return -(-n // per)
+
+
+class Workload:
+    """Device buffers of one rank's minibatch for every stash site, and the step."""
+
+    def __init__(self, gist, cfg: WL.Config, batch: int, sparsity: float, dpr_bits: int, rank: int, dev,
+                 fuse_mask: bool):
+        self.g, self.dev, self.bits, self.fuse = gist, dev, dpr_bits, fuse_mask
+        self.sites = []
+        cidx = CONFIG_INDEX.get(cfg.key, 9)
+        ssdc_sites = [s for s in WL.sites_for(cfg) if s.kind == "ssdc"]
+        self.nnz_all = torch.zeros(max(1, len(ssdc_sites)), dtype=torch.int64, device=dev)
+        k_ssdc = 0
+        max_n = 1
+        for si, s in enumerate(WL.sites_for(cfg)):
+            shape = (batch,) + s.chw
+            n = s.numel(batch)
+            max_n = max(max_n, n)
+            seed = WL.seed_for(cidx, si, rank)
+            d = {"site": s, "shape": shape, "n": n}
+            if s.kind in ("relu_pool", "pool_only"):
+                d["y"] = WL.relu_map(shape, 0.5, seed, dev)  # ReLU output feeding the pool
+                oshape = (batch,) + pool_out(s.chw, s.pool)
+                d["n_out"] = oshape[0] * oshape[1] * oshape[2] * oshape[3]
+                d["out"] = torch.empty(oshape, device=dev)
+                d["arg"] = torch.empty(words(d["n_out"], 8), dtype=torch.int32, device=dev)
+                d["mask"] = torch.empty(words(n, 32), dtype=torch.int32, device=dev) if s.kind == "relu_pool" else None
+                d["dY"] = WL.grad_map(oshape, seed + 500, dev)
+            elif s.kind == "ssdc":
+                d["y"] = WL.relu_map(shape, sparsity, seed, dev)
+                rows = words(n, 256)
+                d["row_end"] = torch.empty(rows, dtype=torch.int32, device=dev)
+                d["col"] = torch.empty(n, dtype=torch.uint8, device=dev)
+                d["val"] = torch.empty(n, dtype=torch.float32, device=dev)
+                d["nnz"] = self.nnz_all[k_ssdc:k_ssdc + 1]
+                d["ws"] = torch.empty(gist.gist_ssdc_workspace_bytes(n), dtype=torch.uint8, device=dev)
+                k_ssdc += 1
+            else:
+                d["y"] = WL.dpr_map(shape, seed, dev)
+                d["packed"] = torch.empty(gist.gist_dpr_words(n, dpr_bits), dtype=torch.int32, device=dev)
+            self.sites.append(d)
+        # decoded maps are short-lived (D lives only at its backward use): one scratch
+        self.scratch = torch.empty(max_n, dtype=torch.float32, device=dev)
+        self.stash_elems = sum(d["n"] for d in self.sites)
+        self.bytes_per_step = 8 * self.stash_elems  # 4n encoded + 4n decoded per site
+
+    # ---- one pass: encode all sites (forward), decode all sites (backward)
+    def step(self, timer=None):
+        g = self.g
+        t = timer or (lambda kind, d: _Null())
+        for d in self.sites:
+            k = d["site"].kind
+            if k == "relu_pool":
+                if self.fuse:
+                    with t("a2_maxpool_fwd_argmax+a1", d):
+                        g.gist_maxpool_fwd_argmax(d["y"], d["site"].pool, out=d["out"], argmax=d["arg"], mask=d["mask"])
+                else:
+                    with t("a1_binarize_encode", d):
+                        g.gist_binarize_encode(d["y"], mask=d["mask"])
+                    with t("a2_maxpool_fwd_argmax", d):
+                        g.gist_maxpool_fwd_argmax(d["y"], d["site"].pool, out=d["out"], argmax=d["arg"])
+            elif k == "pool_only":
+                with t("a2_maxpool_fwd_argmax", d):
+                    g.gist_maxpool_fwd_argmax(d["y"], d["site"].pool, out=d["out"], argmax=d["arg"])
+            elif k == "ssdc":
+                with t("a4_ssdc_encode", d):
+                    g.gist_ssdc_encode(d["y"], capacity=d["n"], row_end=d["row_end"], col=d["col"], val=d["val"],
+                                       nnz=d["nnz"], workspace=d["ws"])
+            else:
+                with t("a6_dpr_encode", d):
+                    g.gist_dpr_encode(d["y"], self.bits, packed=d["packed"])
+        for d in reversed(self.sites):
+            k = d["site"].kind
+            n = d["n"]
+            if k in ("relu_pool", "pool_only"):
+                dx = self.scratch[:n].view(d["shape"])
+                with t("a3_pool_relu_bwd", d):
+                    g.gist_pool_relu_bwd(d["dY"], d["arg"], d["mask"], d["shape"], d["site"].pool, dx=dx)
+            elif k == "ssdc":
+                with t("a5_ssdc_decode", d):
+                    g.gist_ssdc_decode(d["row_end"], d["col"], d["val"], n, x=self.scratch[:n])
+            else:
+                with t("a7_dpr_decode", d):
+                    g.gist_dpr_decode(d["packed"], n, self.bits, x=self.scratch[:n])
+
+    def nnz_host(self):
+        return self.nnz_all.cpu()
+
+    # ---- algorithmic bytes of one launch; nnz from the last step
+    def algo_bytes(self, kind, d, nnz=None):
+        n = d["n"]
+        if kind == "a1_binarize_encode":
+            return 4 * n + 4 * words(n, 32)
+        if kind.startswith("a2_maxpool_fwd_argmax"):
+            b = 4 * n + 4 * d["n_out"] + 4 * words(d["n_out"], 8)
+            return b + (4 * words(n, 32) if kind.endswith("+a1") else 0)
+        if kind == "a3_pool_relu_bwd":
+            return 4 * d["n_out"] + 4 * words(d["n_out"], 8) + (4 * words(n, 32) if d["mask"] is not None else 0) + 4 * n
+        if kind in ("a4_ssdc_encode", "a5_ssdc_decode"):
+            return 4 * n + 5 * nnz + 4 * words(n, 256)
+        if kind in ("a6_dpr_encode", "a7_dpr_decode"):
+            return 4 * n + 4 * words(n, {16: 2, 10: 3, 8: 4}[self.bits])
+        raise KeyError(kind)
+
+    def compression(self, nnz_list):
+        """Per-encoding compression ratio (fp32 bytes / encoded bytes), exact byte counts."""
+        fp32 = {"binarize": 0, "ssdc": 0, "dpr": 0}
+        enc = {"binarize": 0, "ssdc": 0, "dpr": 0}
+        k = 0
+        for d in self.sites:
+            s = d["site"]
+            if s.kind == "relu_pool":
+                fp32["binarize"] += 4 * d["n"]
+                enc["binarize"] += 4 * words(d["n"], 32) + 4 * words(d["n_out"], 8)
+            elif s.kind == "ssdc":
+                fp32["ssdc"] += 4 * d["n"]
+                enc["ssdc"] += 5 * int(nnz_list[k]) + 4 * words(d["n"], 256)
+                k += 1
+            elif s.kind == "dpr":
+                fp32["dpr"] += 4 * d["n"]
+                enc["dpr"] += 4 * words(d["n"], {16: 2, 10: 3, 8: 4}[self.bits])
+        out = {e: round(fp32[e] / enc[e], 4) for e in fp32 if enc[e]}
+        out["total"] = round(sum(fp32.values()) / max(1, sum(enc.values())), 4)
+        return out
+
+
+class _Null:
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        return False
+
+
+class KernelTimer:
+    """CUDA events around every launch, on the stream the kernels are launched on."""
+
+    def __init__(self, stream):
+        self.stream = stream
+        self.records = []  # (kind, site dict, start, end)
+
+    def __call__(self, kind, d):
+        timer = self
+
+        class _Ctx:
+            def __enter__(self_inner):
+                self_inner.s = torch.cuda.Event(enable_timing=True)
+                self_inner.e = torch.cuda.Event(enable_timing=True)
+                self_inner.s.record(timer.stream)
+                return self_inner
+
+            def __exit__(self_inner, *a):
+                self_inner.e.record(timer.stream)
+                timer.records.append((kind, d, self_inner.s, self_inner.e))
+                return False
+        return _Ctx()
+
+
+# --------------------------------------------------------------------------------- clocks
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except (OSError, FileNotFoundError):
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        self.lines = []
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                out, _ = self.proc.communicate(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+                out, _ = self.proc.communicate()
+            self.lines = [ln for ln in out.splitlines() if ln.strip()]
+        return False
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in getattr(self, "lines", []):
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# --------------------------------------------------------------------------------- oracle legs
+def oracle_pass(ref, sites_host, bits):
+    """The oracle (as it stands) over one sample: encode every site, then decode."""
+    for d in sites_host:
+        s = d["site"]
+        if s.kind in ("relu_pool", "pool_only"):
+            if s.kind == "relu_pool":
+                d["mask"] = ref.binarize_encode(d["y"])
+            d["out"], d["arg"] = ref.maxpool_fwd_argmax(d["y"], s.pool)
+        elif s.kind == "ssdc":
+            d["enc"] = ref.ssdc_encode(d["y"])
+        else:
+            d["packed"] = ref.dpr_encode(d["y"], bits)
+    for d in reversed(sites_host):
+        s = d["site"]
+        if s.kind in ("relu_pool", "pool_only"):
+            ref.pool_relu_bwd(d["dY"], d["arg"], d.get("mask"), d["y"].shape, s.pool)
+        elif s.kind == "ssdc":
+            ref.ssdc_decode(*d["enc"], d["n"])
+        else:
+            ref.dpr_decode(d["packed"], d["n"], bits)
+
+
+def oracle_sample(cfg, images: int, sparsity: float, seed0: int):
+    sites = []
+    for si, s in enumerate(WL.sites_for(cfg)):
+        shape = (images,) + s.chw
+        seed = seed0 + 1000 * si
+        d = {"site": s, "n": s.numel(images)}
+        if s.kind in ("relu_pool", "pool_only"):
+            d["y"] = WL.relu_map(shape, 0.5, seed).numpy()
+            d["dY"] = WL.grad_map((images,) + pool_out(s.chw, s.pool), seed + 500).numpy()
+        elif s.kind == "ssdc":
+            d["y"] = WL.relu_map(shape, sparsity, seed).numpy()
+        else:
+            d["y"] = WL.dpr_map(shape, seed).numpy()
+        sites.append(d)
+    return sites
+
+
+def cpu_baseline(cfg, sparsity, bits, budget_s):
+    """Oracle timed on the host (1 thread) on a bounded sample: whole images of the same
+    workload, added until ~budget_s seconds of oracle work."""
+    import oracle as ref
+    ref.lib()
+    images, elapsed, nbytes = 0, 0.0, 0
+    while elapsed < budget_s and images < 64:
+        sample = oracle_sample(cfg, 1, sparsity, 777 + images)
+        t0 = time.perf_counter()
+        oracle_pass(ref, sample, bits)
+        elapsed += time.perf_counter() - t0
+        nbytes += 8 * sum(d["n"] for d in sample)
+        images += 1
+    return {"value": round(nbytes / elapsed / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "sample": f"{images} image(s) of the {cfg.key} workload (all stash sites, encode+decode), "
+                      f"{elapsed:.1f} s single-threaded"}
+
+
+def run_reference(args, cfg):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return  # torchrun N>1: rank 0 alone runs the oracle arm
+    import oracle as ref
+    ref.lib()
+    images = 1
+    sample = oracle_sample(cfg, images, args.sparsity, 999)
+    for _ in range(args.warmup):
+        oracle_pass(ref, sample, args.dpr_bits)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle_pass(ref, sample, args.dpr_bits)
+    dt = (time.perf_counter() - t0) / max(1, args.steps)
+    nbytes = 8 * sum(d["n"] for d in sample)
+    value = nbytes / dt / 1e9
+    line = {
+        "impl": "reference", "metric": baseline_metric(), "value": round(value, 4), "unit": "GB/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": workload_config(args, cfg, images, note="bounded sample: 1 image per step"),
+        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                         "sample": f"{images} image of {cfg.key} per step (all stash sites, encode+decode)"},
+        "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def workload_config(args, cfg, batch, note=None):
+    c = {"workload": f"{cfg.key}: {cfg.description}", "net": cfg.net, "batch_per_gpu": batch,
+         "ssdc_sparsity": args.sparsity, "dpr_bits": args.dpr_bits,
+         "l2": "inputs larger than L2 (no flush needed)", "parallelism": f"dp{args.gpus} (minibatch shards, no "
+         "collective on the hot path)"}
+    if note:
+        c["note"] = note
+    return c
+
+
+# --------------------------------------------------------------------------------- main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["gist", "reference"], default="gist")
+    ap.add_argument("--config", default="C3", choices=sorted(CONFIG_INDEX))
+    ap.add_argument("--batch", type=int, default=None, help="per-GPU batch (default: the config's)")
+    ap.add_argument("--sparsity", type=float, default=None)
+    ap.add_argument("--dpr-bits", type=int, default=None)
+    ap.add_argument("--fuse-mask", action="store_true", help="a1 inside the a2 call")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=8.0)
+    ap.add_argument("--kernels-out", default=None, help="write the per-kernel breakdown JSON here")
+    args = ap.parse_args()
+    cfg = WL.CONFIGS[args.config]
+    args.sparsity = cfg.sparsity if args.sparsity is None else args.sparsity
+    args.dpr_bits = cfg.dpr_bits if args.dpr_bits is None else args.dpr_bits
+    batch = args.batch or cfg.batch
+    args.warmup = max(args.warmup, 3)
+
+    if args.impl == "reference":
+        run_reference(args, cfg)
+        return
+
+    import paper_conf_isca_jainpmtp18_b200 as gist
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+
+    def barrier():
+        if dist is not None:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    wl = Workload(gist, cfg, batch, args.sparsity, args.dpr_bits, rank, dev, args.fuse_mask)
+    stream = torch.cuda.current_stream(dev)
+    for _ in range(args.warmup):
+        wl.step()
+    barrier()
+
+    # ---- timed region: K steps, CUDA events on the launching stream, clocks sampled
+    timer = KernelTimer(stream)
+    launches0 = gist.gist_launch_count()
+    with ClockSampler(local) as clocks:
+        barrier()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record(stream)
+        for _ in range(args.steps):
+            wl.step(timer)
+        ev1.record(stream)
+        barrier()
+    launches = gist.gist_launch_count() - launches0
+    elapsed_ms = ev0.elapsed_time(ev1)
+    nnz = wl.nnz_host().tolist()
+
+    # per-kernel breakdown (device time of each launch, summed per kind)
+    per = {}
+    nnz_of = {}
+    k = 0
+    for d in wl.sites:
+        if d["site"].kind == "ssdc":
+            nnz_of[id(d)] = int(nnz[k])
+            k += 1
+    for kind, d, s, e in timer.records:
+        r = per.setdefault(kind, {"ms": 0.0, "launches": 0, "algo_bytes": 0})
+        r["ms"] += s.elapsed_time(e)
+        r["launches"] += 1
+        r["algo_bytes"] += wl.algo_bytes(kind, d, nnz_of.get(id(d)))
+    peak, peak_src = hbm_peak()
+    step_kernel_ms = sum(r["ms"] for r in per.values())
+    kernels = {}
+    for kind, r in sorted(per.items()):
+        gbs = r["algo_bytes"] / (r["ms"] * 1e-3) / 1e9 if r["ms"] > 0 else 0.0
+        kernels[kind] = {"ms_per_step": round(r["ms"] / args.steps, 4), "share": round(r["ms"] / step_kernel_ms, 4),
+                         "launches_per_step": r["launches"] // args.steps, "algo_GBps": round(gbs, 1),
+                         "frac_hbm": round(gbs / peak, 4)}
+    dom = max(per, key=lambda kk: per[kk]["ms"])
+    dom_gbs = per[dom]["algo_bytes"] / (per[dom]["ms"] * 1e-3) / 1e9
+
+    # ---- multi-rank: max time over ranks, sum of bytes (NCCL, outside the timed region)
+    total_bytes = wl.bytes_per_step * args.steps
+    if dist is not None:
+        t = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        elapsed_ms = float(t.item())
+        tally = torch.tensor([total_bytes, sum(nnz)], dtype=torch.int64, device=dev)
+        dist.all_reduce(tally, op=dist.ReduceOp.SUM)
+        total_bytes = int(tally[0].item())
+    value = total_bytes / (elapsed_ms * 1e-3) / 1e9
+
+    # ---- e2e: host pinned inputs -> H2D -> the same C-ABI calls -> D2H of the nnz tally
+    e2e = None
+    if not args.no_e2e:
+        hosts = [(d, d["y"].cpu().pin_memory(), d["dY"].cpu().pin_memory() if "dY" in d else None) for d in wl.sites]
+        h2d = sum(h.numel() * 4 + (g.numel() * 4 if g is not None else 0) for _, h, g in hosts)
+        d2h = wl.nnz_all.numel() * 8
+        out_host = torch.empty_like(wl.nnz_all, device="cpu").pin_memory()
+        e_steps = max(3, min(args.steps, 10))
+
+        def e2e_step():
+            for d, h, g in hosts:
+                d["y"].copy_(h, non_blocking=True)
+                if g is not None:
+                    d["dY"].copy_(g, non_blocking=True)
+            wl.step()
+            out_host.copy_(wl.nnz_all, non_blocking=True)
+
+        e2e_step()
+        barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(e_steps):
+            e2e_step()
+        b.record(stream)
+        barrier()
+        e_ms = a.elapsed_time(b)
+        e_bytes = wl.bytes_per_step * e_steps
+        if dist is not None:
+            t = torch.tensor([e_ms], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e_ms = float(t.item())
+            e_bytes *= world
+        e2e = {"value": round(e_bytes / (e_ms * 1e-3) / 1e9, 3), "unit": "GB/s", "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h, "steps": e_steps,
+               "note": "pinned host maps copied H2D each step, then the step's C-ABI calls, then D2H of the "
+                       "per-site nnz tally"}
+
+    if rank != 0:
+        if dist is not None:
+            dist.destroy_process_group()
+        return
+
+    cpu = cpu_baseline(cfg, args.sparsity, args.dpr_bits, args.cpu_seconds) if world == 1 else None
+    line = {
+        "metric": baseline_metric(), "value": round(value, 3), "unit": "GB/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(elapsed_ms / args.steps, 4),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": workload_config(args, cfg, batch),
+        "roofline": {"bound": "hbm", "kernel": dom, "achieved": round(dom_gbs, 1), "peak": peak, "unit": "GB/s",
+                     "frac": round(dom_gbs / peak, 4), "traffic": traffic_for(dom), "peak_source": peak_src},
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": launches,
+        "clocks": clocks.summary(),
+        "compression": wl.compression(nnz),
+        "kernels": kernels,
+        "stash_bytes_per_gpu": 4 * wl.stash_elems,
+    }
+    if args.kernels_out:
+        with open(args.kernels_out, "w") as f:
+            json.dump(kernels, f, indent=1)
+    print(json.dumps(line), flush=True)
+    if dist is not None:
+        dist.destroy_process_group()
+
+
+def traffic_for(kind):
+    """DRAM bytes per launch from the committed ncu --set full capture, if one exists."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        t = json.load(f)
+    return t.get(kind, {}).get("dram_bytes_per_launch")
+
+
+if __name__ == "__main__":
+    main()

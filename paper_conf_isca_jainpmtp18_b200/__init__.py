@@ -1,0 +1,249 @@
+"""Python binding of libgist — Gist's stash-time encode/decode hot path on B200 (sm_100a).
+
+Argument marshalling only: every function below validates nothing itself, allocates
+outputs with torch on the input's device when the caller passes none, and forwards raw
+device pointers plus torch's current CUDA stream to the same-named C-ABI call in
+``include/gist.h`` (ctypes).  All arithmetic runs in the CUDA kernels of ``csrc/``.
+There is no CPU fallback: importing this package without ``libgist.so`` raises, and a
+non-CUDA tensor is rejected.
+
+Paper: Jain et al., "Gist: Efficient Data Encoding for Deep Neural Network Training",
+ISCA 2018 (§IV-A, P:151-P:171).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import torch
+
+__all__ = [
+    "GistError", "Pool2d", "lib", "library_path",
+    "gist_binarize_words", "gist_argmax_words", "gist_pool2d_out_dims", "gist_ssdc_rows",
+    "gist_ssdc_bytes", "gist_ssdc_workspace_bytes", "gist_dpr_words", "gist_num_sms", "gist_launch_count",
+    "gist_binarize_encode", "gist_maxpool_fwd_argmax", "gist_pool_relu_bwd",
+    "gist_ssdc_encode", "gist_ssdc_decode", "gist_dpr_encode", "gist_dpr_decode",
+]
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+library_path = os.path.join(_HERE, "libgist.so")
+
+STATUS = {0: "GIST_OK", 1: "GIST_ERR_INVALID_ARGUMENT", 2: "GIST_ERR_MISALIGNED",
+          3: "GIST_ERR_UNSUPPORTED", 4: "GIST_ERR_TOO_LARGE", 5: "GIST_ERR_CUDA"}
+
+
+class GistError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        super().__init__(f"{where}: {STATUS.get(status, status)}")
+
+
+class Pool2d(C.Structure):
+    """gist_pool2d: (kh, kw, sh, sw, ph, pw, ceil_mode), torch max_pool2d semantics."""
+    _fields_ = [(f, C.c_int32) for f in ("kh", "kw", "sh", "sw", "ph", "pw", "ceil_mode")]
+
+    @classmethod
+    def of(cls, g) -> "Pool2d":
+        if isinstance(g, Pool2d):
+            return g
+        return cls(*[int(v) for v in g])
+
+
+def _load() -> C.CDLL:
+    if not os.path.exists(library_path):
+        raise ImportError(
+            f"{library_path} is missing: build it with `python build_gist.py` "
+            "(there is no CPU fallback for the Gist kernels)")
+    L = C.CDLL(library_path)
+    i64, i32, p, sz = C.c_int64, C.c_int32, C.c_void_p, C.c_size_t
+    P = C.POINTER(Pool2d)
+    sigs = {
+        "gist_status_string": (C.c_char_p, [C.c_int]),
+        "gist_binarize_words": (i64, [i64]),
+        "gist_argmax_words": (i64, [i64]),
+        "gist_pool2d_out_dims": (C.c_int, [i32, i32, P, C.POINTER(i32), C.POINTER(i32)]),
+        "gist_ssdc_rows": (i64, [i64]),
+        "gist_ssdc_bytes": (i64, [i64, i64]),
+        "gist_ssdc_workspace_bytes": (sz, [i64]),
+        "gist_dpr_words": (i64, [i64, i32]),
+        "gist_num_sms": (i32, []),
+        "gist_launch_count": (C.c_uint64, []),
+        "gist_binarize_encode": (C.c_int, [p, i64, p, p]),
+        "gist_maxpool_fwd_argmax": (C.c_int, [p, i32, i32, i32, i32, P, p, p, p, p]),
+        "gist_pool_relu_bwd": (C.c_int, [p, p, p, i32, i32, i32, i32, P, p, p]),
+        "gist_ssdc_encode": (C.c_int, [p, i64, p, p, p, i64, p, p, sz, p]),
+        "gist_ssdc_decode": (C.c_int, [p, p, p, i64, p, p]),
+        "gist_dpr_encode": (C.c_int, [p, i64, i32, p, p]),
+        "gist_dpr_decode": (C.c_int, [p, i64, i32, p, p]),
+    }
+    for name, (res, args) in sigs.items():
+        fn = getattr(L, name)
+        fn.restype = res
+        fn.argtypes = args
+    return L
+
+
+lib = _load()
+
+
+# ------------------------------------------------------------------ marshalling helpers
+def _ptr(t: torch.Tensor | None):
+    if t is None:
+        return None
+    if not t.is_cuda:
+        raise ValueError("libgist takes CUDA tensors only (no CPU fallback)")
+    if not t.is_contiguous():
+        raise ValueError("libgist takes contiguous tensors")
+    return t.data_ptr()
+
+
+def _stream(t: torch.Tensor, stream=None):
+    s = stream if stream is not None else torch.cuda.current_stream(t.device)
+    return s.cuda_stream if hasattr(s, "cuda_stream") else s
+
+
+def _check(status: int, where: str):
+    if status != 0:
+        raise GistError(status, where)
+
+
+def _words(n: int, dev, out=None):
+    return out if out is not None else torch.empty(max(n, 0), dtype=torch.int32, device=dev)
+
+
+# ------------------------------------------------------------------ size helpers
+def gist_binarize_words(n: int) -> int:
+    return lib.gist_binarize_words(n)
+
+
+def gist_argmax_words(n_out: int) -> int:
+    return lib.gist_argmax_words(n_out)
+
+
+def gist_pool2d_out_dims(H: int, W: int, pool) -> tuple[int, int]:
+    Ho, Wo = C.c_int32(), C.c_int32()
+    _check(lib.gist_pool2d_out_dims(H, W, C.byref(Pool2d.of(pool)), C.byref(Ho), C.byref(Wo)),
+           "gist_pool2d_out_dims")
+    return Ho.value, Wo.value
+
+
+def gist_ssdc_rows(n: int) -> int:
+    return lib.gist_ssdc_rows(n)
+
+
+def gist_ssdc_bytes(n: int, nnz: int) -> int:
+    return lib.gist_ssdc_bytes(n, nnz)
+
+
+def gist_ssdc_workspace_bytes(n: int) -> int:
+    return lib.gist_ssdc_workspace_bytes(n)
+
+
+def gist_dpr_words(n: int, bits: int) -> int:
+    return lib.gist_dpr_words(n, bits)
+
+
+def gist_num_sms() -> int:
+    return lib.gist_num_sms()
+
+
+def gist_launch_count() -> int:
+    """Kernels libgist has enqueued so far in this process."""
+    return lib.gist_launch_count()
+
+
+# ------------------------------------------------------------------ a1..a7
+def gist_binarize_encode(y: torch.Tensor, mask: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """a1: 1-bit ReLU mask, int32 tensor of uint32 words (bit i = y[i] > 0)."""
+    n = y.numel()
+    mask = _words(gist_binarize_words(n), y.device, mask)
+    _check(lib.gist_binarize_encode(_ptr(y), n, _ptr(mask), _stream(y, stream)), "gist_binarize_encode")
+    return mask
+
+
+def gist_maxpool_fwd_argmax(y: torch.Tensor, pool, out=None, argmax=None, mask=None, fuse_mask=False,
+                            stream=None):
+    """a2: returns (out [N,C,Ho,Wo] fp32, argmax int32 words, mask or None).
+    fuse_mask=True (or a mask tensor) also writes the a1 mask of y."""
+    N, Cc, H, W = y.shape
+    g = Pool2d.of(pool)
+    Ho, Wo = gist_pool2d_out_dims(H, W, g)
+    if out is None:
+        out = torch.empty((N, Cc, Ho, Wo), dtype=torch.float32, device=y.device)
+    argmax = _words(gist_argmax_words(N * Cc * Ho * Wo), y.device, argmax)
+    if mask is None and fuse_mask:
+        mask = _words(gist_binarize_words(y.numel()), y.device)
+    _check(lib.gist_maxpool_fwd_argmax(_ptr(y), N, Cc, H, W, C.byref(g), _ptr(out), _ptr(argmax), _ptr(mask),
+                                       _stream(y, stream)), "gist_maxpool_fwd_argmax")
+    return out, argmax, mask
+
+
+def gist_pool_relu_bwd(dout: torch.Tensor, argmax: torch.Tensor, mask: torch.Tensor | None, shape, pool,
+                       dx: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """a3: dx [N,C,H,W] from dY, the 4-bit argmax map and the 1-bit mask."""
+    N, Cc, H, W = shape
+    if dx is None:
+        dx = torch.empty((N, Cc, H, W), dtype=torch.float32, device=dout.device)
+    _check(lib.gist_pool_relu_bwd(_ptr(dout), _ptr(argmax), _ptr(mask), N, Cc, H, W, C.byref(Pool2d.of(pool)),
+                                  _ptr(dx), _stream(dout, stream)), "gist_pool_relu_bwd")
+    return dx
+
+
+def gist_ssdc_encode(x: torch.Tensor, capacity: int | None = None, row_end=None, col=None, val=None, nnz=None,
+                     workspace=None, trim: bool = False, stream=None):
+    """a4 (P:158-P:164): returns (row_end int32[rows], col uint8[capacity], val fp32[capacity],
+    nnz int64[1] on device).  capacity defaults to n (always complete).  trim=True reads nnz
+    back (one D2H sync) and returns col/val views of exactly nnz entries."""
+    n = x.numel()
+    dev = x.device
+    cap = n if capacity is None else int(capacity)
+    if row_end is None:
+        row_end = torch.empty(gist_ssdc_rows(n), dtype=torch.int32, device=dev)
+    if col is None:
+        col = torch.empty(max(cap, 1), dtype=torch.uint8, device=dev)
+    if val is None:
+        val = torch.empty(max(cap, 1), dtype=torch.float32, device=dev)
+    if nnz is None:
+        nnz = torch.empty(1, dtype=torch.int64, device=dev)
+    wsb = gist_ssdc_workspace_bytes(n)
+    if workspace is None:
+        workspace = torch.empty(wsb, dtype=torch.uint8, device=dev)
+    _check(lib.gist_ssdc_encode(_ptr(x), n, _ptr(row_end), _ptr(col), _ptr(val), cap, _ptr(nnz),
+                                _ptr(workspace), workspace.numel() * workspace.element_size(), _stream(x, stream)),
+           "gist_ssdc_encode")
+    if trim:
+        k = int(nnz.item())
+        if k > cap:
+            raise GistError(4, f"gist_ssdc_encode: nnz {k} exceeds capacity {cap}")
+        return row_end, col[:k], val[:k], nnz
+    return row_end, col, val, nnz
+
+
+def gist_ssdc_decode(row_end: torch.Tensor, col: torch.Tensor, val: torch.Tensor, n: int,
+                     x: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """a5: dense fp32 [n] from the CSR encoding."""
+    if x is None:
+        x = torch.empty(n, dtype=torch.float32, device=row_end.device)
+    _check(lib.gist_ssdc_decode(_ptr(row_end), _ptr(col), _ptr(val), n, _ptr(x), _stream(row_end, stream)),
+           "gist_ssdc_decode")
+    return x
+
+
+def gist_dpr_encode(x: torch.Tensor, bits: int, packed: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """a6: fp32 -> FP16/FP10/FP8 codes packed 2/3/4 per 32-bit word (int32 tensor)."""
+    n = x.numel()
+    words = gist_dpr_words(n, bits)
+    if words < 0:
+        raise GistError(3, "gist_dpr_encode")
+    packed = _words(words, x.device, packed)
+    _check(lib.gist_dpr_encode(_ptr(x), n, bits, _ptr(packed), _stream(x, stream)), "gist_dpr_encode")
+    return packed
+
+
+def gist_dpr_decode(packed: torch.Tensor, n: int, bits: int, x: torch.Tensor | None = None,
+                    stream=None) -> torch.Tensor:
+    """a7: packed codes -> fp32 [n]."""
+    if x is None:
+        x = torch.empty(n, dtype=torch.float32, device=packed.device)
+    _check(lib.gist_dpr_decode(_ptr(packed), n, bits, _ptr(x), _stream(packed, stream)), "gist_dpr_decode")
+    return x

@@ -1,0 +1,51 @@
+// common.cuh — device helpers shared by the sm_100a kernels of libgist.
+// (Product side only; the CPU oracle under oracle/ shares nothing with this file.)
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace gist {
+
+constexpr int kWarp = 32;
+constexpr unsigned kFull = 0xffffffffu;
+
+// Streaming 128-bit load: the input feature map is read exactly once per call, so ask
+// L2 to evict it first (ld.global.cs) and keep the encodings resident instead.
+__device__ __forceinline__ float4 ld_stream_f4(const float4 *p) { return __ldcs(p); }
+__device__ __forceinline__ uint4 ld_stream_u4(const uint4 *p) { return __ldcs(p); }
+__device__ __forceinline__ uint2 ld_stream_u2(const uint2 *p) { return __ldcs(p); }
+__device__ __forceinline__ uint32_t ld_stream_u32(const uint32_t *p) { return __ldcs(p); }
+__device__ __forceinline__ float ld_stream_f32(const float *p) { return __ldcs(p); }
+__device__ __forceinline__ float2 ld_stream_f2(const float2 *p) { return __ldcs(p); }
+
+// Read-only path through L1 for data re-read by neighbouring threads (pool windows).
+template <typename T>
+__device__ __forceinline__ T ld_ro(const T *p) { return __ldg(p); }
+
+// Division by a runtime constant d (< 2^31) for numerators < 2^31: q = umulhi(n, mul) >> shr
+// (round-up reciprocal, Granlund-Montgomery).  Host builds it once per launch.
+struct FastDiv {
+    uint32_t d, mul, shr;
+    __host__ static FastDiv make(uint32_t d_) {
+        FastDiv f{d_, 0u, 0u};
+        if (d_ > 1) {
+            uint32_t l = 0;
+            while ((1ull << l) < d_) ++l;  // ceil(log2 d)
+            uint32_t p = 31 + l;
+            f.mul = (uint32_t)(((1ull << p) + d_ - 1) / d_);
+            f.shr = p - 32;
+        }
+        return f;
+    }
+    __device__ __forceinline__ uint32_t div(uint32_t n) const {
+        return d == 1 ? n : (__umulhi(n, mul) >> shr);
+    }
+    __device__ __forceinline__ void divmod(uint32_t n, uint32_t &q, uint32_t &r) const {
+        q = div(n);
+        r = n - q * d;
+    }
+};
+
+__host__ __device__ __forceinline__ int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+}  // namespace gist

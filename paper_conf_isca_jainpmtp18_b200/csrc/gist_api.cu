@@ -1,0 +1,215 @@
+// gist_api.cu — the C ABI (include/gist.h): host-side validation, size helpers, dispatch
+// to the sm_100a kernels.  Stateless apart from the cached SM count.
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <mutex>
+
+#include "../../include/gist.h"
+#include "kernels.h"
+
+namespace gist {
+
+static std::atomic<uint64_t> g_launches{0};
+void count_launches(int k) { g_launches.fetch_add((uint64_t)k, std::memory_order_relaxed); }
+
+int num_sms() {
+    static std::once_flag once;
+    static int sms = 148;
+    std::call_once(once, [] {
+        int dev = 0, v = 0;
+        if (cudaGetDevice(&dev) == cudaSuccess &&
+            cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && v > 0)
+            sms = v;
+    });
+    return sms;
+}
+
+}  // namespace gist
+
+namespace {
+
+constexpr int64_t kI32Limit = (int64_t)1 << 31;
+
+bool misaligned(const void *p) { return p != nullptr && (reinterpret_cast<uintptr_t>(p) & 15u) != 0; }
+
+struct Range {
+    const void *p;
+    int64_t bytes;
+};
+
+bool overlap(Range a, Range b) {
+    if (!a.p || !b.p || a.bytes <= 0 || b.bytes <= 0) return false;
+    const uintptr_t a0 = reinterpret_cast<uintptr_t>(a.p), b0 = reinterpret_cast<uintptr_t>(b.p);
+    return a0 < b0 + (uintptr_t)b.bytes && b0 < a0 + (uintptr_t)a.bytes;
+}
+
+bool any_overlap(std::initializer_list<Range> ins, std::initializer_list<Range> outs) {
+    for (const Range &o : outs) {
+        for (const Range &i : ins)
+            if (overlap(i, o)) return true;
+    }
+    for (auto o1 = outs.begin(); o1 != outs.end(); ++o1)
+        for (auto o2 = o1 + 1; o2 != outs.end(); ++o2)
+            if (overlap(*o1, *o2)) return true;
+    return false;
+}
+
+gist_status launched(cudaError_t e, int kernels) {
+    if (e != cudaSuccess) return GIST_ERR_CUDA;
+    gist::count_launches(kernels);
+    return GIST_OK;
+}
+
+int32_t pool_dim(int32_t in, int32_t k, int32_t s, int32_t p, int32_t ceil_mode) {
+    const int32_t span = in + 2 * p - k;
+    if (span < 0) return 0;
+    int32_t out = ceil_mode ? (span + s - 1) / s + 1 : span / s + 1;
+    if (ceil_mode && (int64_t)(out - 1) * s >= (int64_t)in + p) out -= 1;
+    return out;
+}
+
+gist_status check_pool(int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d *p, int32_t *Ho, int32_t *Wo) {
+    if (!p || N < 0 || C < 0 || H < 0 || W < 0) return GIST_ERR_INVALID_ARGUMENT;
+    if (p->kh < 1 || p->kw < 1 || p->sh < 1 || p->sw < 1 || p->ph < 0 || p->pw < 0 || p->ph > p->kh / 2 ||
+        p->pw > p->kw / 2)
+        return GIST_ERR_INVALID_ARGUMENT;
+    if (p->kh * p->kw > 16) return GIST_ERR_UNSUPPORTED;  // argmax must fit 4 bits
+    *Ho = pool_dim(H, p->kh, p->sh, p->ph, p->ceil_mode);
+    *Wo = pool_dim(W, p->kw, p->sw, p->pw, p->ceil_mode);
+    if ((H > 0 && *Ho < 1) || (W > 0 && *Wo < 1)) return GIST_ERR_INVALID_ARGUMENT;
+    return GIST_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *gist_status_string(gist_status s) {
+    switch (s) {
+        case GIST_OK: return "GIST_OK";
+        case GIST_ERR_INVALID_ARGUMENT: return "GIST_ERR_INVALID_ARGUMENT";
+        case GIST_ERR_MISALIGNED: return "GIST_ERR_MISALIGNED";
+        case GIST_ERR_UNSUPPORTED: return "GIST_ERR_UNSUPPORTED";
+        case GIST_ERR_TOO_LARGE: return "GIST_ERR_TOO_LARGE";
+        case GIST_ERR_CUDA: return "GIST_ERR_CUDA";
+    }
+    return "GIST_ERR_UNKNOWN";
+}
+
+int64_t gist_binarize_words(int64_t n) { return n < 0 ? -1 : (n + 31) / 32; }
+int64_t gist_argmax_words(int64_t n_out) { return n_out < 0 ? -1 : (n_out + 7) / 8; }
+int64_t gist_ssdc_rows(int64_t n) { return n < 0 ? -1 : (n + 255) / 256; }
+int64_t gist_ssdc_bytes(int64_t n, int64_t nnz) { return n < 0 || nnz < 0 ? -1 : 5 * nnz + 4 * gist_ssdc_rows(n); }
+size_t gist_ssdc_workspace_bytes(int64_t n) { return gist::ssdc_workspace_bytes(n < 0 ? 0 : n); }
+int64_t gist_dpr_words(int64_t n, int32_t bits) {
+    const int k = bits == 16 ? 2 : bits == 10 ? 3 : bits == 8 ? 4 : 0;
+    if (!k || n < 0) return -1;
+    return (n + k - 1) / k;
+}
+int32_t gist_num_sms(void) { return gist::num_sms(); }
+uint64_t gist_launch_count(void) { return gist::g_launches.load(std::memory_order_relaxed); }
+
+gist_status gist_pool2d_out_dims(int32_t H, int32_t W, const gist_pool2d *p, int32_t *Ho, int32_t *Wo) {
+    if (!Ho || !Wo) return GIST_ERR_INVALID_ARGUMENT;
+    return check_pool(1, 1, H, W, p, Ho, Wo);
+}
+
+gist_status gist_binarize_encode(const float *y, int64_t n, uint32_t *mask, cudaStream_t stream) {
+    if (n < 0) return GIST_ERR_INVALID_ARGUMENT;
+    if (n == 0) return GIST_OK;
+    if (!y || !mask) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(y) || misaligned(mask)) return GIST_ERR_MISALIGNED;
+    if (any_overlap({{y, 4 * n}}, {{mask, 4 * gist_binarize_words(n)}})) return GIST_ERR_INVALID_ARGUMENT;
+    return launched(gist::launch_binarize(y, n, mask, stream), 1);
+}
+
+gist_status gist_maxpool_fwd_argmax(const float *y, int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d *p,
+                                    float *out, uint32_t *argmax, uint32_t *mask, cudaStream_t stream) {
+    int32_t Ho = 0, Wo = 0;
+    const gist_status st = check_pool(N, C, H, W, p, &Ho, &Wo);
+    if (st != GIST_OK) return st;
+    const int64_t n = (int64_t)N * C * H * W, n_out = (int64_t)N * C * Ho * Wo;
+    if (n == 0) return GIST_OK;
+    if (!y || !out || !argmax) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(y) || misaligned(out) || misaligned(argmax) || misaligned(mask)) return GIST_ERR_MISALIGNED;
+    if (n >= kI32Limit || n_out >= kI32Limit) return GIST_ERR_TOO_LARGE;
+    if (any_overlap({{y, 4 * n}},
+                    {{out, 4 * n_out}, {argmax, 4 * gist_argmax_words(n_out)}, {mask, mask ? 4 * gist_binarize_words(n) : 0}}))
+        return GIST_ERR_INVALID_ARGUMENT;
+    cudaError_t e = gist::launch_maxpool_fwd(y, N, C, H, W, *p, Ho, Wo, out, argmax, stream);
+    if (e == cudaSuccess && mask) e = gist::launch_binarize(y, n, mask, stream);
+    return launched(e, mask ? 2 : 1);
+}
+
+gist_status gist_pool_relu_bwd(const float *dout, const uint32_t *argmax, const uint32_t *mask, int32_t N, int32_t C,
+                               int32_t H, int32_t W, const gist_pool2d *p, float *dx, cudaStream_t stream) {
+    int32_t Ho = 0, Wo = 0;
+    const gist_status st = check_pool(N, C, H, W, p, &Ho, &Wo);
+    if (st != GIST_OK) return st;
+    const int64_t n = (int64_t)N * C * H * W, n_out = (int64_t)N * C * Ho * Wo;
+    if (n == 0) return GIST_OK;
+    if (!dout || !argmax || !dx) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(dout) || misaligned(argmax) || misaligned(mask) || misaligned(dx)) return GIST_ERR_MISALIGNED;
+    if (n >= kI32Limit || n_out >= kI32Limit) return GIST_ERR_TOO_LARGE;
+    if (any_overlap({{dout, 4 * n_out}, {argmax, 4 * gist_argmax_words(n_out)}, {mask, mask ? 4 * gist_binarize_words(n) : 0}},
+                    {{dx, 4 * n}}))
+        return GIST_ERR_INVALID_ARGUMENT;
+    return launched(gist::launch_pool_bwd(dout, argmax, mask, N, C, H, W, *p, Ho, Wo, dx, stream), 1);
+}
+
+gist_status gist_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val, int64_t capacity,
+                             int64_t *nnz, void *workspace, size_t workspace_bytes, cudaStream_t stream) {
+    if (n < 0 || capacity < 0) return GIST_ERR_INVALID_ARGUMENT;
+    if (n >= kI32Limit) return GIST_ERR_TOO_LARGE;
+    if (!nnz) return GIST_ERR_INVALID_ARGUMENT;
+    if (n > 0 && (!x || !row_end || !workspace)) return GIST_ERR_INVALID_ARGUMENT;
+    if (capacity > 0 && (!col || !val)) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(x) || misaligned(row_end) || misaligned(col) || misaligned(val) || misaligned(workspace) ||
+        (reinterpret_cast<uintptr_t>(nnz) & 7u))
+        return GIST_ERR_MISALIGNED;
+    if (n > 0 && workspace_bytes < gist_ssdc_workspace_bytes(n)) return GIST_ERR_INVALID_ARGUMENT;
+    const int64_t cap = capacity < n ? capacity : n;
+    if (any_overlap({{x, 4 * n}}, {{row_end, 4 * gist_ssdc_rows(n)}, {col, cap}, {val, 4 * cap}, {nnz, 8},
+                                   {workspace, (int64_t)workspace_bytes}}))
+        return GIST_ERR_INVALID_ARGUMENT;
+    if (n == 0) {  // still publish nnz = 0 (stream-ordered)
+        return cudaMemsetAsync(nnz, 0, sizeof(int64_t), stream) == cudaSuccess ? GIST_OK : GIST_ERR_CUDA;
+    }
+    return launched(gist::launch_ssdc_encode(x, n, row_end, col, val, capacity, nnz, workspace, stream), 2);
+}
+
+gist_status gist_ssdc_decode(const int32_t *row_end, const uint8_t *col, const float *val, int64_t n, float *x,
+                             cudaStream_t stream) {
+    if (n < 0) return GIST_ERR_INVALID_ARGUMENT;
+    if (n >= kI32Limit) return GIST_ERR_TOO_LARGE;
+    if (n == 0) return GIST_OK;
+    if (!row_end || !x) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(row_end) || misaligned(col) || misaligned(val) || misaligned(x)) return GIST_ERR_MISALIGNED;
+    if (any_overlap({{row_end, 4 * gist_ssdc_rows(n)}}, {{x, 4 * n}})) return GIST_ERR_INVALID_ARGUMENT;
+    // col/val extents are only known on the device (row_end[rows-1]); they may be NULL only
+    // for an all-zero map, which the kernel then never dereferences.
+    return launched(gist::launch_ssdc_decode(row_end, col, val, n, x, stream), 1);
+}
+
+gist_status gist_dpr_encode(const float *x, int64_t n, int32_t bits, uint32_t *packed, cudaStream_t stream) {
+    if (bits != 8 && bits != 10 && bits != 16) return GIST_ERR_UNSUPPORTED;
+    if (n < 0) return GIST_ERR_INVALID_ARGUMENT;
+    if (n == 0) return GIST_OK;
+    if (!x || !packed) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(x) || misaligned(packed)) return GIST_ERR_MISALIGNED;
+    if (any_overlap({{x, 4 * n}}, {{packed, 4 * gist_dpr_words(n, bits)}})) return GIST_ERR_INVALID_ARGUMENT;
+    return launched(gist::launch_dpr_encode(x, n, bits, packed, stream), 1);
+}
+
+gist_status gist_dpr_decode(const uint32_t *packed, int64_t n, int32_t bits, float *x, cudaStream_t stream) {
+    if (bits != 8 && bits != 10 && bits != 16) return GIST_ERR_UNSUPPORTED;
+    if (n < 0) return GIST_ERR_INVALID_ARGUMENT;
+    if (n == 0) return GIST_OK;
+    if (!x || !packed) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(x) || misaligned(packed)) return GIST_ERR_MISALIGNED;
+    if (any_overlap({{packed, 4 * gist_dpr_words(n, bits)}}, {{x, 4 * n}})) return GIST_ERR_INVALID_ARGUMENT;
+    return launched(gist::launch_dpr_decode(packed, n, bits, x, stream), 1);
+}
+
+}  // extern "C"

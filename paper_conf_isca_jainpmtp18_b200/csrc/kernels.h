@@ -1,0 +1,28 @@
+// kernels.h — internal launchers behind the C ABI (include/gist.h).  Each returns the
+// launch status; argument validation happens in gist_api.cu before these are called.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/gist.h"
+
+namespace gist {
+
+int num_sms();
+void count_launches(int k);  // bookkeeping for gist_launch_count()
+
+cudaError_t launch_binarize(const float *y, int64_t n, uint32_t *mask, cudaStream_t s);
+cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p,
+                               int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, cudaStream_t s);
+cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uint32_t *mask, int32_t N, int32_t C,
+                            int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo, float *dx,
+                            cudaStream_t s);
+size_t ssdc_workspace_bytes(int64_t n);
+cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val,
+                               int64_t capacity, int64_t *nnz, void *workspace, cudaStream_t s);
+cudaError_t launch_ssdc_decode(const int32_t *row_end, const uint8_t *col, const float *val, int64_t n, float *x,
+                               cudaStream_t s);
+cudaError_t launch_dpr_encode(const float *x, int64_t n, int bits, uint32_t *packed, cudaStream_t s);
+cudaError_t launch_dpr_decode(const uint32_t *packed, int64_t n, int bits, float *x, cudaStream_t s);
+
+}  // namespace gist

@@ -1,0 +1,251 @@
+// pool.cu — a2: MaxPool forward + 4-bit Y->X argmax map, a3: fused pool+ReLU backward from
+// the encodings (§III-A, P:151-P:156 §IV-A).
+//
+// Forward: one thread per pool output; a warp covers 32 consecutive outputs (4 argmax
+// words), ORs the nibbles of each 8-lane group with three xor-shuffles and lane 8g stores
+// word g.  Windows are read through L1 (__ldg): neighbouring outputs share input rows.
+// The 2x2/s2 unpadded case (VGG16, OverFeat) reads each window row as one aligned float2.
+//
+// Backward: gather form — one thread per input element (2 adjacent elements for 2x2/s2)
+// walks the covering windows in ascending output order, adds dY of every window whose
+// argmax is this element (accumulator starts at +0.0f: reading R6), and selects with the
+// ReLU mask bit (R7).  Every dx element is written exactly once with no atomics, so the
+// result is deterministic and equal to the oracle's ascending-o scatter.
+#include <math_constants.h>
+
+#include "common.cuh"
+#include "kernels.h"
+
+namespace gist {
+
+namespace {
+
+constexpr int kPoolThreads = 256;
+
+struct PoolArgs {
+    int32_t H, W, Ho, Wo;
+    int32_t kh, kw, sh, sw, ph, pw;
+    int32_t n_out;  // N*C*Ho*Wo
+    int32_t n_in;   // N*C*H*W
+    FastDiv div_wo, div_ho, div_w, div_h;
+};
+
+__device__ __forceinline__ void take(float v, int idx, float &best, int &bi) {
+    if (v > best || v != v) {  // R3: strict '>' keeps the first maximum; NaN always wins
+        best = v;
+        bi = idx;
+    }
+}
+
+// KH/KW > 0: compile-time window; 0: runtime (a.kh, a.kw).
+template <int KH, int KW>
+__global__ void __launch_bounds__(kPoolThreads)
+maxpool_fwd_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ out, uint32_t *__restrict__ arg) {
+    const int kh = KH ? KH : a.kh, kw = KW ? KW : a.kw;
+    const int lane = threadIdx.x & 31;
+    const int64_t chunks = ((int64_t)a.n_out + 31) / 32;
+    const int64_t nwarps = ((int64_t)gridDim.x * kPoolThreads) >> 5;
+    for (int64_t c = ((int64_t)blockIdx.x * kPoolThreads + threadIdx.x) >> 5; c < chunks; c += nwarps) {
+        const int64_t o = c * 32 + lane;
+        uint32_t nib = 0;
+        if (o < a.n_out) {
+            uint32_t q, ow, nc, oh;
+            a.div_wo.divmod((uint32_t)o, q, ow);
+            a.div_ho.divmod(q, nc, oh);
+            const int h0 = (int)oh * a.sh - a.ph, w0 = (int)ow * a.sw - a.pw;
+            const float *plane = y + (int64_t)nc * a.H * a.W;
+            float best = -CUDART_INF_F;
+            int bi = -1;
+            for (int dy = 0; dy < kh; ++dy) {
+                const int ih = h0 + dy;
+                if (ih < 0 || ih >= a.H) continue;
+                for (int dx = 0; dx < kw; ++dx) {
+                    const int iw = w0 + dx;
+                    if (iw < 0 || iw >= a.W) continue;
+                    const float v = ld_ro(plane + ih * a.W + iw);
+                    if (bi < 0) bi = dy * kw + dx;  // first in-bounds position (all -inf case)
+                    take(v, dy * kw + dx, best, bi);
+                }
+            }
+            out[o] = best;
+            nib = (uint32_t)bi << (4 * (lane & 7));
+        }
+        nib |= __shfl_xor_sync(kFull, nib, 1);
+        nib |= __shfl_xor_sync(kFull, nib, 2);
+        nib |= __shfl_xor_sync(kFull, nib, 4);
+        if ((lane & 7) == 0 && o < a.n_out) arg[o >> 3] = nib;
+    }
+}
+
+// 2x2 stride 2, no padding, every window fully inside (W even): two float2 row loads.
+__global__ void __launch_bounds__(kPoolThreads)
+maxpool_fwd_k2s2_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ out,
+                        uint32_t *__restrict__ arg) {
+    const int lane = threadIdx.x & 31;
+    const int64_t chunks = ((int64_t)a.n_out + 31) / 32;
+    const int64_t nwarps = ((int64_t)gridDim.x * kPoolThreads) >> 5;
+    for (int64_t c = ((int64_t)blockIdx.x * kPoolThreads + threadIdx.x) >> 5; c < chunks; c += nwarps) {
+        const int64_t o = c * 32 + lane;
+        uint32_t nib = 0;
+        if (o < a.n_out) {
+            uint32_t q, ow, nc, oh;
+            a.div_wo.divmod((uint32_t)o, q, ow);
+            a.div_ho.divmod(q, nc, oh);
+            const float *p = y + (int64_t)nc * a.H * a.W + (int64_t)(2 * oh) * a.W + 2 * ow;
+            const float2 r0 = ld_stream_f2(reinterpret_cast<const float2 *>(p));
+            const float2 r1 = ld_stream_f2(reinterpret_cast<const float2 *>(p + a.W));
+            float best = -CUDART_INF_F;
+            int bi = 0;
+            take(r0.x, 0, best, bi);
+            take(r0.y, 1, best, bi);
+            take(r1.x, 2, best, bi);
+            take(r1.y, 3, best, bi);
+            out[o] = best;
+            nib = (uint32_t)bi << (4 * (lane & 7));
+        }
+        nib |= __shfl_xor_sync(kFull, nib, 1);
+        nib |= __shfl_xor_sync(kFull, nib, 2);
+        nib |= __shfl_xor_sync(kFull, nib, 4);
+        if ((lane & 7) == 0 && o < a.n_out) arg[o >> 3] = nib;
+    }
+}
+
+__device__ __forceinline__ uint32_t nibble(const uint32_t *__restrict__ arg, int64_t o) {
+    return (ld_ro(arg + (o >> 3)) >> (4 * (o & 7))) & 0xfu;
+}
+
+__device__ __forceinline__ bool mask_bit(const uint32_t *__restrict__ mask, int64_t i) {
+    return (ld_ro(mask + (i >> 5)) >> (i & 31)) & 1u;
+}
+
+// Generic gather backward: one thread per input element.
+template <int KH, int KW, int SH, int SW>
+__global__ void __launch_bounds__(kPoolThreads)
+pool_bwd_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg, const uint32_t *__restrict__ mask,
+                PoolArgs a, float *__restrict__ dx) {
+    const int kh = KH ? KH : a.kh, kw = KW ? KW : a.kw;
+    const int sh = SH ? SH : a.sh, sw = SW ? SW : a.sw;
+    const int64_t stride = (int64_t)gridDim.x * kPoolThreads;
+    for (int64_t i = (int64_t)blockIdx.x * kPoolThreads + threadIdx.x; i < a.n_in; i += stride) {
+        uint32_t q, iw, nc, ih;
+        a.div_w.divmod((uint32_t)i, q, iw);
+        a.div_h.divmod(q, nc, ih);
+        float acc = 0.0f;
+        if (mask == nullptr || mask_bit(mask, i)) {
+            const int th = (int)ih + a.ph, tw = (int)iw + a.pw;
+            const int oh_lo = th - kh + 1 > 0 ? (th - kh + 1 + sh - 1) / sh : 0;
+            const int oh_hi = min(a.Ho - 1, th / sh);
+            const int ow_lo = tw - kw + 1 > 0 ? (tw - kw + 1 + sw - 1) / sw : 0;
+            const int ow_hi = min(a.Wo - 1, tw / sw);
+            const int64_t obase = (int64_t)nc * a.Ho;
+            for (int oh = oh_lo; oh <= oh_hi; ++oh) {
+                const int ly = th - oh * sh;  // = ih - (oh*sh - ph)
+                for (int ow = ow_lo; ow <= ow_hi; ++ow) {
+                    const int64_t o = (obase + oh) * a.Wo + ow;
+                    if (nibble(arg, o) == (uint32_t)(ly * kw + (tw - ow * sw))) acc = acc + ld_ro(dout + o);
+                }
+            }
+        }
+        dx[i] = acc;
+    }
+}
+
+// 2x2 stride 2, no padding, W even: one thread per pair of adjacent inputs (same window).
+__global__ void __launch_bounds__(kPoolThreads)
+pool_bwd_k2s2_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
+                     const uint32_t *__restrict__ mask, PoolArgs a, float *__restrict__ dx) {
+    const int64_t pairs = (int64_t)a.n_in / 2;
+    const int64_t stride = (int64_t)gridDim.x * kPoolThreads;
+    for (int64_t p = (int64_t)blockIdx.x * kPoolThreads + threadIdx.x; p < pairs; p += stride) {
+        const int64_t i = 2 * p;
+        uint32_t q, iw, nc, ih;
+        a.div_w.divmod((uint32_t)i, q, iw);
+        a.div_h.divmod(q, nc, ih);
+        const uint32_t oh = ih >> 1, ow = iw >> 1;
+        float2 r = make_float2(0.0f, 0.0f);
+        if ((int)oh < a.Ho) {
+            const int64_t o = ((int64_t)nc * a.Ho + oh) * a.Wo + ow;
+            const uint32_t nib = nibble(arg, o);
+            const uint32_t m = mask ? (ld_ro(mask + (i >> 5)) >> (i & 31)) : 3u;
+            const uint32_t l0 = (ih & 1u) * 2u;
+            if ((nib == l0 && (m & 1u)) || (nib == l0 + 1 && (m & 2u))) {
+                const float g = 0.0f + ld_ro(dout + o);
+                r.x = (nib == l0 && (m & 1u)) ? g : 0.0f;
+                r.y = (nib == l0 + 1 && (m & 2u)) ? g : 0.0f;
+            }
+        }
+        reinterpret_cast<float2 *>(dx)[p] = r;
+    }
+}
+
+PoolArgs make_args(int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo) {
+    PoolArgs a;
+    a.H = H;
+    a.W = W;
+    a.Ho = Ho;
+    a.Wo = Wo;
+    a.kh = p.kh;
+    a.kw = p.kw;
+    a.sh = p.sh;
+    a.sw = p.sw;
+    a.ph = p.ph;
+    a.pw = p.pw;
+    a.n_out = (int32_t)((int64_t)N * C * Ho * Wo);
+    a.n_in = (int32_t)((int64_t)N * C * H * W);
+    a.div_wo = FastDiv::make((uint32_t)Wo);
+    a.div_ho = FastDiv::make((uint32_t)Ho);
+    a.div_w = FastDiv::make((uint32_t)W);
+    a.div_h = FastDiv::make((uint32_t)H);
+    return a;
+}
+
+bool is_k2s2_exact(const gist_pool2d &p, int32_t H, int32_t W, int32_t Ho, int32_t Wo) {
+    // every window fully inside: 2x2/s2/p0 with 2*Ho <= H and 2*Wo == W (W even)
+    return p.kh == 2 && p.kw == 2 && p.sh == 2 && p.sw == 2 && p.ph == 0 && p.pw == 0 && (W % 2 == 0) &&
+           2 * Ho <= H && 2 * Wo == W;
+}
+
+unsigned grid_for(int64_t work_items, int64_t items_per_block, int per_sm) {
+    int64_t blocks = ceil_div(work_items, items_per_block);
+    const int64_t cap = (int64_t)num_sms() * per_sm;
+    if (blocks > cap) blocks = cap;
+    if (blocks < 1) blocks = 1;
+    return (unsigned)blocks;
+}
+
+}  // namespace
+
+cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p,
+                               int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, cudaStream_t s) {
+    const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
+    const unsigned grid = grid_for(a.n_out, kPoolThreads, 8);
+    if (is_k2s2_exact(p, H, W, Ho, Wo))
+        maxpool_fwd_k2s2_kernel<<<grid, kPoolThreads, 0, s>>>(y, a, out, argmax);
+    else if (p.kh == 3 && p.kw == 3)
+        maxpool_fwd_kernel<3, 3><<<grid, kPoolThreads, 0, s>>>(y, a, out, argmax);
+    else if (p.kh == 2 && p.kw == 2)
+        maxpool_fwd_kernel<2, 2><<<grid, kPoolThreads, 0, s>>>(y, a, out, argmax);
+    else
+        maxpool_fwd_kernel<0, 0><<<grid, kPoolThreads, 0, s>>>(y, a, out, argmax);
+    return cudaPeekAtLastError();
+}
+
+cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uint32_t *mask, int32_t N, int32_t C,
+                            int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo, float *dx,
+                            cudaStream_t s) {
+    const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
+    if (is_k2s2_exact(p, H, W, Ho, Wo)) {
+        pool_bwd_k2s2_kernel<<<grid_for(a.n_in / 2, kPoolThreads, 8), kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+    } else {
+        const unsigned grid = grid_for(a.n_in, kPoolThreads, 8);
+        if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2)
+            pool_bwd_kernel<3, 3, 2, 2><<<grid, kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+        else if (p.kh == 3 && p.kw == 3 && p.sh == 1 && p.sw == 1)
+            pool_bwd_kernel<3, 3, 1, 1><<<grid, kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+        else
+            pool_bwd_kernel<0, 0, 0, 0><<<grid, kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+    }
+    return cudaPeekAtLastError();
+}
+
+}  // namespace gist

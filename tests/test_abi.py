@@ -1,0 +1,112 @@
+"""CPU-only checks of the C-ABI boundary: libgist.so loads, exports every symbol that
+include/gist.h declares, its host size helpers follow the closed forms, and its
+synchronous argument validation returns the documented status codes without touching a
+GPU."""
+import ctypes as C
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def declared():
+    src = open(os.path.join(ROOT, "include", "gist.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(gist_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_header_declares_the_seven_calls():
+    names = declared()
+    for call in ["gist_binarize_encode", "gist_maxpool_fwd_argmax", "gist_pool_relu_bwd", "gist_ssdc_encode",
+                 "gist_ssdc_decode", "gist_dpr_encode", "gist_dpr_decode"]:
+        assert call in names
+
+
+def test_library_exports_every_declared_symbol(gist):
+    raw = C.CDLL(gist.library_path)
+    missing = [n for n in declared() if not hasattr(raw, n)]
+    assert not missing, missing
+
+
+def test_binding_names_match_abi(gist):
+    for n in declared():
+        if n != "gist_status_string":
+            assert callable(getattr(gist, n)), n
+
+
+def test_status_strings(gist):
+    for code, name in gist.STATUS.items():
+        assert gist.lib.gist_status_string(code).decode() == name
+
+
+def test_size_helpers(gist):
+    assert gist.gist_binarize_words(0) == 0
+    assert gist.gist_binarize_words(33) == 2
+    assert gist.gist_argmax_words(9) == 2
+    assert gist.gist_ssdc_rows(257) == 2
+    assert gist.gist_ssdc_bytes(512, 100) == 5 * 100 + 4 * 2
+    for bits, k in ((16, 2), (10, 3), (8, 4)):
+        assert gist.gist_dpr_words(10, bits) == -(-10 // k)
+    assert gist.gist_dpr_words(10, 12) == -1
+    assert gist.gist_ssdc_workspace_bytes(1 << 20) >= 8 + 8 * ((1 << 20) // 8192)
+    assert gist.gist_pool2d_out_dims(56, 56, (3, 3, 2, 2, 0, 0, 0)) == (27, 27)
+    assert gist.gist_pool2d_out_dims(54, 54, (3, 3, 2, 2, 0, 0, 1)) == (27, 27)  # NiN ceil
+    assert gist.gist_pool2d_out_dims(112, 112, (3, 3, 2, 2, 0, 0, 1)) == (56, 56)  # GoogLeNet
+    assert gist.gist_pool2d_out_dims(28, 28, (3, 3, 1, 1, 1, 1, 0)) == (28, 28)
+
+
+def test_pool_dims_match_oracle(gist, ref):
+    from pool_cases import GEOMS
+    for g in GEOMS:
+        for H in range(1, 40):
+            if H + 2 * g[4] < g[0]:
+                continue
+            Ho, _ = gist.gist_pool2d_out_dims(H, H + 2 * g[5] if H + 2 * g[5] >= g[1] else g[1], g)
+            assert Ho == ref.pool_out_dim(H, g[0], g[2], g[4], g[6])
+
+
+OK, INVALID, MISALIGNED, UNSUPPORTED, TOO_LARGE = 0, 1, 2, 3, 4
+A, B = 0x10000, 0x20000000  # fake, 16-byte aligned, non-overlapping device addresses
+
+
+def test_validation_without_gpu(gist):
+    L = gist.lib
+    P = gist.Pool2d
+    # n == 0 launches nothing
+    assert L.gist_binarize_encode(None, 0, None, None) == OK
+    assert L.gist_dpr_encode(None, 0, 16, None, None) == OK
+    assert L.gist_dpr_decode(None, 0, 8, None, None) == OK
+    assert L.gist_ssdc_decode(None, None, None, 0, None, None) == OK
+    # NULL / negative
+    assert L.gist_binarize_encode(None, 10, B, None) == INVALID
+    assert L.gist_binarize_encode(A, -1, B, None) == INVALID
+    # misaligned
+    assert L.gist_binarize_encode(A + 4, 10, B, None) == MISALIGNED
+    assert L.gist_dpr_encode(A, 10, 16, B + 8, None) == MISALIGNED
+    # overlap
+    assert L.gist_binarize_encode(A, 1000, A + 16, None) == INVALID
+    assert L.gist_dpr_decode(A, 1000, 16, A, None) == INVALID
+    # DPR widths (16, 10, 8 only)
+    for bits in (0, 4, 9, 12, 32):
+        assert L.gist_dpr_encode(A, 10, bits, B, None) == UNSUPPORTED
+        assert L.gist_dpr_decode(A, 10, bits, B, None) == UNSUPPORTED
+    # pooling geometry
+    g = P(5, 5, 1, 1, 0, 0, 0)  # 25 window positions do not fit 4 bits
+    assert L.gist_maxpool_fwd_argmax(A, 1, 1, 8, 8, C.byref(g), B, B + 4096, None, None) == UNSUPPORTED
+    g = P(3, 3, 2, 2, 2, 2, 0)  # padding > k/2
+    assert L.gist_maxpool_fwd_argmax(A, 1, 1, 8, 8, C.byref(g), B, B + 4096, None, None) == INVALID
+    g = P(3, 3, 0, 2, 0, 0, 0)  # zero stride
+    assert L.gist_pool_relu_bwd(A, B, None, 1, 1, 8, 8, C.byref(g), B + 4096, None) == INVALID
+    g = P(3, 3, 2, 2, 0, 0, 0)
+    assert L.gist_maxpool_fwd_argmax(A, 1, 1, 2, 2, C.byref(g), B, B + 4096, None, None) == INVALID  # Ho < 1
+    assert L.gist_maxpool_fwd_argmax(A, 1 << 16, 1 << 10, 64, 64, C.byref(g), B, B + 4096, None, None) == TOO_LARGE
+    # SSDC
+    n = 1 << 31
+    assert L.gist_ssdc_encode(A, n, B, None, None, 0, B + 64, B + 128, 1 << 20, None) == TOO_LARGE
+    assert L.gist_ssdc_decode(A, None, None, n, B, None) == TOO_LARGE
+    assert L.gist_ssdc_encode(A, 1024, B, None, None, 16, B + 4096, B + 8192, 4096, None) == INVALID  # cap w/o col
+    assert L.gist_ssdc_encode(A, 1 << 20, B, B + (1 << 24), B + (1 << 26), 1 << 20, B + (1 << 28), B + (1 << 29),
+                              8, None) == INVALID  # workspace too small
+    assert L.gist_ssdc_encode(A, 1024, B, None, None, 0, B + 4100, B + 8192, 4096, None) == MISALIGNED  # nnz

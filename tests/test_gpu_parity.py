@@ -1,0 +1,262 @@
+"""GPU parity: every CUDA kernel, called through the C ABI (Python binding), against the
+CPU oracle on the same seeded inputs — bit-exact (the north star's bar: encodings and
+recomputed gradients identical; no float reduction order differs, reading R6).
+
+Sizes span several tiles/warps with ragged tails; the full-size cases use BASELINE.json's
+configurations in the launch configuration bench.py times."""
+import numpy as np
+import pytest
+import torch
+
+import workloads as WL
+from pool_cases import GEOMS, gid
+
+pytestmark = pytest.mark.gpu
+
+
+def host(t):
+    return t.detach().cpu().numpy()
+
+
+def u32(a):
+    return np.ascontiguousarray(a).view(np.uint32)
+
+
+def assert_bits_equal(got, expect, what=""):
+    got, expect = np.ascontiguousarray(got), np.ascontiguousarray(expect)
+    assert got.shape == expect.shape, (what, got.shape, expect.shape)
+    g, e = got.view(np.uint8), expect.view(np.uint8)
+    if not np.array_equal(g, e):
+        bad = np.flatnonzero(got.reshape(-1).view(np.uint32 if got.itemsize == 4 else np.uint8)
+                             != expect.reshape(-1).view(np.uint32 if expect.itemsize == 4 else np.uint8))
+        raise AssertionError(f"{what}: {bad.size} mismatches, first at {bad[:8]}")
+
+
+def mixed_values(n, seed, device):
+    g = torch.Generator(device=device).manual_seed(seed)
+    x = torch.randn(n, generator=g, device=device)
+    r = torch.rand(n, generator=g, device=device)
+    x = torch.where(r < 0.3, torch.zeros_like(x), x)
+    x = torch.where((r >= 0.3) & (r < 0.35), torch.full_like(x, -0.0), x)
+    x = torch.where((r >= 0.35) & (r < 0.36), torch.full_like(x, float("nan")), x)
+    x = torch.where((r >= 0.36) & (r < 0.37), torch.full_like(x, float("inf")), x)
+    x = torch.where((r >= 0.37) & (r < 0.38), torch.full_like(x, -float("inf")), x)
+    return x
+
+
+RAGGED = [1, 7, 31, 32, 33, 255, 256, 257, 1000, 1023, 1024, 1025, 4097, 8191, 8192, 8193, 65537,
+          200_704, 1_000_003]
+
+
+# ------------------------------------------------------------------------ a1 Binarize
+@pytest.mark.parametrize("n", RAGGED)
+def test_binarize(gist, ref, cuda, n):
+    y = mixed_values(n, n, cuda)
+    got = gist.gist_binarize_encode(y)
+    torch.cuda.synchronize()
+    assert_bits_equal(host(got), ref.binarize_encode(host(y)), "mask")
+
+
+def test_binarize_offset_views_rejected(gist, cuda):
+    y = torch.zeros(1000, device=cuda)
+    with pytest.raises(gist.GistError):
+        gist.gist_binarize_encode(y[1:])  # 4-byte offset -> GIST_ERR_MISALIGNED
+
+
+# ------------------------------------------------------------------------ a2/a3 pooling
+def pool_case(shape, g, seed, cuda, ties=True):
+    y = WL.relu_map(shape, 0.5, seed, cuda)
+    if ties:  # quantize so windows hold exact ties; plant -inf / NaN / -0.0
+        y = torch.round(y * 2) / 2
+        r = torch.rand(shape, generator=torch.Generator(device=cuda).manual_seed(seed + 1), device=cuda)
+        y = torch.where(r < 0.01, torch.full_like(y, float("nan")), y)
+        y = torch.where((r >= 0.01) & (r < 0.03), torch.full_like(y, -float("inf")), y)
+        y = torch.where((r >= 0.03) & (r < 0.1), torch.full_like(y, -0.0), y)
+    return y
+
+
+SHAPES = [(1, 1, 5, 7), (2, 3, 13, 13), (1, 64, 56, 56), (2, 5, 27, 27), (1, 7, 14, 14), (3, 2, 55, 55),
+          (1, 3, 9, 16), (2, 4, 12, 24), (1, 1, 1, 1)]
+
+
+@pytest.mark.parametrize("g", GEOMS, ids=gid)
+@pytest.mark.parametrize("shape", SHAPES, ids=lambda s: "x".join(map(str, s)))
+def test_maxpool_fwd_and_fused_bwd(gist, ref, cuda, g, shape):
+    N, Cc, H, W = shape
+    if H + 2 * g[4] < g[0] or W + 2 * g[5] < g[1]:
+        pytest.skip("window larger than padded input")
+    y = pool_case(shape, g, sum(shape) + g[0], cuda)
+    out, arg, mask = gist.gist_maxpool_fwd_argmax(y, g, fuse_mask=True)
+    r_out, r_arg = ref.maxpool_fwd_argmax(host(y), g)
+    assert_bits_equal(host(out), r_out, "out")
+    assert_bits_equal(host(arg), r_arg, "argmax")
+    assert_bits_equal(host(mask), ref.binarize_encode(host(y)), "fused mask")
+    dout = WL.grad_map(tuple(out.shape), 7, cuda)
+    dout = torch.where(torch.rand_like(dout) < 0.05, torch.full_like(dout, -0.0), dout)
+    for m, rm in ((mask, ref.binarize_encode(host(y))), (None, None)):
+        dx = gist.gist_pool_relu_bwd(dout, arg, m, shape, g)
+        r_dx = ref.pool_relu_bwd(host(dout), r_arg, rm, shape, g)
+        assert_bits_equal(host(dx), r_dx, "dx" + (" (pool-only)" if m is None else ""))
+
+
+def test_fused_bwd_equals_torch_autograd_on_gpu_inputs(gist, cuda):
+    # Same chain as the CPU pin, but on the GPU kernels: relu -> max_pool2d (AlexNet 3x3/s2).
+    g = (3, 3, 2, 2, 0, 0, 0)
+    z = WL.grad_map((4, 16, 55, 55), 3, cuda)
+    y = torch.relu(z)
+    out, arg, mask = gist.gist_maxpool_fwd_argmax(y, g, fuse_mask=True)
+    dout = WL.grad_map(tuple(out.shape), 4, cuda)
+    dx = gist.gist_pool_relu_bwd(dout, arg, mask, y.shape, g)
+    zc = z.cpu().requires_grad_()
+    oc = torch.nn.functional.max_pool2d(torch.relu(zc), 3, 2)
+    oc.backward(dout.cpu())
+    assert_bits_equal(host(out), oc.detach().numpy(), "out vs torch")
+    assert_bits_equal(host(dx), zc.grad.numpy(), "dx vs torch autograd")
+
+
+# ------------------------------------------------------------------------ a4/a5 SSDC
+@pytest.mark.parametrize("n", RAGGED + [256 * 32 * 70 + 5])
+@pytest.mark.parametrize("s", [0.0, 0.5, 0.9, 1.0])
+def test_ssdc_round_trip(gist, ref, cuda, n, s):
+    x = WL.relu_map((n,), s, n, cuda, negative_zero=True) if s < 1 else torch.zeros(n, device=cuda)
+    row_end, col, val, nnz = gist.gist_ssdc_encode(x, trim=True)
+    r_row_end, r_col, r_val = ref.ssdc_encode(host(x))
+    assert int(nnz.item()) == r_col.size
+    assert_bits_equal(host(row_end), r_row_end, "row_end")
+    assert_bits_equal(host(col), r_col, "col")
+    assert_bits_equal(host(val), r_val, "val")
+    back = gist.gist_ssdc_decode(row_end, col, val, n)
+    assert_bits_equal(host(back), host(x), "decode(encode(x))")
+    assert_bits_equal(host(back), ref.ssdc_decode(r_row_end, r_col, r_val, n), "decode vs oracle")
+
+
+def test_ssdc_structured_sparsity(gist, ref, cuda):
+    x = WL.relu_map((2, 64, 56, 56), 0.8, 11, cuda, structured=True)
+    row_end, col, val, nnz = gist.gist_ssdc_encode(x, trim=True)
+    r_row_end, r_col, r_val = ref.ssdc_encode(host(x))
+    assert_bits_equal(host(row_end), r_row_end, "row_end")
+    assert_bits_equal(host(col), r_col, "col")
+    assert_bits_equal(host(val), r_val, "val")
+
+
+@pytest.mark.parametrize("cap_frac", [0.0, 0.3, 0.999])
+def test_ssdc_capacity(gist, ref, cuda, cap_frac):
+    n = 256 * 32 * 9 + 77
+    x = WL.relu_map((n,), 0.6, 5, cuda)
+    r_row_end, r_col, r_val = ref.ssdc_encode(host(x))
+    cap = int(cap_frac * r_col.size)
+    row_end, col, val, nnz = gist.gist_ssdc_encode(x, capacity=cap)
+    assert int(nnz.item()) == r_col.size  # true nnz always published
+    assert_bits_equal(host(row_end), r_row_end, "row_end")
+    if cap:
+        assert_bits_equal(host(col)[:cap], r_col[:cap], "col prefix")
+        assert_bits_equal(host(val)[:cap], r_val[:cap], "val prefix")
+
+
+def test_ssdc_repeated_calls_reuse_workspace(gist, ref, cuda):
+    n = 256 * 1000 + 3
+    ws = torch.empty(gist.gist_ssdc_workspace_bytes(n), dtype=torch.uint8, device=cuda)
+    for seed in range(3):
+        x = WL.relu_map((n,), 0.7, seed, cuda)
+        row_end, col, val, nnz = gist.gist_ssdc_encode(x, workspace=ws, trim=True)
+        r_row_end, r_col, _ = ref.ssdc_encode(host(x))
+        assert_bits_equal(host(row_end), r_row_end, "row_end")
+        assert_bits_equal(host(col), r_col, "col")
+
+
+# ------------------------------------------------------------------------ a6/a7 DPR
+@pytest.mark.parametrize("bits", [16, 10, 8])
+@pytest.mark.parametrize("n", RAGGED)
+def test_dpr(gist, ref, cuda, bits, n):
+    x = WL.dpr_map((n,), n + bits, cuda)
+    if n >= 200:
+        sp = WL.dpr_specials().to(cuda)
+        x[: sp.numel()] = sp[: n]
+    packed = gist.gist_dpr_encode(x, bits)
+    r_packed = ref.dpr_encode(host(x), bits)
+    assert_bits_equal(host(packed), r_packed, f"fp{bits} packed")
+    back = gist.gist_dpr_decode(packed, n, bits)
+    assert_bits_equal(host(back), ref.dpr_decode(r_packed, n, bits), f"fp{bits} decode")
+
+
+@pytest.mark.parametrize("bits", [16, 10, 8])
+def test_dpr_decode_every_code(gist, ref, cuda, bits):
+    # all 2^bits codes in every field position of the word
+    k = {16: 2, 10: 3, 8: 4}[bits]
+    codes = np.arange(1 << bits, dtype=np.uint32)
+    n = codes.size
+    words = np.zeros(-(-n // k), np.uint32)
+    idx = np.arange(n)
+    np.bitwise_or.at(words, idx // k, codes << (bits * (idx % k)))
+    back = gist.gist_dpr_decode(torch.from_numpy(words.view(np.int32)).to(cuda), n, bits)
+    assert_bits_equal(host(back), ref.dpr_values(codes, bits), f"fp{bits} all codes")
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("bits", [16, 10, 8])
+def test_dpr_exhaustive_all_fp32_patterns(gist, ref, cuda, bits):
+    # Every one of the 2^32 fp32 bit patterns, in chunks; oracle on all host cores.
+    import concurrent.futures as cf
+    import os
+    chunk = 1 << 27
+    k = {16: 2, 10: 3, 8: 4}[bits]
+    chunk -= chunk % (12 * k)
+    workers = max(1, os.cpu_count() or 1)
+    with cf.ThreadPoolExecutor(workers) as ex:
+        start = 0
+        while start < (1 << 32):
+            m = min(chunk, (1 << 32) - start)
+            pat = torch.arange(start, start + m, dtype=torch.int64, device=cuda).to(torch.int32)
+            x = pat.view(torch.float32)
+            got = host(gist.gist_dpr_encode(x, bits))
+            xs = host(x)
+            parts = np.array_split(np.arange(m), workers)
+            parts = [p for p in parts if p.size]
+            # split on word boundaries
+            bounds = [0] + [int(p[-1] + 1) // k * k for p in parts[:-1]] + [m]
+            futs = [ex.submit(ref.dpr_encode, xs[a:b], bits) for a, b in zip(bounds[:-1], bounds[1:])]
+            expect = np.concatenate([f.result() for f in futs])
+            assert_bits_equal(got, expect, f"fp{bits} patterns [{start}, {start + m})")
+            start += m
+
+
+# ------------------------------------------------------------------------ full-size configs
+def _vgg_site(name):
+    return next(s for s in WL.NETS["vgg16"] if s.name == name)
+
+
+@pytest.mark.parametrize("site", ["relu1_2", "relu5_3"])
+def test_full_size_vgg16_relu_pool(gist, ref, cuda, site):
+    """C3 (VGG16 b64) ReLU->Pool site at full size: every output compared."""
+    s = _vgg_site(site)
+    shape = (64,) + s.chw
+    y = WL.relu_map(shape, 0.8, 3_000_000 + 1, cuda)
+    out, arg, mask = gist.gist_maxpool_fwd_argmax(y, s.pool)
+    mask = gist.gist_binarize_encode(y)
+    dout = WL.grad_map(tuple(out.shape), 17, cuda)
+    dx = gist.gist_pool_relu_bwd(dout, arg, mask, shape, s.pool)
+    yh = host(y)
+    r_out, r_arg = ref.maxpool_fwd_argmax(yh, s.pool)
+    r_mask = ref.binarize_encode(yh)
+    assert_bits_equal(host(mask), r_mask, "mask")
+    assert_bits_equal(host(out), r_out, "out")
+    assert_bits_equal(host(arg), r_arg, "arg")
+    del yh
+    assert_bits_equal(host(dx), ref.pool_relu_bwd(host(dout), r_arg, r_mask, shape, s.pool), "dx")
+
+
+def test_full_size_vgg16_ssdc_and_dpr(gist, ref, cuda):
+    s = _vgg_site("relu1_1")
+    x = WL.relu_map((64,) + s.chw, 0.8, 3_000_000 + 2, cuda)
+    row_end, col, val, nnz = gist.gist_ssdc_encode(x, trim=True)
+    xh = host(x)
+    r_row_end, r_col, r_val = ref.ssdc_encode(xh)
+    assert int(nnz.item()) == r_col.size
+    assert_bits_equal(host(row_end), r_row_end, "row_end")
+    assert_bits_equal(host(col), r_col, "col")
+    assert_bits_equal(host(val), r_val, "val")
+    back = gist.gist_ssdc_decode(row_end, col, val, x.numel())
+    assert torch.equal(back.view(torch.int32), x.reshape(-1).view(torch.int32))
+    for bits in (16, 10, 8):
+        packed = gist.gist_dpr_encode(x, bits)
+        assert_bits_equal(host(packed), ref.dpr_encode(xh, bits), f"fp{bits}")
