@@ -77,36 +77,51 @@ maxpool_fwd_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ 
     }
 }
 
-// 2x2 stride 2, no padding, every window fully inside (W even): two float2 row loads.
+// 2x2 stride 2, no padding, every window fully inside (W even): two float2 row loads per
+// output.  A warp handles kFwdU chunks of 32 consecutive outputs per iteration with all
+// 2*kFwdU loads issued before any compare (memory-level parallelism).
+constexpr int kFwdU = 4;
+
 __global__ void __launch_bounds__(kPoolThreads)
 maxpool_fwd_k2s2_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ out,
                         uint32_t *__restrict__ arg) {
     const int lane = threadIdx.x & 31;
     const int64_t chunks = ((int64_t)a.n_out + 31) / 32;
     const int64_t nwarps = ((int64_t)gridDim.x * kPoolThreads) >> 5;
-    for (int64_t c = ((int64_t)blockIdx.x * kPoolThreads + threadIdx.x) >> 5; c < chunks; c += nwarps) {
-        const int64_t o = c * 32 + lane;
-        uint32_t nib = 0;
-        if (o < a.n_out) {
-            uint32_t q, ow, nc, oh;
-            a.div_wo.divmod((uint32_t)o, q, ow);
-            a.div_ho.divmod(q, nc, oh);
-            const float *p = y + (int64_t)nc * a.H * a.W + (int64_t)(2 * oh) * a.W + 2 * ow;
-            const float2 r0 = ld_stream_f2(reinterpret_cast<const float2 *>(p));
-            const float2 r1 = ld_stream_f2(reinterpret_cast<const float2 *>(p + a.W));
-            float best = -CUDART_INF_F;
-            int bi = 0;
-            take(r0.x, 0, best, bi);
-            take(r0.y, 1, best, bi);
-            take(r1.x, 2, best, bi);
-            take(r1.y, 3, best, bi);
-            out[o] = best;
-            nib = (uint32_t)bi << (4 * (lane & 7));
+    for (int64_t c0 = (((int64_t)blockIdx.x * kPoolThreads + threadIdx.x) >> 5) * kFwdU; c0 < chunks;
+         c0 += nwarps * kFwdU) {
+        float2 r0[kFwdU], r1[kFwdU];
+#pragma unroll
+        for (int u = 0; u < kFwdU; ++u) {
+            const int64_t o = (c0 + u) * 32 + lane;
+            if (o < a.n_out) {
+                uint32_t q, ow, nc, oh;
+                a.div_wo.divmod((uint32_t)o, q, ow);
+                a.div_ho.divmod(q, nc, oh);
+                const float *p = y + (int64_t)nc * a.H * a.W + (int64_t)(2 * oh) * a.W + 2 * ow;
+                r0[u] = ld_stream_f2(reinterpret_cast<const float2 *>(p));
+                r1[u] = ld_stream_f2(reinterpret_cast<const float2 *>(p + a.W));
+            }
         }
-        nib |= __shfl_xor_sync(kFull, nib, 1);
-        nib |= __shfl_xor_sync(kFull, nib, 2);
-        nib |= __shfl_xor_sync(kFull, nib, 4);
-        if ((lane & 7) == 0 && o < a.n_out) arg[o >> 3] = nib;
+#pragma unroll
+        for (int u = 0; u < kFwdU; ++u) {
+            const int64_t o = (c0 + u) * 32 + lane;
+            uint32_t nib = 0;
+            if (o < a.n_out) {
+                float best = -CUDART_INF_F;
+                int bi = 0;
+                take(r0[u].x, 0, best, bi);
+                take(r0[u].y, 1, best, bi);
+                take(r1[u].x, 2, best, bi);
+                take(r1[u].y, 3, best, bi);
+                out[o] = best;
+                nib = (uint32_t)bi << (4 * (lane & 7));
+            }
+            nib |= __shfl_xor_sync(kFull, nib, 1);
+            nib |= __shfl_xor_sync(kFull, nib, 2);
+            nib |= __shfl_xor_sync(kFull, nib, 4);
+            if ((lane & 7) == 0 && o < a.n_out) arg[o >> 3] = nib;
+        }
     }
 }
 
@@ -150,31 +165,61 @@ pool_bwd_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg
     }
 }
 
-// 2x2 stride 2, no padding, W even: one thread per pair of adjacent inputs (same window).
+// 2x2 stride 2, no padding, every window inside: one thread per pool output writes its
+// whole 2x2 input block (two float2 rows).  Windows do not overlap, so dx is dY routed to
+// the argmax slot (+0.0f + dY, R6) and selected by the mask (R7); inputs in an uncovered
+// last row (odd H, floor mode) are zeroed by the owner of the row above.  All loads of
+// kBwdU outputs are issued before use.
+constexpr int kBwdU = 4;
+
 __global__ void __launch_bounds__(kPoolThreads)
 pool_bwd_k2s2_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
                      const uint32_t *__restrict__ mask, PoolArgs a, float *__restrict__ dx) {
-    const int64_t pairs = (int64_t)a.n_in / 2;
     const int64_t stride = (int64_t)gridDim.x * kPoolThreads;
-    for (int64_t p = (int64_t)blockIdx.x * kPoolThreads + threadIdx.x; p < pairs; p += stride) {
-        const int64_t i = 2 * p;
-        uint32_t q, iw, nc, ih;
-        a.div_w.divmod((uint32_t)i, q, iw);
-        a.div_h.divmod(q, nc, ih);
-        const uint32_t oh = ih >> 1, ow = iw >> 1;
-        float2 r = make_float2(0.0f, 0.0f);
-        if ((int)oh < a.Ho) {
-            const int64_t o = ((int64_t)nc * a.Ho + oh) * a.Wo + ow;
-            const uint32_t nib = nibble(arg, o);
-            const uint32_t m = mask ? (ld_ro(mask + (i >> 5)) >> (i & 31)) : 3u;
-            const uint32_t l0 = (ih & 1u) * 2u;
-            if ((nib == l0 && (m & 1u)) || (nib == l0 + 1 && (m & 2u))) {
-                const float g = 0.0f + ld_ro(dout + o);
-                r.x = (nib == l0 && (m & 1u)) ? g : 0.0f;
-                r.y = (nib == l0 + 1 && (m & 2u)) ? g : 0.0f;
+    const bool odd_h = (a.H & 1) != 0;
+    for (int64_t o0 = (int64_t)blockIdx.x * kPoolThreads + threadIdx.x; o0 < a.n_out; o0 += stride * kBwdU) {
+        float g[kBwdU];
+        uint32_t nib[kBwdU], m0[kBwdU], m1[kBwdU];
+        int64_t i0[kBwdU];
+#pragma unroll
+        for (int u = 0; u < kBwdU; ++u) {
+            const int64_t o = o0 + u * stride;
+            if (o < a.n_out) {
+                uint32_t q, ow, nc, oh;
+                a.div_wo.divmod((uint32_t)o, q, ow);
+                a.div_ho.divmod(q, nc, oh);
+                i0[u] = ((int64_t)nc * a.H + 2 * oh) * a.W + 2 * ow;  // top-left input
+                g[u] = ld_stream_f32(dout + o);
+                nib[u] = ld_ro(arg + (o >> 3)) >> (4 * (o & 7));
+                if (mask) {
+                    m0[u] = ld_ro(mask + (i0[u] >> 5)) >> (i0[u] & 31);
+                    m1[u] = ld_ro(mask + ((i0[u] + a.W) >> 5)) >> ((i0[u] + a.W) & 31);
+                } else {
+                    m0[u] = m1[u] = 3u;
+                }
             }
         }
-        reinterpret_cast<float2 *>(dx)[p] = r;
+#pragma unroll
+        for (int u = 0; u < kBwdU; ++u) {
+            const int64_t o = o0 + u * stride;
+            if (o >= a.n_out) break;
+            const float v = 0.0f + g[u];
+            const uint32_t k = nib[u] & 0xfu;
+            float2 top, bot;
+            top.x = (k == 0 && (m0[u] & 1u)) ? v : 0.0f;
+            top.y = (k == 1 && (m0[u] & 2u)) ? v : 0.0f;
+            bot.x = (k == 2 && (m1[u] & 1u)) ? v : 0.0f;
+            bot.y = (k == 3 && (m1[u] & 2u)) ? v : 0.0f;
+            *reinterpret_cast<float2 *>(dx + i0[u]) = top;
+            *reinterpret_cast<float2 *>(dx + i0[u] + a.W) = bot;
+            if (odd_h) {  // zero the uncovered last input row of the plane
+                uint32_t q, ow, nc, oh;
+                a.div_wo.divmod((uint32_t)o, q, ow);
+                a.div_ho.divmod(q, nc, oh);
+                if ((int)oh == a.Ho - 1 && 2 * a.Ho < a.H)
+                    *reinterpret_cast<float2 *>(dx + i0[u] + 2 * (int64_t)a.W) = make_float2(0.0f, 0.0f);
+            }
+        }
     }
 }
 
@@ -220,7 +265,7 @@ cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, 
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
     const unsigned grid = grid_for(a.n_out, kPoolThreads, 8);
     if (is_k2s2_exact(p, H, W, Ho, Wo))
-        maxpool_fwd_k2s2_kernel<<<grid, kPoolThreads, 0, s>>>(y, a, out, argmax);
+        maxpool_fwd_k2s2_kernel<<<grid_for(ceil_div(a.n_out, kFwdU), kPoolThreads, 8), kPoolThreads, 0, s>>>(y, a, out, argmax);
     else if (p.kh == 3 && p.kw == 3)
         maxpool_fwd_kernel<3, 3><<<grid, kPoolThreads, 0, s>>>(y, a, out, argmax);
     else if (p.kh == 2 && p.kw == 2)
@@ -235,7 +280,7 @@ cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uin
                             cudaStream_t s) {
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
     if (is_k2s2_exact(p, H, W, Ho, Wo)) {
-        pool_bwd_k2s2_kernel<<<grid_for(a.n_in / 2, kPoolThreads, 8), kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+        pool_bwd_k2s2_kernel<<<grid_for(ceil_div(a.n_out, kBwdU), kPoolThreads, 8), kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
     } else {
         const unsigned grid = grid_for(a.n_in, kPoolThreads, 8);
         if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2)

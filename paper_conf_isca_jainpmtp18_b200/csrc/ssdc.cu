@@ -1,30 +1,37 @@
 // ssdc.cu — a4/a5: Sparse Storage, Dense Compute (PAPER.md P:158-P:164 §IV-A).
 //
 // Encode: dense fp32 -> CSR with 256-column rows and uint8 column indices (Narrow Value
-// Optimization).  One pass over x (4n bytes read, 5*nnz + 4*rows written):
-//   * a CTA owns a tile of 32 rows (8192 elements); tiles are claimed in order through an
-//     atomic ticket so every predecessor is already running (forward progress);
-//   * each warp holds 4 rows in registers (8 LDG.128 per lane), counts nonzero bit
-//     patterns per half-row and scans 4 rows at once with one packed 8-bit-lane
-//     shuffle scan; warp 0 scans the tile's 32 row counts;
-//   * the tile's global offset comes from a decoupled look-back over the predecessors'
-//     {aggregate, inclusive-prefix} descriptors (one 64-bit word each: 2-bit status +
-//     value), read 32 at a time by warp 0;
-//   * rows are then written straight from registers: row_end, and each lane's nonzeros
-//     at consecutive offsets (stores of a warp fall in one contiguous output range).
+// Optimization).  One pass over x (4n bytes read, 5*nnz + 4*rows written).
+// Persistent, warp-specialized CTAs (3 per SM) stream 16-row tiles (4096 elements, 16 KB)
+// through a 4-stage shared-memory ring filled by 1-D TMA bulk copies (cp.async.bulk +
+// mbarrier).  Tiles are claimed in order through an atomic ticket, so every predecessor of a
+// tile is held by a running CTA (forward progress).  Roles, linked only by mbarriers:
+//   * counter warp: as soon as a tile lands, counts the nonzero bit patterns of its rows
+//     (R8), scans the 16 row counts and publishes the tile aggregate — aggregates appear one
+//     TMA latency after the ticket, independent of how far the writers are;
+//   * look-back warp: decoupled look-back (32 predecessors' 64-bit {status, value}
+//     descriptors per round) -> the tile's global offset; publishes the inclusive prefix and
+//     the tile's row_end entries;
+//   * 4 writer warps: each holds 4 rows in registers (lane: cols [4l,4l+4) and
+//     [128+4l,128+4l+4)), takes ranks from warp ballots, compacts the whole tile in place,
+//     shifted to the global 16-byte phase, and lane 0 of warp 0 writes the aligned bodies of
+//     val/col with TMA bulk stores (cp.async.bulk.global.shared::cta); ragged ends by lanes.
 // Decode: a warp expands 4 consecutive rows (whose entries are one contiguous range)
 //   through a 4 KB shared-memory row buffer and writes them back with float4 stores.
 #include "common.cuh"
 #include "kernels.h"
+#include "tma.cuh"
+
+#include <mutex>
 
 namespace gist {
 
 namespace {
 
 constexpr int kRow = 256;
-constexpr int kEncThreads = 256;
+constexpr int kEncThreads = 128;  // worker threads (4 warps x 4 rows)
 constexpr int kRowsPerWarp = 4;
-constexpr int kTileRows = (kEncThreads / 32) * kRowsPerWarp;  // 32
+constexpr int kTileRows = (kEncThreads / 32) * kRowsPerWarp;  // 16
 constexpr uint64_t kStatusA = 1ull << 62;                    // aggregate available
 constexpr uint64_t kStatusP = 2ull << 62;                    // inclusive prefix available
 constexpr uint64_t kValueMask = (1ull << 62) - 1;
@@ -44,159 +51,251 @@ __device__ __forceinline__ void st_relaxed(uint64_t *p, uint64_t v) {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-__device__ __forceinline__ uint32_t nz(float v) { return __float_as_uint(v) != 0u; }
 
 __global__ void ssdc_ws_init(uint64_t *ws, int64_t words) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += (int64_t)gridDim.x * blockDim.x)
         ws[i] = 0ull;
 }
 
-__global__ void __launch_bounds__(kEncThreads)
+constexpr int kStages = 4;                       // TMA ring depth per CTA
+constexpr int kCtasPerSm = 3;                    // smem/register-limited residency
+constexpr int kTileElems = kTileRows * kRow;     // 4096 elements
+constexpr uint32_t kTileBytes = kTileElems * 4;  // 16 KB
+constexpr int kWarps = kEncThreads / 32;         // writer warps (4 rows each)
+constexpr int kCountWarp = kWarps;               // counts every tile as soon as it lands
+constexpr int kLbWarp = kWarps + 1;              // first of kLbWarps look-back warps
+constexpr int kLbWarps = 1;                      // (more take alternate tiles)
+constexpr int kCtaThreads = kEncThreads + 32 + 32 * kLbWarps;
+
+struct __align__(128) EncSmem {
+    float tile[kStages][kTileElems + 4];    // TMA destinations; the written tile is compacted in place
+    uint8_t colbuf[kTileElems + 16];        // compacted column bytes of the tile being written
+    uint64_t full[kStages];                 // TMA landed (or no tile: arrive without bytes)
+    uint64_t counted[kStages];              // counter warp -> look-back warp
+    uint64_t resolved[kStages];             // look-back warp -> writers
+    int64_t ticket[kStages];                // tile index held by each stage
+    uint32_t row_cnt[kStages][kTileRows];   // per-row nonzeros
+    uint32_t row_excl[kStages][kTileRows];  // tile-local exclusive row offsets
+    int64_t excl[kStages];                  // global offset of each stage's tile
+    int32_t last_j;                         // CTA-local index of the first "no tile" ticket
+};
+
+// Start the TMA bulk load of tile t (a ticket claimed earlier, in order, so every predecessor
+// is held by a running CTA) into stage s.  Always completes one arrival on full[s], so the
+// counter warp also learns about "no more tiles".  One thread.
+__device__ __forceinline__ void load_tile(EncSmem &S, int s, int64_t t, const float *x, int64_t n, int64_t tiles) {
+    S.ticket[s] = t;
+    uint32_t bytes = 0;
+    if (t < tiles) {
+        const int64_t avail = n - t * kTileElems;
+        bytes = avail >= kTileElems ? kTileBytes : (uint32_t)((avail * 4) & ~15ll);
+    }
+    fence_proxy_async_smem();
+    mbar_arrive_expect_tx(&S.full[s], bytes);
+    if (bytes) tma_load_1d(S.tile[s], x + t * kTileElems, bytes, &S.full[s]);
+}
+
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+// Decoupled look-back by one warp: lane i reads tile base-i.  Sums aggregates up to and
+// including the nearest inclusive prefix, re-polling only needed unpublished descriptors.
+__device__ __forceinline__ int64_t look_back(const Workspace *ws, int64_t tile, int lane) {
+    int64_t excl = 0;
+    for (int64_t base = tile - 1;; base -= 32) {
+        const int64_t idx = base - lane;
+        uint64_t d = (idx >= 0) ? ld_relaxed(&ws->desc[idx]) : kStatusP;  // virtual P(0)
+        uint32_t pm, need;
+        for (;;) {
+            pm = __ballot_sync(kFull, (d >> 62) == 2);
+            const uint32_t xm = __ballot_sync(kFull, (d >> 62) == 0);
+            need = pm ? (((pm & (0u - pm)) << 1) - 1u) : kFull;
+            if (!(xm & need)) break;
+            if ((d >> 62) == 0) d = ld_relaxed(&ws->desc[idx]);
+        }
+        uint64_t v = ((need >> lane) & 1u) ? (d & kValueMask) : 0ull;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+        excl += (int64_t)v;
+        if (pm) return excl;
+    }
+}
+
+__device__ __forceinline__ void writers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kEncThreads) : "memory"); }
+
+__global__ void __launch_bounds__(kCtaThreads, kCtasPerSm)
 ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t tiles,
                    int32_t *__restrict__ row_end, uint8_t *__restrict__ col, float *__restrict__ val,
                    int64_t capacity, int64_t *__restrict__ nnz_out, Workspace *__restrict__ ws) {
-    __shared__ uint32_t s_tile;
-    __shared__ uint32_t s_row_cnt[kTileRows];
-    __shared__ uint32_t s_row_excl[kTileRows];
-    __shared__ int64_t s_prefix;
-
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    EncSmem &S = *reinterpret_cast<EncSmem *>(smem_raw);
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
-    if (threadIdx.x == 0) s_tile = atomicAdd(&ws->ticket, 1u);
-    __syncthreads();
-    const int64_t tile = s_tile;
-    if (tile >= tiles) return;
 
-    // ---- load 4 rows per warp: lane holds cols [4l, 4l+4) and [128+4l, 128+4l+4)
-    const int64_t row0 = tile * kTileRows + warp * kRowsPerWarp;
-    float4 lo[kRowsPerWarp], hi[kRowsPerWarp];
-#pragma unroll
-    for (int r = 0; r < kRowsPerWarp; ++r) {
-        const int64_t base = (row0 + r) * kRow;
-        if (base + kRow <= n) {
-            lo[r] = ld_stream_f4(reinterpret_cast<const float4 *>(x + base) + lane);
-            hi[r] = ld_stream_f4(reinterpret_cast<const float4 *>(x + base + 128) + lane);
-        } else {  // ragged last row (or beyond the end): scalar, zero-filled
-            float t[8];
-#pragma unroll
-            for (int j = 0; j < 8; ++j) {
-                const int64_t i = base + (j < 4 ? 4 * lane + j : 128 + 4 * lane + j - 4);
-                t[j] = (i < n) ? x[i] : 0.0f;
-            }
-            lo[r] = make_float4(t[0], t[1], t[2], t[3]);
-            hi[r] = make_float4(t[4], t[5], t[6], t[7]);
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kStages; ++s) {
+            mbar_init(&S.full[s], 1);
+            mbar_init(&S.counted[s], 1);
+            mbar_init(&S.resolved[s], 1);
         }
-    }
-
-    // ---- per-lane counts, 4 rows x {lo, hi} packed into two 4x8-bit words, warp scan
-    uint32_t m_lo[kRowsPerWarp], m_hi[kRowsPerWarp];
-    uint32_t pk_lo = 0, pk_hi = 0;
-#pragma unroll
-    for (int r = 0; r < kRowsPerWarp; ++r) {
-        m_lo[r] = nz(lo[r].x) | (nz(lo[r].y) << 1) | (nz(lo[r].z) << 2) | (nz(lo[r].w) << 3);
-        m_hi[r] = nz(hi[r].x) | (nz(hi[r].y) << 1) | (nz(hi[r].z) << 2) | (nz(hi[r].w) << 3);
-        pk_lo |= (uint32_t)__popc(m_lo[r]) << (8 * r);
-        pk_hi |= (uint32_t)__popc(m_hi[r]) << (8 * r);
-    }
-    uint32_t in_lo = pk_lo, in_hi = pk_hi;  // inclusive scans (each 8-bit lane <= 128)
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const uint32_t a = __shfl_up_sync(kFull, in_lo, d);
-        const uint32_t b = __shfl_up_sync(kFull, in_hi, d);
-        if (lane >= d) {
-            in_lo += a;
-            in_hi += b;
-        }
-    }
-    const uint32_t tot_lo = __shfl_sync(kFull, in_lo, 31);
-    const uint32_t tot_hi = __shfl_sync(kFull, in_hi, 31);
-    if (lane < kRowsPerWarp)
-        s_row_cnt[warp * kRowsPerWarp + lane] = ((tot_lo >> (8 * lane)) & 0xffu) + ((tot_hi >> (8 * lane)) & 0xffu);
-    __syncthreads();
-
-    // ---- warp 0: tile-level row scan + decoupled look-back for the tile's offset
-    if (warp == 0) {
-        const uint32_t c = s_row_cnt[lane];
-        uint32_t inc = c;
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const uint32_t t = __shfl_up_sync(kFull, inc, d);
-            if (lane >= d) inc += t;
-        }
-        s_row_excl[lane] = inc - c;
-        const uint64_t total = __shfl_sync(kFull, inc, 31);
-        int64_t excl = 0;
-        if (tile == 0) {
-            if (lane == 0) st_relaxed(&ws->desc[0], kStatusP | total);
-        } else {
-            if (lane == 0) st_relaxed(&ws->desc[tile], kStatusA | total);
-            // Look back over predecessors base, base-1, ... 32 at a time (lane i reads
-            // tile base-i).  Sum aggregates up to and including the nearest inclusive
-            // prefix; spin only on descriptors that are still unpublished and needed.
-            int64_t base = tile - 1;
-            while (true) {
-                const int64_t idx = base - lane;
-                uint64_t d = (idx >= 0) ? ld_relaxed(&ws->desc[idx]) : kStatusP;  // virtual P(0)
-                uint32_t pmask, need;
-                while (true) {
-                    pmask = __ballot_sync(kFull, (d >> 62) == 2);
-                    const uint32_t xmask = __ballot_sync(kFull, (d >> 62) == 0);
-                    need = pmask ? (((pmask & (0u - pmask)) << 1) - 1u) : kFull;
-                    if (!(xmask & need)) break;
-                    if ((d >> 62) == 0) d = ld_relaxed(&ws->desc[idx]);
-                }
-                uint64_t v = ((need >> lane) & 1u) ? (d & kValueMask) : 0ull;
-#pragma unroll
-                for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
-                excl += (int64_t)v;
-                if (pmask) break;
-                base -= 32;
-            }
-            if (lane == 0) st_relaxed(&ws->desc[tile], kStatusP | (uint64_t)(excl + (int64_t)total));
-        }
-        if (lane == 0) {
-            s_prefix = excl;
-            if (tile == tiles - 1) *nnz_out = excl + (int64_t)total;
-        }
-        // row ends for the tile
-        const int64_t r = tile * kTileRows + lane;
-        if (r < rows) row_end[r] = (int32_t)(excl + inc);
+        fence_mbar_init();
+        S.last_j = 0x7fffffff;
+        for (int s = 0; s < kStages; ++s) load_tile(S, s, atomicAdd(&ws->ticket, 1u), x, n, tiles);
     }
     __syncthreads();
 
-    // ---- scatter this warp's nonzeros (ascending column order within each row)
-    const int64_t prefix = s_prefix;
-#pragma unroll
-    for (int r = 0; r < kRowsPerWarp; ++r) {
-        const int rr = warp * kRowsPerWarp + r;
-        const int64_t row_base = prefix + s_row_excl[rr];
-        const uint32_t ex_lo = ((in_lo >> (8 * r)) & 0xffu) - __popc(m_lo[r]);
-        const uint32_t ex_hi = ((in_hi >> (8 * r)) & 0xffu) - __popc(m_hi[r]);
-        const uint32_t t_lo = (tot_lo >> (8 * r)) & 0xffu;
-        int64_t o = row_base + ex_lo;
-        const float vl[4] = {lo[r].x, lo[r].y, lo[r].z, lo[r].w};
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            if ((m_lo[r] >> j) & 1u) {
-                if (o < capacity) {
-                    col[o] = (uint8_t)(4 * lane + j);
-                    val[o] = vl[j];
+    if (warp == kCountWarp) {
+        // ---- counter: nonzero bit patterns (R8) of every row, tile scan, publish aggregate
+        for (int j = 0;; ++j) {
+            const int s = j % kStages;
+            mbar_wait(&S.full[s], (uint32_t)(j / kStages) & 1u);
+            const int64_t tile = S.ticket[s];
+            if (tile < tiles) {
+                float *T = S.tile[s];
+                if (tile == tiles - 1) {  // ragged last tile: tail the TMA could not copy, zeros
+                    const int64_t avail = n - tile * kTileElems;
+                    const int from = avail >= kTileElems ? kTileElems : (int)(((avail * 4) & ~15ll) / 4);
+                    for (int i = from + lane; i < kTileElems; i += 32)
+                        T[i] = (i < avail) ? x[tile * kTileElems + i] : 0.0f;
+                    __syncwarp();
                 }
-                ++o;
+                uint32_t mine = 0;  // lane r ends up with row r's count
+#pragma unroll 4
+                for (int r = 0; r < kTileRows; ++r) {
+                    const uint4 *row4 = reinterpret_cast<const uint4 *>(T + r * kRow);
+                    const uint4 a = row4[lane], b = row4[32 + lane];
+                    const uint32_t c = (a.x != 0u) + (a.y != 0u) + (a.z != 0u) + (a.w != 0u) + (b.x != 0u) +
+                                       (b.y != 0u) + (b.z != 0u) + (b.w != 0u);
+                    const uint32_t t = __reduce_add_sync(kFull, c);
+                    if (lane == r) mine = t;
+                }
+                uint32_t inc = mine;
+#pragma unroll
+                for (int d = 1; d < 32; d <<= 1) {
+                    const uint32_t t = __shfl_up_sync(kFull, inc, d);
+                    if (lane >= d) inc += t;
+                }
+                if (lane < kTileRows) {
+                    S.row_cnt[s][lane] = mine;
+                    S.row_excl[s][lane] = inc - mine;
+                }
+                if (lane == 31) st_relaxed(&ws->desc[tile], (tile == 0 ? kStatusP : kStatusA) | (uint64_t)inc);
+            }
+            __syncwarp();
+            if (lane == 0) {
+                if (tile >= tiles) *(volatile int32_t *)&S.last_j = j;  // before the arrival
+                mbar_arrive(&S.counted[s]);
+            }
+            if (tile >= tiles) break;
+        }
+    } else if (warp >= kLbWarp) {
+        // ---- look-back: global offset of each counted tile; publish prefix, row ends, nnz.
+        // Warp kLbWarp + i resolves the CTA's tiles j = i, i + kLbWarps, ...
+        for (int j = warp - kLbWarp;; j += kLbWarps) {
+            const int s = j % kStages;
+            // poll: past the CTA's last tile no arrival will ever come for this j
+            bool ready = false;
+            while (!(ready = mbar_test(&S.counted[s], (uint32_t)(j / kStages) & 1u)))
+                if (*(volatile int32_t *)&S.last_j < j) break;
+            if (!ready) break;
+            const int64_t tile = S.ticket[s];
+            if (tile < tiles) {
+                const int64_t excl = (tile == 0) ? 0 : look_back(ws, tile, lane);
+                const uint32_t total = S.row_excl[s][kTileRows - 1] + S.row_cnt[s][kTileRows - 1];
+                if (lane == 0) {
+                    S.excl[s] = excl;
+                    if (tile > 0) st_relaxed(&ws->desc[tile], kStatusP | (uint64_t)(excl + total));
+                    if (tile == tiles - 1) *nnz_out = excl + total;
+                }
+                const int64_t r = tile * kTileRows + lane;
+                if (lane < kTileRows && r < rows)
+                    row_end[r] = (int32_t)(excl + S.row_excl[s][lane] + S.row_cnt[s][lane]);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&S.resolved[s]);
+            if (tile >= tiles) break;
+        }
+    } else {
+        // ---- writers: compact the tile contiguously in place, shifted so smem and global share
+        // their 16-byte phase (value k -> T[sv + k] = val[excl + k], column -> colbuf[sc + k]),
+        // then TMA bulk-store the aligned bodies; ranks from ballots (lane l holds cols 4l+j
+        // "lo" and 128+4l+j "hi", j = 0..3).
+        const uint32_t lt = (1u << lane) - 1u;
+        for (int j = 0;; ++j) {
+            const int s = j % kStages;
+            mbar_wait(&S.resolved[s], (uint32_t)(j / kStages) & 1u);
+            const int64_t tile = S.ticket[s];
+            if (tile >= tiles) break;
+            float *T = S.tile[s];
+            const int64_t excl = S.excl[s];
+            const uint32_t sv = (uint32_t)excl & 3u, sc = (uint32_t)excl & 15u;
+            float v[kRowsPerWarp][8];
+            uint32_t bal[kRowsPerWarp][8];
+#pragma unroll
+            for (int r = 0; r < kRowsPerWarp; ++r) {
+                const float4 *row4 = reinterpret_cast<const float4 *>(T + (warp * kRowsPerWarp + r) * kRow);
+                const float4 a = row4[lane], b = row4[32 + lane];
+                v[r][0] = a.x; v[r][1] = a.y; v[r][2] = a.z; v[r][3] = a.w;
+                v[r][4] = b.x; v[r][5] = b.y; v[r][6] = b.z; v[r][7] = b.w;
+#pragma unroll
+                for (int k = 0; k < 8; ++k) bal[r][k] = __ballot_sync(kFull, __float_as_uint(v[r][k]) != 0u);
+            }
+            writers_sync();  // whole tile in registers (and the previous bulk store read out)
+#pragma unroll
+            for (int r = 0; r < kRowsPerWarp; ++r) {
+                const uint32_t q0 = sv + S.row_excl[s][warp * kRowsPerWarp + r];
+                uint32_t p_lo = q0 + __popc(bal[r][0] & lt) + __popc(bal[r][1] & lt) + __popc(bal[r][2] & lt) +
+                                __popc(bal[r][3] & lt);
+                uint32_t p_hi = q0 + __popc(bal[r][0]) + __popc(bal[r][1]) + __popc(bal[r][2]) + __popc(bal[r][3]) +
+                                __popc(bal[r][4] & lt) + __popc(bal[r][5] & lt) + __popc(bal[r][6] & lt) +
+                                __popc(bal[r][7] & lt);
+                uint8_t *cb = S.colbuf + sc - sv;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const uint32_t on = (bal[r][k] >> lane) & 1u;
+                    if (on) {
+                        T[p_lo] = v[r][k];
+                        cb[p_lo] = (uint8_t)(4 * lane + k);
+                    }
+                    p_lo += on;
+                }
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const uint32_t on = (bal[r][4 + k] >> lane) & 1u;
+                    if (on) {
+                        T[p_hi] = v[r][4 + k];
+                        cb[p_hi] = (uint8_t)(128 + 4 * lane + k);
+                    }
+                    p_hi += on;
+                }
+            }
+            fence_proxy_async_smem();  // generic smem writes before the async-proxy bulk store
+            writers_sync();
+            if (warp == 0) {
+                const int64_t total = S.row_excl[s][kTileRows - 1] + S.row_cnt[s][kTileRows - 1];
+                int64_t lim = total;
+                if (excl + lim > capacity) lim = capacity > excl ? capacity - excl : 0;
+                const int64_t hv = (4 - sv) & 3, hc = (16 - sc) & 15;  // heads up to 16-B alignment
+                const int64_t bv = lim > hv ? (lim - hv) & ~3ll : 0, bc = lim > hc ? (lim - hc) & ~15ll : 0;
+                // ragged ends: < 4 values and < 16 columns at each end
+                const int64_t k0 = lane, k1 = hv + bv + lane, k2 = hc + bc + lane;
+                if (k0 < hv && k0 < lim) val[excl + k0] = T[sv + k0];
+                if (lane < 4 && k1 < lim) val[excl + k1] = T[sv + k1];
+                if (k0 < hc && k0 < lim) col[excl + k0] = S.colbuf[sc + k0];
+                if (lane < 16 && k2 < lim) col[excl + k2] = S.colbuf[sc + k2];
+                __syncwarp();
+                if (lane == 0) {
+                    if (bv) tma_store_1d(val + excl + hv, T + sv + hv, (uint32_t)(4 * bv));
+                    if (bc) tma_store_1d(col + excl + hc, S.colbuf + sc + hc, (uint32_t)bc);
+                    bulk_commit();
+                    bulk_wait_read();  // stage + colbuf read out
+                    load_tile(S, s, atomicAdd(&ws->ticket, 1u), x, n, tiles);  // refill this stage
+                }
+                __syncwarp();
             }
         }
-        o = row_base + t_lo + ex_hi;
-        const float vh[4] = {hi[r].x, hi[r].y, hi[r].z, hi[r].w};
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            if ((m_hi[r] >> j) & 1u) {
-                if (o < capacity) {
-                    col[o] = (uint8_t)(128 + 4 * lane + j);
-                    val[o] = vh[j];
-                }
-                ++o;
-            }
-        }
+        if (threadIdx.x == 0) bulk_wait_all();
     }
 }
 
@@ -264,8 +363,14 @@ cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint
     int64_t iblocks = ceil_div(ws_words, 256);
     if (iblocks > 1024) iblocks = 1024;
     ssdc_ws_init<<<(unsigned)iblocks, 256, 0, s>>>(reinterpret_cast<uint64_t *>(workspace), ws_words);
-    ssdc_encode_kernel<<<(unsigned)tiles, kEncThreads, 0, s>>>(x, n, rows, tiles, row_end, col, val, capacity,
-                                                               nnz, reinterpret_cast<Workspace *>(workspace));
+    static std::once_flag attr_once;
+    std::call_once(attr_once, [] {
+        cudaFuncSetAttribute(ssdc_encode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(EncSmem));
+    });
+    int64_t grid = (int64_t)num_sms() * kCtasPerSm;  // persistent, smem-limited residency
+    if (grid > tiles) grid = tiles;
+    ssdc_encode_kernel<<<(unsigned)grid, kCtaThreads, sizeof(EncSmem), s>>>(
+        x, n, rows, tiles, row_end, col, val, capacity, nnz, reinterpret_cast<Workspace *>(workspace));
     return cudaPeekAtLastError();
 }
 
