@@ -1,9 +1,11 @@
 // dpr.cu — a6/a7: Delayed Precision Reduction encode/decode (PAPER.md P:166-P:171 §IV-A).
 //
 // fp32 -> FP16 (IEEE 1-5-10) / FP10 (1-5-4) / FP8 (1-4-3), 2/3/4 codes per 32-bit word.
-// HBM-bound streaming kernels: every thread converts whole 16-byte groups (FP16: 1 float4
-// -> 2 words; FP8: 1 float4 -> 1 word; FP10: 3 float4 -> 4 words = one uint4), with four
-// independent groups in flight per thread.
+// HBM-bound streaming kernels.  Encode: every thread converts whole 16-byte groups (FP16:
+// 1 float4 -> 2 words; FP8: 1 float4 -> 1 word; FP10: 3 float4 -> 4 words = one uint4), with
+// 8 (FP16/FP8) or 4 (FP10) independent groups in flight per thread.  Decode: FP16/FP8 mirror
+// that mapping (both sides of every warp access contiguous); FP10 decodes 128 words per warp
+// and transposes the 384 values through shared memory so the float4 stores are coalesced.
 //
 // FP10/FP8 use branch-free integer rounding on the fp32 bit pattern: adding
 // 2^(s-1)-1 + lsb and shifting right by s = 23-M rounds the significand to M bits with ties
@@ -21,7 +23,8 @@ namespace gist {
 namespace {
 
 constexpr int kDprThreads = 256;
-constexpr int kUnroll = 4;
+constexpr int kUnroll = 4;  // groups in flight per thread (FP10: 48 B each)
+constexpr int kUnroll4 = 8;  // FP16/FP8: 16-byte groups, so twice as many in flight
 
 template <int E, int M>
 __device__ __forceinline__ uint32_t enc_small(float x) {
@@ -119,11 +122,12 @@ dpr_encode_kernel(const float *__restrict__ x, int64_t n, uint32_t *__restrict__
     const int64_t tid = (int64_t)blockIdx.x * kDprThreads + threadIdx.x;
     const int64_t nthreads = (int64_t)gridDim.x * kDprThreads;
     const float4 *x4 = reinterpret_cast<const float4 *>(x);
+    constexpr int U = (BITS == 10) ? kUnroll : kUnroll4;
 
-    for (int64_t g0 = tid; g0 < groups; g0 += nthreads * kUnroll) {
-        float4 v[kUnroll][GF / 4];
+    for (int64_t g0 = tid; g0 < groups; g0 += nthreads * U) {
+        float4 v[U][GF / 4];
 #pragma unroll
-        for (int u = 0; u < kUnroll; ++u) {
+        for (int u = 0; u < U; ++u) {
             const int64_t g = g0 + (int64_t)u * nthreads;
             if (g < groups) {
 #pragma unroll
@@ -131,7 +135,7 @@ dpr_encode_kernel(const float *__restrict__ x, int64_t n, uint32_t *__restrict__
             }
         }
 #pragma unroll
-        for (int u = 0; u < kUnroll; ++u) {
+        for (int u = 0; u < U; ++u) {
             const int64_t g = g0 + (int64_t)u * nthreads;
             if (g >= groups) break;
             if constexpr (BITS == 16) {
@@ -166,57 +170,77 @@ template <int BITS>
 __global__ void __launch_bounds__(kDprThreads)
 dpr_decode_kernel(const uint32_t *__restrict__ packed, int64_t n, float *__restrict__ x) {
     constexpr int K = Fmt<BITS>::K;
-    constexpr int GF = (BITS == 10) ? 12 : 4;  // floats per group
-    constexpr int GW = GF / K;                 // words per group: 2 / 4 / 1
     constexpr uint32_t FIELD = (1u << BITS) - 1u;
-    const int64_t groups = n / GF;
     const int64_t tid = (int64_t)blockIdx.x * kDprThreads + threadIdx.x;
     const int64_t nthreads = (int64_t)gridDim.x * kDprThreads;
     float4 *x4 = reinterpret_cast<float4 *>(x);
-
-    for (int64_t g0 = tid; g0 < groups; g0 += nthreads * kUnroll) {
-        uint32_t w[kUnroll][GW];
+    if constexpr (BITS != 10) {
+        // FP16: one uint2 (2 words) -> one float4; FP8: one word -> one float4.  Both sides of
+        // every warp access are contiguous.
+        constexpr int GW = 4 / K;  // words per float4 group: 2 / 1
+        const int64_t groups = n / 4;
+        for (int64_t g0 = tid; g0 < groups; g0 += nthreads * kUnroll4) {
+            uint32_t w[kUnroll4][GW];
 #pragma unroll
-        for (int u = 0; u < kUnroll; ++u) {
-            const int64_t g = g0 + (int64_t)u * nthreads;
-            if (g < groups) {
-                if constexpr (GW == 1) {
-                    w[u][0] = ld_stream_u32(packed + g);
-                } else if constexpr (GW == 2) {
-                    uint2 t = ld_stream_u2(reinterpret_cast<const uint2 *>(packed) + g);
-                    w[u][0] = t.x;
-                    w[u][1] = t.y;
-                } else {
-                    uint4 t = ld_stream_u4(reinterpret_cast<const uint4 *>(packed) + g);
-                    w[u][0] = t.x;
-                    w[u][1] = t.y;
-                    w[u][2] = t.z;
-                    w[u][3] = t.w;
+            for (int u = 0; u < kUnroll4; ++u) {
+                const int64_t g = g0 + (int64_t)u * nthreads;
+                if (g < groups) {
+                    if constexpr (GW == 1) {
+                        w[u][0] = ld_stream_u32(packed + g);
+                    } else {
+                        const uint2 t = ld_stream_u2(reinterpret_cast<const uint2 *>(packed) + g);
+                        w[u][0] = t.x;
+                        w[u][1] = t.y;
+                    }
                 }
             }
+#pragma unroll
+            for (int u = 0; u < kUnroll4; ++u) {
+                const int64_t g = g0 + (int64_t)u * nthreads;
+                if (g >= groups) break;
+                float f[4];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) f[i] = value<BITS>((w[u][i / K] >> (BITS * (i % K))) & FIELD);
+                x4[g] = make_float4(f[0], f[1], f[2], f[3]);
+            }
         }
+        if (tid == nthreads - 1)
+            for (int64_t i = groups * 4; i < n; ++i) x[i] = value<BITS>((packed[i / K] >> (BITS * (i % K))) & FIELD);
+    } else {
+        // FP10: a warp decodes 128 consecutive words (384 values): lane l loads words
+        // [4l, 4l+4) as one uint4, writes its 12 values to shared memory, and the warp stores
+        // the 384 values back as 96 contiguous float4 (3 coalesced waves), instead of 48-byte
+        // strided stores that leave every write sector half-filled.
+        __shared__ __align__(16) float s_buf[kDprThreads / 32][384];
+        const int lane = threadIdx.x & 31;
+        float *buf = s_buf[threadIdx.x >> 5];
+        const int64_t chunks = n / 384;
+        const int64_t gwarp = tid >> 5, nwarps = nthreads >> 5;
+        for (int64_t c = gwarp; c < chunks; c += nwarps) {
+            const uint4 t = ld_stream_u4(reinterpret_cast<const uint4 *>(packed + c * 128) + lane);
+            const uint32_t w[4] = {t.x, t.y, t.z, t.w};
+            float f[12];
 #pragma unroll
-        for (int u = 0; u < kUnroll; ++u) {
-            const int64_t g = g0 + (int64_t)u * nthreads;
-            if (g >= groups) break;
-            float f[GF];
+            for (int i = 0; i < 12; ++i) f[i] = value<10>((w[i / 3] >> (10 * (i % 3))) & FIELD);
+            float4 *b4 = reinterpret_cast<float4 *>(buf);
 #pragma unroll
-            for (int i = 0; i < GF; ++i) f[i] = value<BITS>((w[u][i / K] >> (BITS * (i % K))) & FIELD);
+            for (int q = 0; q < 3; ++q) b4[3 * lane + q] = make_float4(f[4 * q], f[4 * q + 1], f[4 * q + 2], f[4 * q + 3]);
+            __syncwarp();
 #pragma unroll
-            for (int q = 0; q < GF / 4; ++q)
-                x4[g * (GF / 4) + q] = make_float4(f[4 * q], f[4 * q + 1], f[4 * q + 2], f[4 * q + 3]);
+            for (int q = 0; q < 3; ++q) x4[c * 96 + 32 * q + lane] = b4[32 * q + lane];
+            __syncwarp();
         }
-    }
-    if (tid == nthreads - 1) {
-        for (int64_t i = groups * GF; i < n; ++i) x[i] = value<BITS>((packed[i / K] >> (BITS * (i % K))) & FIELD);
+        if (tid == nthreads - 1)
+            for (int64_t i = chunks * 384; i < n; ++i) x[i] = value<10>((packed[i / 3] >> (10 * (i % 3))) & FIELD);
     }
 }
 
 template <int BITS>
 int64_t dpr_blocks(int64_t n) {
     constexpr int GF = (BITS == 10) ? 12 : 4;
+    constexpr int U = (BITS == 10) ? kUnroll : kUnroll4;
     int64_t groups = n / GF + 1;
-    int64_t blocks = ceil_div(ceil_div(groups, kUnroll), kDprThreads);
+    int64_t blocks = ceil_div(ceil_div(groups, U), kDprThreads);
     const int64_t cap = (int64_t)num_sms() * 8;
     return blocks > cap ? cap : blocks;
 }

@@ -125,6 +125,124 @@ maxpool_fwd_k2s2_kernel(const float *__restrict__ y, PoolArgs a, float *__restri
     }
 }
 
+// ---- 2x2 stride 2, no padding, W % 4 == 0 (every VGG16 / most OverFeat sites): one thread
+// per PAIR of adjacent outputs = one 2x4 input block, so both input rows are single aligned
+// float4 accesses.  Flat output row R = o / Wo needs one fast division; when H is even the
+// window's top input row is simply 2R.  Four consecutive lanes own one argmax word.
+constexpr int kPairU = 2;
+
+template <bool EVEN_H>
+__device__ __forceinline__ int64_t pair_top_left(const PoolArgs &a, uint32_t o, uint32_t &R, uint32_t &ow) {
+    a.div_wo.divmod(o, R, ow);
+    if (EVEN_H) return (int64_t)(2 * R) * a.W + 2 * ow;
+    uint32_t nc, oh;
+    a.div_ho.divmod(R, nc, oh);
+    return ((int64_t)nc * a.H + 2 * oh) * a.W + 2 * ow;
+}
+
+__device__ __forceinline__ void win4(float t0, float t1, float b0, float b1, float &best, uint32_t &bi) {
+    float m = -CUDART_INF_F;
+    int k = 0;
+    take(t0, 0, m, k);
+    take(t1, 1, m, k);
+    take(b0, 2, m, k);
+    take(b1, 3, m, k);
+    best = m;
+    bi = (uint32_t)k;
+}
+
+template <bool EVEN_H>
+__global__ void __launch_bounds__(kPoolThreads)
+maxpool_fwd_k2s2_pair_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ out,
+                             uint32_t *__restrict__ arg) {
+    const int lane = threadIdx.x & 31;
+    const int64_t pairs = (int64_t)a.n_out / 2;
+    const int64_t chunks = (pairs + 31) / 32;
+    const int64_t nwarps = ((int64_t)gridDim.x * kPoolThreads) >> 5;
+    for (int64_t c0 = (((int64_t)blockIdx.x * kPoolThreads + threadIdx.x) >> 5) * kPairU; c0 < chunks;
+         c0 += nwarps * kPairU) {
+        float4 t[kPairU], b[kPairU];
+#pragma unroll
+        for (int u = 0; u < kPairU; ++u) {
+            const int64_t q = (c0 + u) * 32 + lane;
+            if (q < pairs) {
+                uint32_t R, ow;
+                const int64_t i0 = pair_top_left<EVEN_H>(a, (uint32_t)(2 * q), R, ow);
+                t[u] = ld_stream_f4(reinterpret_cast<const float4 *>(y + i0));
+                b[u] = ld_stream_f4(reinterpret_cast<const float4 *>(y + i0 + a.W));
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < kPairU; ++u) {
+            const int64_t q = (c0 + u) * 32 + lane;
+            uint32_t byte = 0;
+            if (q < pairs) {
+                float m0, m1;
+                uint32_t k0, k1;
+                win4(t[u].x, t[u].y, b[u].x, b[u].y, m0, k0);
+                win4(t[u].z, t[u].w, b[u].z, b[u].w, m1, k1);
+                reinterpret_cast<float2 *>(out)[q] = make_float2(m0, m1);
+                byte = (k0 | (k1 << 4)) << (8 * (lane & 3));
+            }
+            byte |= __shfl_xor_sync(kFull, byte, 1);
+            byte |= __shfl_xor_sync(kFull, byte, 2);
+            if ((lane & 3) == 0 && q < pairs) arg[q >> 2] = byte;
+        }
+    }
+}
+
+template <bool EVEN_H>
+__global__ void __launch_bounds__(kPoolThreads)
+pool_bwd_k2s2_pair_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
+                          const uint32_t *__restrict__ mask, PoolArgs a, float *__restrict__ dx) {
+    const int64_t pairs = (int64_t)a.n_out / 2;
+    const int64_t stride = (int64_t)gridDim.x * kPoolThreads;
+    for (int64_t q0 = (int64_t)blockIdx.x * kPoolThreads + threadIdx.x; q0 < pairs; q0 += stride * kPairU) {
+        float2 g[kPairU];
+        uint32_t nb[kPairU], m0[kPairU], m1[kPairU], R[kPairU], ow[kPairU];
+        int64_t i0[kPairU];
+#pragma unroll
+        for (int u = 0; u < kPairU; ++u) {
+            const int64_t q = q0 + u * stride;
+            if (q < pairs) {
+                i0[u] = pair_top_left<EVEN_H>(a, (uint32_t)(2 * q), R[u], ow[u]);
+                g[u] = ld_stream_f2(reinterpret_cast<const float2 *>(dout) + q);
+                nb[u] = ld_ro(arg + (q >> 2)) >> (8 * (q & 3));
+                if (mask) {
+                    m0[u] = ld_ro(mask + (i0[u] >> 5)) >> (i0[u] & 31);
+                    m1[u] = ld_ro(mask + ((i0[u] + a.W) >> 5)) >> ((i0[u] + a.W) & 31);
+                } else {
+                    m0[u] = m1[u] = 0xfu;
+                }
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < kPairU; ++u) {
+            const int64_t q = q0 + u * stride;
+            if (q >= pairs) break;
+            const float v0 = 0.0f + g[u].x, v1 = 0.0f + g[u].y;  // R6: +0.0f + dY
+            const uint32_t k0 = nb[u] & 0xfu, k1 = (nb[u] >> 4) & 0xfu;
+            float4 top, bot;
+            top.x = (k0 == 0 && (m0[u] & 1u)) ? v0 : 0.0f;
+            top.y = (k0 == 1 && (m0[u] & 2u)) ? v0 : 0.0f;
+            top.z = (k1 == 0 && (m0[u] & 4u)) ? v1 : 0.0f;
+            top.w = (k1 == 1 && (m0[u] & 8u)) ? v1 : 0.0f;
+            bot.x = (k0 == 2 && (m1[u] & 1u)) ? v0 : 0.0f;
+            bot.y = (k0 == 3 && (m1[u] & 2u)) ? v0 : 0.0f;
+            bot.z = (k1 == 2 && (m1[u] & 4u)) ? v1 : 0.0f;
+            bot.w = (k1 == 3 && (m1[u] & 8u)) ? v1 : 0.0f;
+            *reinterpret_cast<float4 *>(dx + i0[u]) = top;
+            *reinterpret_cast<float4 *>(dx + i0[u] + a.W) = bot;
+            if (!EVEN_H) {  // floor mode, odd H: zero the plane's uncovered last input row
+                uint32_t nc, oh;
+                a.div_ho.divmod(R[u], nc, oh);
+                if ((int)oh == a.Ho - 1)
+                    *reinterpret_cast<float4 *>(dx + i0[u] + 2 * (int64_t)a.W) = make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+        }
+    }
+}
+
 __device__ __forceinline__ uint32_t nibble(const uint32_t *__restrict__ arg, int64_t o) {
     return (ld_ro(arg + (o >> 3)) >> (4 * (o & 7))) & 0xfu;
 }
@@ -264,7 +382,11 @@ cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, 
                                int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, cudaStream_t s) {
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
     const unsigned grid = grid_for(a.n_out, kPoolThreads, 8);
-    if (is_k2s2_exact(p, H, W, Ho, Wo))
+    if (is_k2s2_exact(p, H, W, Ho, Wo) && W % 4 == 0) {
+        const unsigned g2 = grid_for(ceil_div(a.n_out / 2, 32 * kPairU), kPoolThreads / 32, 8);
+        if (H == 2 * Ho) maxpool_fwd_k2s2_pair_kernel<true><<<g2, kPoolThreads, 0, s>>>(y, a, out, argmax);
+        else maxpool_fwd_k2s2_pair_kernel<false><<<g2, kPoolThreads, 0, s>>>(y, a, out, argmax);
+    } else if (is_k2s2_exact(p, H, W, Ho, Wo))
         maxpool_fwd_k2s2_kernel<<<grid_for(ceil_div(a.n_out, kFwdU), kPoolThreads, 8), kPoolThreads, 0, s>>>(y, a, out, argmax);
     else if (p.kh == 3 && p.kw == 3)
         maxpool_fwd_kernel<3, 3><<<grid, kPoolThreads, 0, s>>>(y, a, out, argmax);
@@ -279,7 +401,11 @@ cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uin
                             int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo, float *dx,
                             cudaStream_t s) {
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
-    if (is_k2s2_exact(p, H, W, Ho, Wo)) {
+    if (is_k2s2_exact(p, H, W, Ho, Wo) && W % 4 == 0) {
+        const unsigned g2 = grid_for(ceil_div(a.n_out / 2, kPairU), kPoolThreads, 8);
+        if (H == 2 * Ho) pool_bwd_k2s2_pair_kernel<true><<<g2, kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+        else pool_bwd_k2s2_pair_kernel<false><<<g2, kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+    } else if (is_k2s2_exact(p, H, W, Ho, Wo)) {
         pool_bwd_k2s2_kernel<<<grid_for(ceil_div(a.n_out, kBwdU), kPoolThreads, 8), kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
     } else {
         const unsigned grid = grid_for(a.n_in, kPoolThreads, 8);
