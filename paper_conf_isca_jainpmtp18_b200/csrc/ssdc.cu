@@ -2,20 +2,21 @@
 //
 // Encode: dense fp32 -> CSR with 256-column rows and uint8 column indices (Narrow Value
 // Optimization).  One pass over x (4n bytes read, 5*nnz + 4*rows written).
-// Persistent, warp-specialized CTAs (3 per SM) stream 16-row tiles (4096 elements, 16 KB)
-// through a 4-stage shared-memory ring filled by 1-D TMA bulk copies (cp.async.bulk +
-// mbarrier).  Tiles are claimed in order through an atomic ticket, so every predecessor of a
-// tile is held by a running CTA (forward progress).  Roles, linked only by mbarriers:
-//   * counter warp: as soon as a tile lands, counts the nonzero bit patterns of its rows
-//     (R8), scans the 16 row counts and publishes the tile aggregate — aggregates appear one
-//     TMA latency after the ticket, independent of how far the writers are;
-//   * look-back warp: decoupled look-back (32 predecessors' 64-bit {status, value}
-//     descriptors per round) -> the tile's global offset; publishes the inclusive prefix and
-//     the tile's row_end entries;
-//   * 4 writer warps: each holds 4 rows in registers (lane: cols [4l,4l+4) and
-//     [128+4l,128+4l+4)), takes ranks from warp ballots, compacts the whole tile in place,
-//     shifted to the global 16-byte phase, and lane 0 of warp 0 writes the aligned bodies of
-//     val/col with TMA bulk stores (cp.async.bulk.global.shared::cta); ragged ends by lanes.
+// Persistent, warp-specialized CTAs (2 per SM, 9 warps), all roles linked by mbarriers:
+//   * producer warp: claims tiles (16 rows = 4096 elements = 16 KB) in ticket order — so every
+//     predecessor of a tile is held by a running CTA (forward progress) — and keeps a 4-stage
+//     raw ring full with 1-D TMA bulk copies (cp.async.bulk + mbarrier complete_tx);
+//   * counter warp: as soon as a tile lands, counts the nonzero bit patterns of its rows (R8),
+//     scans the 16 row counts and publishes the tile aggregate (so aggregates appear one TMA
+//     latency after the ticket);
+//   * look-back warp: decoupled look-back over 64-bit {status, value} descriptors, 32 per
+//     round -> the tile's global offset; publishes the inclusive prefix and row_end;
+//   * 4 compactor warps: rank nonzeros with warp ballots (lane l holds cols [4l,4l+4) and
+//     [128+4l,128+4l+4)), move them into a variable-size pending ring in shared memory and
+//     release the raw stage at once — the raw ring turns over at TMA speed while compacted
+//     tiles (~1/5 of the raw bytes at 80% sparsity) wait for their offsets;
+//   * 2 store warps: copy each resolved tile from the pending ring to val/col with coalesced
+//     stores, then release its ring space and queue slot, in order.
 // Decode: a warp expands 4 consecutive rows (whose entries are one contiguous range)
 //   through a 4 KB shared-memory row buffer and writes them back with float4 stores.
 #include "common.cuh"
@@ -57,34 +58,46 @@ __global__ void ssdc_ws_init(uint64_t *ws, int64_t words) {
         ws[i] = 0ull;
 }
 
-constexpr int kStages = 4;                       // TMA ring depth per CTA
-constexpr int kCtasPerSm = 3;                    // smem/register-limited residency
+constexpr int kStages = 4;                       // raw TMA ring (16 KB tiles)
+constexpr int kRing = 8192;                      // pending ring entries (compacted, awaiting offset)
+constexpr int kQ = 16;                           // per-CTA tile queue slots (counted .. stored)
+constexpr int kCtasPerSm = 2;
 constexpr int kTileElems = kTileRows * kRow;     // 4096 elements
 constexpr uint32_t kTileBytes = kTileElems * 4;  // 16 KB
-constexpr int kWarps = kEncThreads / 32;         // writer warps (4 rows each)
+constexpr int kWarps = kEncThreads / 32;         // compactor warps (4 rows each)
 constexpr int kCountWarp = kWarps;               // counts every tile as soon as it lands
-constexpr int kLbWarp = kWarps + 1;              // first of kLbWarps look-back warps
-constexpr int kLbWarps = 1;                      // (more take alternate tiles)
-constexpr int kCtaThreads = kEncThreads + 32 + 32 * kLbWarps;
+constexpr int kLbWarp = kWarps + 1;              // decoupled look-back
+constexpr int kProdWarp = kWarps + 2;            // claims tickets, issues TMA loads
+constexpr int kStoreWarp = kWarps + 3;           // first of kStoreWarps store warps
+constexpr int kStoreWarps = 2;
+constexpr int kCtaThreads = 32 * (kStoreWarp + kStoreWarps);
 
 struct __align__(128) EncSmem {
-    float tile[kStages][kTileElems + 4];    // TMA destinations; the written tile is compacted in place
-    uint8_t colbuf[kTileElems + 16];        // compacted column bytes of the tile being written
-    uint64_t full[kStages];                 // TMA landed (or no tile: arrive without bytes)
-    uint64_t counted[kStages];              // counter warp -> look-back warp
-    uint64_t resolved[kStages];             // look-back warp -> writers
-    int64_t ticket[kStages];                // tile index held by each stage
-    uint32_t row_cnt[kStages][kTileRows];   // per-row nonzeros
-    uint32_t row_excl[kStages][kTileRows];  // tile-local exclusive row offsets
-    int64_t excl[kStages];                  // global offset of each stage's tile
-    int32_t last_j;                         // CTA-local index of the first "no tile" ticket
+    float tile[kStages][kTileElems];  // raw tiles (TMA destinations)
+    float vring[kRing];               // compacted values, tile-local order
+    uint8_t cring[kRing];             // compacted column bytes
+    uint64_t full[kStages];           // TMA landed (or "no tile" arrival)
+    uint64_t empty[kStages];          // compactors done with the raw tile
+    uint64_t counted[kQ];             // counter -> look-back, compactors
+    uint64_t resolved[kQ];            // look-back -> storers
+    uint64_t compacted[kQ];           // compactors -> storers
+    int64_t st_ticket[kStages];       // tile index per raw stage
+    int64_t q_ticket[kQ];             // tile index per queue slot
+    uint32_t row_cnt[kQ][kTileRows];  // per-row nonzeros
+    uint32_t row_excl[kQ][kTileRows]; // tile-local exclusive row offsets
+    uint32_t total[kQ];               // tile nonzeros
+    int64_t excl[kQ];                 // global offset of the tile
+    uint32_t pos[kQ];                 // ring offset of the tile's compacted entries
+    int64_t ring_end[kQ];             // monotonic ring position after the tile
+    int64_t alloc_pos;                // monotonic ring allocation cursor (compactor leader)
+    volatile int64_t free_pos;        // monotonic ring release cursor (storers)
+    volatile int32_t stored;          // tiles fully stored by this CTA
 };
 
-// Start the TMA bulk load of tile t (a ticket claimed earlier, in order, so every predecessor
-// is held by a running CTA) into stage s.  Always completes one arrival on full[s], so the
-// counter warp also learns about "no more tiles".  One thread.
+// Start the TMA bulk load of tile t (claimed in ticket order) into stage s; always one arrival
+// on full[s] (zero bytes when there is no tile), so consumers also learn about the end.
 __device__ __forceinline__ void load_tile(EncSmem &S, int s, int64_t t, const float *x, int64_t n, int64_t tiles) {
-    S.ticket[s] = t;
+    S.st_ticket[s] = t;
     uint32_t bytes = 0;
     if (t < tiles) {
         const int64_t avail = n - t * kTileElems;
@@ -122,7 +135,8 @@ __device__ __forceinline__ int64_t look_back(const Workspace *ws, int64_t tile, 
     }
 }
 
-__device__ __forceinline__ void writers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kEncThreads) : "memory"); }
+__device__ __forceinline__ void compactors_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kEncThreads) : "memory"); }
+__device__ __forceinline__ void storers_sync() { asm volatile("bar.sync 2, %0;" ::"n"(32 * kStoreWarps) : "memory"); }
 
 __global__ void __launch_bounds__(kCtaThreads, kCtasPerSm)
 ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t tiles,
@@ -136,21 +150,40 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
     if (threadIdx.x == 0) {
         for (int s = 0; s < kStages; ++s) {
             mbar_init(&S.full[s], 1);
-            mbar_init(&S.counted[s], 1);
-            mbar_init(&S.resolved[s], 1);
+            mbar_init(&S.empty[s], kWarps);
         }
+        for (int q = 0; q < kQ; ++q) {
+            mbar_init(&S.counted[q], 1);
+            mbar_init(&S.resolved[q], 1);
+            mbar_init(&S.compacted[q], kWarps);
+        }
+        S.alloc_pos = 0;
+        S.free_pos = 0;
+        S.stored = 0;
         fence_mbar_init();
-        S.last_j = 0x7fffffff;
-        for (int s = 0; s < kStages; ++s) load_tile(S, s, atomicAdd(&ws->ticket, 1u), x, n, tiles);
     }
     __syncthreads();
 
-    if (warp == kCountWarp) {
+    if (warp == kProdWarp) {
+        // ---- producer: keep the raw ring full, in ticket order
+        if (lane == 0) {
+            for (int j = 0;; ++j) {
+                const int s = j % kStages;
+                if (j >= kStages) mbar_wait(&S.empty[s], (uint32_t)(j / kStages - 1) & 1u);
+                const int64_t t = atomicAdd(&ws->ticket, 1u);
+                load_tile(S, s, t, x, n, tiles);
+                if (t >= tiles) break;
+            }
+        }
+    } else if (warp == kCountWarp) {
         // ---- counter: nonzero bit patterns (R8) of every row, tile scan, publish aggregate
         for (int j = 0;; ++j) {
-            const int s = j % kStages;
+            const int s = j % kStages, q = j % kQ;
             mbar_wait(&S.full[s], (uint32_t)(j / kStages) & 1u);
-            const int64_t tile = S.ticket[s];
+            while (j - S.stored >= kQ) {  // queue slot still held by a tile not yet stored
+            }
+            const int64_t tile = S.st_ticket[s];
+            if (lane == 0) S.q_ticket[q] = tile;
             if (tile < tiles) {
                 float *T = S.tile[s];
                 if (tile == tiles - 1) {  // ragged last tile: tail the TMA could not copy, zeros
@@ -177,125 +210,132 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                     if (lane >= d) inc += t;
                 }
                 if (lane < kTileRows) {
-                    S.row_cnt[s][lane] = mine;
-                    S.row_excl[s][lane] = inc - mine;
+                    S.row_cnt[q][lane] = mine;
+                    S.row_excl[q][lane] = inc - mine;
                 }
-                if (lane == 31) st_relaxed(&ws->desc[tile], (tile == 0 ? kStatusP : kStatusA) | (uint64_t)inc);
+                if (lane == 31) {
+                    S.total[q] = inc;
+                    st_relaxed(&ws->desc[tile], (tile == 0 ? kStatusP : kStatusA) | (uint64_t)inc);
+                }
             }
             __syncwarp();
-            if (lane == 0) {
-                if (tile >= tiles) *(volatile int32_t *)&S.last_j = j;  // before the arrival
-                mbar_arrive(&S.counted[s]);
-            }
+            if (lane == 0) mbar_arrive(&S.counted[q]);
             if (tile >= tiles) break;
         }
-    } else if (warp >= kLbWarp) {
-        // ---- look-back: global offset of each counted tile; publish prefix, row ends, nnz.
-        // Warp kLbWarp + i resolves the CTA's tiles j = i, i + kLbWarps, ...
-        for (int j = warp - kLbWarp;; j += kLbWarps) {
-            const int s = j % kStages;
-            // poll: past the CTA's last tile no arrival will ever come for this j
-            bool ready = false;
-            while (!(ready = mbar_test(&S.counted[s], (uint32_t)(j / kStages) & 1u)))
-                if (*(volatile int32_t *)&S.last_j < j) break;
-            if (!ready) break;
-            const int64_t tile = S.ticket[s];
+    } else if (warp == kLbWarp) {
+        // ---- look-back: global offset of each counted tile; publish prefix, row ends, nnz
+        for (int j = 0;; ++j) {
+            const int q = j % kQ;
+            mbar_wait(&S.counted[q], (uint32_t)(j / kQ) & 1u);
+            const int64_t tile = S.q_ticket[q];
             if (tile < tiles) {
                 const int64_t excl = (tile == 0) ? 0 : look_back(ws, tile, lane);
-                const uint32_t total = S.row_excl[s][kTileRows - 1] + S.row_cnt[s][kTileRows - 1];
+                const uint32_t total = S.total[q];
                 if (lane == 0) {
-                    S.excl[s] = excl;
+                    S.excl[q] = excl;
                     if (tile > 0) st_relaxed(&ws->desc[tile], kStatusP | (uint64_t)(excl + total));
                     if (tile == tiles - 1) *nnz_out = excl + total;
                 }
                 const int64_t r = tile * kTileRows + lane;
-                if (lane < kTileRows && r < rows)
-                    row_end[r] = (int32_t)(excl + S.row_excl[s][lane] + S.row_cnt[s][lane]);
+                if (lane < kTileRows && r < rows) row_end[r] = (int32_t)(excl + S.row_excl[q][lane] + S.row_cnt[q][lane]);
             }
             __syncwarp();
-            if (lane == 0) mbar_arrive(&S.resolved[s]);
+            if (lane == 0) mbar_arrive(&S.resolved[q]);
             if (tile >= tiles) break;
         }
-    } else {
-        // ---- writers: compact the tile contiguously in place, shifted so smem and global share
-        // their 16-byte phase (value k -> T[sv + k] = val[excl + k], column -> colbuf[sc + k]),
-        // then TMA bulk-store the aligned bodies; ranks from ballots (lane l holds cols 4l+j
-        // "lo" and 128+4l+j "hi", j = 0..3).
+    } else if (warp < kWarps) {
+        // ---- compactors: move the tile's nonzeros into the pending ring (tile-local order),
+        // then release the raw stage at once.  Ranks from ballots: lane l holds cols 4l+k
+        // ("lo") and 128+4l+k ("hi"), k = 0..3.
         const uint32_t lt = (1u << lane) - 1u;
         for (int j = 0;; ++j) {
-            const int s = j % kStages;
-            mbar_wait(&S.resolved[s], (uint32_t)(j / kStages) & 1u);
-            const int64_t tile = S.ticket[s];
+            const int s = j % kStages, q = j % kQ;
+            mbar_wait(&S.counted[q], (uint32_t)(j / kQ) & 1u);
+            const int64_t tile = S.q_ticket[q];
             if (tile >= tiles) break;
-            float *T = S.tile[s];
-            const int64_t excl = S.excl[s];
-            const uint32_t sv = (uint32_t)excl & 3u, sc = (uint32_t)excl & 15u;
-            float v[kRowsPerWarp][8];
-            uint32_t bal[kRowsPerWarp][8];
-#pragma unroll
-            for (int r = 0; r < kRowsPerWarp; ++r) {
-                const float4 *row4 = reinterpret_cast<const float4 *>(T + (warp * kRowsPerWarp + r) * kRow);
-                const float4 a = row4[lane], b = row4[32 + lane];
-                v[r][0] = a.x; v[r][1] = a.y; v[r][2] = a.z; v[r][3] = a.w;
-                v[r][4] = b.x; v[r][5] = b.y; v[r][6] = b.z; v[r][7] = b.w;
-#pragma unroll
-                for (int k = 0; k < 8; ++k) bal[r][k] = __ballot_sync(kFull, __float_as_uint(v[r][k]) != 0u);
+            if (threadIdx.x == 0) {  // allocate T contiguous ring entries (skip the ring end)
+                const uint32_t T = S.total[q];
+                int64_t p = S.alloc_pos;
+                const int64_t pm = p % kRing;
+                if (pm + T > kRing) p += kRing - pm;
+                while (p + T - S.free_pos > kRing) {
+                }
+                S.pos[q] = (uint32_t)(p % kRing);
+                S.ring_end[q] = p + T;
+                S.alloc_pos = p + T;
             }
-            writers_sync();  // whole tile in registers (and the previous bulk store read out)
+            compactors_sync();
+            const float *Tr = S.tile[s];
+            float *vr = S.vring + S.pos[q];
+            uint8_t *cr = S.cring + S.pos[q];
 #pragma unroll
             for (int r = 0; r < kRowsPerWarp; ++r) {
-                const uint32_t q0 = sv + S.row_excl[s][warp * kRowsPerWarp + r];
-                uint32_t p_lo = q0 + __popc(bal[r][0] & lt) + __popc(bal[r][1] & lt) + __popc(bal[r][2] & lt) +
-                                __popc(bal[r][3] & lt);
-                uint32_t p_hi = q0 + __popc(bal[r][0]) + __popc(bal[r][1]) + __popc(bal[r][2]) + __popc(bal[r][3]) +
-                                __popc(bal[r][4] & lt) + __popc(bal[r][5] & lt) + __popc(bal[r][6] & lt) +
-                                __popc(bal[r][7] & lt);
-                uint8_t *cb = S.colbuf + sc - sv;
+                const int rr = warp * kRowsPerWarp + r;
+                const float4 *row4 = reinterpret_cast<const float4 *>(Tr + rr * kRow);
+                const float4 a = row4[lane], b = row4[32 + lane];
+                const float v[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+                uint32_t bal[8];
+#pragma unroll
+                for (int k = 0; k < 8; ++k) bal[k] = __ballot_sync(kFull, __float_as_uint(v[k]) != 0u);
+                const uint32_t q0 = S.row_excl[q][rr];
+                uint32_t p_lo = q0 + __popc(bal[0] & lt) + __popc(bal[1] & lt) + __popc(bal[2] & lt) + __popc(bal[3] & lt);
+                uint32_t p_hi = q0 + __popc(bal[0]) + __popc(bal[1]) + __popc(bal[2]) + __popc(bal[3]) +
+                                __popc(bal[4] & lt) + __popc(bal[5] & lt) + __popc(bal[6] & lt) + __popc(bal[7] & lt);
 #pragma unroll
                 for (int k = 0; k < 4; ++k) {
-                    const uint32_t on = (bal[r][k] >> lane) & 1u;
+                    const uint32_t on = (bal[k] >> lane) & 1u;
                     if (on) {
-                        T[p_lo] = v[r][k];
-                        cb[p_lo] = (uint8_t)(4 * lane + k);
+                        vr[p_lo] = v[k];
+                        cr[p_lo] = (uint8_t)(4 * lane + k);
                     }
                     p_lo += on;
                 }
 #pragma unroll
                 for (int k = 0; k < 4; ++k) {
-                    const uint32_t on = (bal[r][4 + k] >> lane) & 1u;
+                    const uint32_t on = (bal[4 + k] >> lane) & 1u;
                     if (on) {
-                        T[p_hi] = v[r][4 + k];
-                        cb[p_hi] = (uint8_t)(128 + 4 * lane + k);
+                        vr[p_hi] = v[4 + k];
+                        cr[p_hi] = (uint8_t)(128 + 4 * lane + k);
                     }
                     p_hi += on;
                 }
             }
-            fence_proxy_async_smem();  // generic smem writes before the async-proxy bulk store
-            writers_sync();
-            if (warp == 0) {
-                const int64_t total = S.row_excl[s][kTileRows - 1] + S.row_cnt[s][kTileRows - 1];
-                int64_t lim = total;
-                if (excl + lim > capacity) lim = capacity > excl ? capacity - excl : 0;
-                const int64_t hv = (4 - sv) & 3, hc = (16 - sc) & 15;  // heads up to 16-B alignment
-                const int64_t bv = lim > hv ? (lim - hv) & ~3ll : 0, bc = lim > hc ? (lim - hc) & ~15ll : 0;
-                // ragged ends: < 4 values and < 16 columns at each end
-                const int64_t k0 = lane, k1 = hv + bv + lane, k2 = hc + bc + lane;
-                if (k0 < hv && k0 < lim) val[excl + k0] = T[sv + k0];
-                if (lane < 4 && k1 < lim) val[excl + k1] = T[sv + k1];
-                if (k0 < hc && k0 < lim) col[excl + k0] = S.colbuf[sc + k0];
-                if (lane < 16 && k2 < lim) col[excl + k2] = S.colbuf[sc + k2];
-                __syncwarp();
-                if (lane == 0) {
-                    if (bv) tma_store_1d(val + excl + hv, T + sv + hv, (uint32_t)(4 * bv));
-                    if (bc) tma_store_1d(col + excl + hc, S.colbuf + sc + hc, (uint32_t)bc);
-                    bulk_commit();
-                    bulk_wait_read();  // stage + colbuf read out
-                    load_tile(S, s, atomicAdd(&ws->ticket, 1u), x, n, tiles);  // refill this stage
-                }
-                __syncwarp();
+            fence_proxy_async_smem();  // our reads of the raw stage precede the next TMA write
+            __syncwarp();
+            if (lane == 0) {
+                mbar_arrive(&S.empty[s]);
+                mbar_arrive(&S.compacted[q]);
             }
         }
-        if (threadIdx.x == 0) bulk_wait_all();
+    } else {
+        // ---- storers: once a tile is compacted and resolved, copy its entries to val/col
+        // (coalesced), then release its ring space and queue slot, in order.
+        const int sl = threadIdx.x - 32 * kStoreWarp;
+        for (int j = 0;; ++j) {
+            const int q = j % kQ;
+            const uint32_t par = (uint32_t)(j / kQ) & 1u;
+            mbar_wait(&S.resolved[q], par);
+            const int64_t tile = S.q_ticket[q];
+            if (tile >= tiles) break;
+            mbar_wait(&S.compacted[q], par);
+            const int64_t excl = S.excl[q];
+            int64_t lim = S.total[q];
+            if (excl + lim > capacity) lim = capacity > excl ? capacity - excl : 0;
+            const float *vr = S.vring + S.pos[q];
+            const uint8_t *cr = S.cring + S.pos[q];
+            float *vo = val + excl;
+            uint8_t *co = col + excl;
+#pragma unroll 4
+            for (int k = sl; k < (int)lim; k += 32 * kStoreWarps) {
+                vo[k] = vr[k];
+                co[k] = cr[k];
+            }
+            storers_sync();
+            if (sl == 0) {
+                S.free_pos = S.ring_end[q];
+                S.stored = j + 1;
+            }
+        }
     }
 }
 
