@@ -402,6 +402,9 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=8.0)
     ap.add_argument("--kernels-out", default=None, help="write the per-kernel breakdown JSON here")
+    ap.add_argument("--same-device", action="store_true",
+                    help="testing only: put every rank on cuda:0 and tally over gloo (exercises the N>1 "
+                         "path on a 1-GPU box)")
     args = ap.parse_args()
     cfg = WL.CONFIGS[args.config]
     args.sparsity = cfg.sparsity if args.sparsity is None else args.sparsity
@@ -417,12 +420,15 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    dev = torch.device("cuda", local)
+    dev = torch.device("cuda", 0 if args.same_device else local)
     torch.cuda.set_device(dev)
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        if args.same_device:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
 
     def barrier():
         if dist is not None:
@@ -474,15 +480,12 @@ def main():
     dom = max(per, key=lambda kk: per[kk]["ms"])
     dom_gbs = per[dom]["algo_bytes"] / (per[dom]["ms"] * 1e-3) / 1e9
 
-    # ---- multi-rank: max time over ranks, sum of bytes (NCCL, outside the timed region)
-    total_bytes = wl.bytes_per_step * args.steps
-    if dist is not None:
-        t = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        elapsed_ms = float(t.item())
-        tally = torch.tensor([total_bytes, sum(nnz)], dtype=torch.int64, device=dev)
-        dist.all_reduce(tally, op=dist.ReduceOp.SUM)
-        total_bytes = int(tally[0].item())
+    # ---- multi-rank: max time over ranks, sum of bytes (one collective, outside the timed region)
+    from paper_conf_isca_jainpmtp18_b200.shard import tally
+    tdev = torch.device("cpu") if (dist is not None and args.same_device) else dev
+    totals, elapsed_ms = tally(dist, {"fp32_bytes": wl.bytes_per_step * args.steps, "nnz": sum(nnz)}, elapsed_ms,
+                               device=tdev)
+    total_bytes = totals["fp32_bytes"]
     value = total_bytes / (elapsed_ms * 1e-3) / 1e9
 
     # ---- e2e: host pinned inputs -> H2D -> the same C-ABI calls -> D2H of the nnz tally
@@ -511,12 +514,8 @@ def main():
         b.record(stream)
         barrier()
         e_ms = a.elapsed_time(b)
-        e_bytes = wl.bytes_per_step * e_steps
-        if dist is not None:
-            t = torch.tensor([e_ms], dtype=torch.float64, device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            e_ms = float(t.item())
-            e_bytes *= world
+        e_tot, e_ms = tally(dist, {"fp32_bytes": wl.bytes_per_step * e_steps}, e_ms, device=tdev)
+        e_bytes = e_tot["fp32_bytes"]
         e2e = {"value": round(e_bytes / (e_ms * 1e-3) / 1e9, 3), "unit": "GB/s", "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "steps": e_steps,
                "note": "pinned host maps copied H2D each step, then the step's C-ABI calls, then D2H of the "

@@ -44,16 +44,20 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False, ptxas_v: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, ptxas_v: bool = False, defines=(), out: str | None = None) -> str:
+    """Build libgist.so.  `defines`/`out` build a tuning variant (e.g. -DGIST_SSDC_STAGES=3) into
+    another file, selected at run time with GIST_LIBRARY=<path> (developer knob only)."""
+    target = out or LIB
+    if not defines and out is None and not force and not _stale():
         return LIB
-    os.makedirs(BUILD, exist_ok=True)
+    build_dir = BUILD if not defines else os.path.join(BUILD, "variant_" + "_".join(d.strip("-D") for d in defines))
+    os.makedirs(build_dir, exist_ok=True)
     cc = nvcc()
     extra = ["-Xptxas", "-v"] if ptxas_v else []
 
     def compile_one(src):
-        obj = os.path.join(BUILD, os.path.basename(src) + ".o")
-        cmd = [cc, *NVCC_FLAGS, *extra, "-c", src, "-o", obj]
+        obj = os.path.join(build_dir, os.path.basename(src) + ".o")
+        cmd = [cc, *NVCC_FLAGS, *defines, *extra, "-c", src, "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"nvcc failed for {src}:\n{r.stderr}")
@@ -66,10 +70,10 @@ def build(force: bool = False, verbose: bool = False, ptxas_v: bool = False) -> 
             if err:
                 sys.stderr.write(err)
     objs = [o for o, _ in results]
-    tmp = LIB + f".tmp{os.getpid()}"
+    tmp = target + f".tmp{os.getpid()}"
     subprocess.check_call([cc, *ARCH, "-shared", "--cudart", "static", "-o", tmp, *objs])
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":

@@ -26,7 +26,7 @@ __all__ = [
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-library_path = os.path.join(_HERE, "libgist.so")
+library_path = os.environ.get("GIST_LIBRARY") or os.path.join(_HERE, "libgist.so")  # override: tuning variants
 
 STATUS = {0: "GIST_OK", 1: "GIST_ERR_INVALID_ARGUMENT", 2: "GIST_ERR_MISALIGNED",
           3: "GIST_ERR_UNSUPPORTED", 4: "GIST_ERR_TOO_LARGE", 5: "GIST_ERR_CUDA"}

@@ -129,7 +129,10 @@ maxpool_fwd_k2s2_kernel(const float *__restrict__ y, PoolArgs a, float *__restri
 // per PAIR of adjacent outputs = one 2x4 input block, so both input rows are single aligned
 // float4 accesses.  Flat output row R = o / Wo needs one fast division; when H is even the
 // window's top input row is simply 2R.  Four consecutive lanes own one argmax word.
-constexpr int kPairU = 2;
+#ifndef GIST_POOL_PAIR_U
+#define GIST_POOL_PAIR_U 1
+#endif
+constexpr int kPairU = GIST_POOL_PAIR_U;  // output pairs in flight per thread
 
 template <bool EVEN_H>
 __device__ __forceinline__ int64_t pair_top_left(const PoolArgs &a, uint32_t o, uint32_t &R, uint32_t &ow) {

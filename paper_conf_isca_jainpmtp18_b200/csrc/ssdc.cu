@@ -11,8 +11,8 @@
 //     latency after the ticket);
 //   * look-back warp: decoupled look-back over 64-bit {status, value} descriptors, 32 per
 //     round -> the tile's global offset; publishes the inclusive prefix and row_end;
-//   * 4 compactor warps: rank nonzeros with warp ballots (lane l holds cols [4l,4l+4) and
-//     [128+4l,128+4l+4)), move them into a variable-size pending ring in shared memory and
+//   * 4 compactor warps (4 rows each): rank nonzeros with warp ballots (lane l holds cols [4l,4l+4) and
+//     [128+4l,128+4l+4)), move them into a variable-size (wrapping) pending ring in smem and
 //     release the raw stage at once — the raw ring turns over at TMA speed while compacted
 //     tiles (~1/5 of the raw bytes at 80% sparsity) wait for their offsets;
 //   * 2 store warps: copy each resolved tile from the pending ring to val/col with coalesced
@@ -30,7 +30,7 @@ namespace gist {
 namespace {
 
 constexpr int kRow = 256;
-constexpr int kEncThreads = 128;  // worker threads (4 warps x 4 rows)
+constexpr int kEncThreads = 128;  // compactor threads (4 warps x 4 rows)
 constexpr int kRowsPerWarp = 4;
 constexpr int kTileRows = (kEncThreads / 32) * kRowsPerWarp;  // 16
 constexpr uint64_t kStatusA = 1ull << 62;                    // aggregate available
@@ -58,19 +58,42 @@ __global__ void ssdc_ws_init(uint64_t *ws, int64_t words) {
         ws[i] = 0ull;
 }
 
-constexpr int kStages = 4;                       // raw TMA ring (16 KB tiles)
-constexpr int kRing = 8192;                      // pending ring entries (compacted, awaiting offset)
+#ifndef GIST_SSDC_STAGES
+#define GIST_SSDC_STAGES 4
+#endif
+#ifndef GIST_SSDC_RING
+#define GIST_SSDC_RING 8192
+#endif
+#ifndef GIST_SSDC_CTAS
+#define GIST_SSDC_CTAS 2
+#endif
+#ifndef GIST_SSDC_COUNTERS
+#define GIST_SSDC_COUNTERS 2
+#endif
+#ifndef GIST_SSDC_LBS
+#define GIST_SSDC_LBS 2
+#endif
+constexpr int kStages = GIST_SSDC_STAGES;         // raw TMA ring (16 KB tiles)
+constexpr int kRing = GIST_SSDC_RING;            // pending ring entries (compacted, awaiting offset)
 constexpr int kQ = 16;                           // per-CTA tile queue slots (counted .. stored)
-constexpr int kCtasPerSm = 2;
+constexpr int kCtasPerSm = GIST_SSDC_CTAS;
 constexpr int kTileElems = kTileRows * kRow;     // 4096 elements
 constexpr uint32_t kTileBytes = kTileElems * 4;  // 16 KB
-constexpr int kWarps = kEncThreads / 32;         // compactor warps (4 rows each)
-constexpr int kCountWarp = kWarps;               // counts every tile as soon as it lands
-constexpr int kLbWarp = kWarps + 1;              // decoupled look-back
-constexpr int kProdWarp = kWarps + 2;            // claims tickets, issues TMA loads
-constexpr int kStoreWarp = kWarps + 3;           // first of kStoreWarps store warps
+constexpr int kWarps = kEncThreads / 32;         // compactor warps (kRowsPerWarp rows each)
+constexpr int kCountWarp = kWarps;               // first of kCountWarps counters (alternate tiles)
+constexpr int kCountWarps = GIST_SSDC_COUNTERS;
+constexpr int kLbWarp = kCountWarp + kCountWarps;  // first of kLbWarps look-back warps (alternate tiles)
+constexpr int kLbWarps = GIST_SSDC_LBS;
+constexpr int kProdWarp = kLbWarp + kLbWarps;    // claims tickets, issues TMA loads
+constexpr int kStoreWarp = kProdWarp + 1;        // first of kStoreWarps store warps
 constexpr int kStoreWarps = 2;
 constexpr int kCtaThreads = 32 * (kStoreWarp + kStoreWarps);
+static_assert((kRing & (kRing - 1)) == 0 && kRing >= kTileRows * kRow, "pending ring: power of two >= one tile");
+// Each mbarrier phase must be awaited by one warp only (test_wait.parity on a phase that has not
+// started would alias the previous one), so role warps that alternate tiles must own disjoint
+// stages / queue slots.
+static_assert(kStages % kCountWarps == 0, "counter warps must own disjoint raw stages");
+static_assert(kQ % kLbWarps == 0, "look-back warps must own disjoint queue slots");
 
 struct __align__(128) EncSmem {
     float tile[kStages][kTileElems];  // raw tiles (TMA destinations)
@@ -90,8 +113,9 @@ struct __align__(128) EncSmem {
     uint32_t pos[kQ];                 // ring offset of the tile's compacted entries
     int64_t ring_end[kQ];             // monotonic ring position after the tile
     int64_t alloc_pos;                // monotonic ring allocation cursor (compactor leader)
-    volatile int64_t free_pos;        // monotonic ring release cursor (storers)
-    volatile int32_t stored;          // tiles fully stored by this CTA
+    unsigned long long free_pos;      // monotonic ring release cursor (storers; atomic access)
+    int32_t stored;                   // tiles fully stored by this CTA (atomic access)
+    int32_t last_j;                   // CTA-local index of the "no more tiles" ticket (atomic access)
 };
 
 // Start the TMA bulk load of tile t (claimed in ticket order) into stage s; always one arrival
@@ -135,6 +159,27 @@ __device__ __forceinline__ int64_t look_back(const Workspace *ws, int64_t tile, 
     }
 }
 
+// Cross-role flags in shared memory: release (fence, then atomic store) / acquire (atomic load,
+// then fence), so the hand-offs that are not mbarrier phases are ordered like them.
+__device__ __forceinline__ int32_t flag_ld(int32_t *p) {
+    const int32_t v = atomicAdd(p, 0);
+    __threadfence_block();
+    return v;
+}
+__device__ __forceinline__ void flag_st(int32_t *p, int32_t v) {
+    __threadfence_block();
+    atomicExch(p, v);
+}
+__device__ __forceinline__ int64_t flag_ld64(unsigned long long *p) {
+    const unsigned long long v = atomicAdd(p, 0ull);
+    __threadfence_block();
+    return (int64_t)v;
+}
+__device__ __forceinline__ void flag_st64(unsigned long long *p, int64_t v) {
+    __threadfence_block();
+    atomicExch(p, (unsigned long long)v);
+}
+
 __device__ __forceinline__ void compactors_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kEncThreads) : "memory"); }
 __device__ __forceinline__ void storers_sync() { asm volatile("bar.sync 2, %0;" ::"n"(32 * kStoreWarps) : "memory"); }
 
@@ -160,28 +205,34 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
         S.alloc_pos = 0;
         S.free_pos = 0;
         S.stored = 0;
+        S.last_j = 0x7fffffff;
         fence_mbar_init();
     }
     __syncthreads();
 
     if (warp == kProdWarp) {
-        // ---- producer: keep the raw ring full, in ticket order
+        // ---- producer: keep the raw ring full, in ticket order.  The next ticket is claimed
+        // while waiting for a free stage, so the atomic's round trip is off the refill path.
         if (lane == 0) {
+            int64_t t = atomicAdd(&ws->ticket, 1u);
             for (int j = 0;; ++j) {
                 const int s = j % kStages;
                 if (j >= kStages) mbar_wait(&S.empty[s], (uint32_t)(j / kStages - 1) & 1u);
-                const int64_t t = atomicAdd(&ws->ticket, 1u);
                 load_tile(S, s, t, x, n, tiles);
                 if (t >= tiles) break;
+                t = atomicAdd(&ws->ticket, 1u);
             }
         }
-    } else if (warp == kCountWarp) {
-        // ---- counter: nonzero bit patterns (R8) of every row, tile scan, publish aggregate
-        for (int j = 0;; ++j) {
+    } else if (warp >= kCountWarp && warp < kCountWarp + kCountWarps) {
+        // ---- counters (alternate tiles): nonzero bit patterns (R8) of every row, tile scan,
+        // publish the aggregate as soon as the tile lands
+        for (int j = warp - kCountWarp;; j += kCountWarps) {
             const int s = j % kStages, q = j % kQ;
-            mbar_wait(&S.full[s], (uint32_t)(j / kStages) & 1u);
-            while (j - S.stored >= kQ) {  // queue slot still held by a tile not yet stored
-            }
+            bool ready;  // sleep-wait; past the CTA's last tile no arrival ever comes for this j
+            while (!(ready = mbar_try(&S.full[s], (uint32_t)(j / kStages) & 1u, 1000)))
+                if (flag_ld(&S.last_j) < j) break;
+            if (!ready) break;
+            while (j - flag_ld(&S.stored) >= kQ) __nanosleep(64);  // queue slot still held by an unstored tile
             const int64_t tile = S.st_ticket[s];
             if (lane == 0) S.q_ticket[q] = tile;
             if (tile < tiles) {
@@ -194,14 +245,17 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                     __syncwarp();
                 }
                 uint32_t mine = 0;  // lane r ends up with row r's count
-#pragma unroll 4
-                for (int r = 0; r < kTileRows; ++r) {
+#pragma unroll
+                for (int r = 0; r < kTileRows; r += 2) {  // two rows per reduction (16-bit fields)
                     const uint4 *row4 = reinterpret_cast<const uint4 *>(T + r * kRow);
-                    const uint4 a = row4[lane], b = row4[32 + lane];
-                    const uint32_t c = (a.x != 0u) + (a.y != 0u) + (a.z != 0u) + (a.w != 0u) + (b.x != 0u) +
-                                       (b.y != 0u) + (b.z != 0u) + (b.w != 0u);
-                    const uint32_t t = __reduce_add_sync(kFull, c);
-                    if (lane == r) mine = t;
+                    const uint4 a = row4[lane], b = row4[32 + lane], c = row4[64 + lane], d = row4[96 + lane];
+                    const uint32_t c0 = (a.x != 0u) + (a.y != 0u) + (a.z != 0u) + (a.w != 0u) + (b.x != 0u) +
+                                        (b.y != 0u) + (b.z != 0u) + (b.w != 0u);
+                    const uint32_t c1 = (c.x != 0u) + (c.y != 0u) + (c.z != 0u) + (c.w != 0u) + (d.x != 0u) +
+                                        (d.y != 0u) + (d.z != 0u) + (d.w != 0u);
+                    const uint32_t t = __reduce_add_sync(kFull, c0 | (c1 << 16));
+                    if (lane == r) mine = t & 0xffffu;
+                    if (lane == r + 1) mine = t >> 16;
                 }
                 uint32_t inc = mine;
 #pragma unroll
@@ -219,17 +273,28 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                 }
             }
             __syncwarp();
-            if (lane == 0) mbar_arrive(&S.counted[q]);
+            if (lane == 0) {
+                if (tile >= tiles) flag_st(&S.last_j, j);  // before the arrival
+                mbar_arrive(&S.counted[q]);
+            }
             if (tile >= tiles) break;
         }
-    } else if (warp == kLbWarp) {
-        // ---- look-back: global offset of each counted tile; publish prefix, row ends, nnz
-        for (int j = 0;; ++j) {
+    } else if (warp >= kLbWarp && warp < kLbWarp + kLbWarps) {
+        // ---- look-back (alternate tiles): global offset of each counted tile; publish the
+        // inclusive prefix, row ends and, for the last tile, nnz
+        for (int j = warp - kLbWarp;; j += kLbWarps) {
             const int q = j % kQ;
-            mbar_wait(&S.counted[q], (uint32_t)(j / kQ) & 1u);
+            bool ready;  // sleep-wait; past the CTA's last tile no arrival ever comes for this j
+            while (!(ready = mbar_try(&S.counted[q], (uint32_t)(j / kQ) & 1u, 1000)))
+                if (flag_ld(&S.last_j) < j) break;
+            if (!ready) break;
             const int64_t tile = S.q_ticket[q];
             if (tile < tiles) {
+#ifdef GIST_SSDC_ABLATE_LOOKBACK  // timing experiment only: no look-back (wrong output)
+                const int64_t excl = 0;
+#else
                 const int64_t excl = (tile == 0) ? 0 : look_back(ws, tile, lane);
+#endif
                 const uint32_t total = S.total[q];
                 if (lane == 0) {
                     S.excl[q] = excl;
@@ -253,21 +318,28 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
             mbar_wait(&S.counted[q], (uint32_t)(j / kQ) & 1u);
             const int64_t tile = S.q_ticket[q];
             if (tile >= tiles) break;
-            if (threadIdx.x == 0) {  // allocate T contiguous ring entries (skip the ring end)
+            if (threadIdx.x == 0) {  // allocate T ring entries (indices wrap modulo kRing)
                 const uint32_t T = S.total[q];
-                int64_t p = S.alloc_pos;
-                const int64_t pm = p % kRing;
-                if (pm + T > kRing) p += kRing - pm;
-                while (p + T - S.free_pos > kRing) {
-                }
-                S.pos[q] = (uint32_t)(p % kRing);
+                const int64_t p = S.alloc_pos;
+                while (p + T - flag_ld64(&S.free_pos) > kRing) __nanosleep(64);
+                S.pos[q] = (uint32_t)(p & (kRing - 1));
                 S.ring_end[q] = p + T;
                 S.alloc_pos = p + T;
             }
             compactors_sync();
+#ifdef GIST_SSDC_ABLATE_COMPACT  // timing experiment only: skip compaction (wrong output)
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (lane == 0) {
+                mbar_arrive(&S.empty[s]);
+                mbar_arrive(&S.compacted[q]);
+            }
+            continue;
+#endif
             const float *Tr = S.tile[s];
-            float *vr = S.vring + S.pos[q];
-            uint8_t *cr = S.cring + S.pos[q];
+            const uint32_t rp = S.pos[q];
+            float *vr = S.vring;
+            uint8_t *cr = S.cring;
 #pragma unroll
             for (int r = 0; r < kRowsPerWarp; ++r) {
                 const int rr = warp * kRowsPerWarp + r;
@@ -285,8 +357,9 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                 for (int k = 0; k < 4; ++k) {
                     const uint32_t on = (bal[k] >> lane) & 1u;
                     if (on) {
-                        vr[p_lo] = v[k];
-                        cr[p_lo] = (uint8_t)(4 * lane + k);
+                        const uint32_t m = (rp + p_lo) & (kRing - 1);
+                        vr[m] = v[k];
+                        cr[m] = (uint8_t)(4 * lane + k);
                     }
                     p_lo += on;
                 }
@@ -294,8 +367,9 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                 for (int k = 0; k < 4; ++k) {
                     const uint32_t on = (bal[4 + k] >> lane) & 1u;
                     if (on) {
-                        vr[p_hi] = v[4 + k];
-                        cr[p_hi] = (uint8_t)(128 + 4 * lane + k);
+                        const uint32_t m = (rp + p_hi) & (kRing - 1);
+                        vr[m] = v[4 + k];
+                        cr[m] = (uint8_t)(128 + 4 * lane + k);
                     }
                     p_hi += on;
                 }
@@ -321,19 +395,22 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
             const int64_t excl = S.excl[q];
             int64_t lim = S.total[q];
             if (excl + lim > capacity) lim = capacity > excl ? capacity - excl : 0;
-            const float *vr = S.vring + S.pos[q];
-            const uint8_t *cr = S.cring + S.pos[q];
+            const uint32_t rp = S.pos[q];
             float *vo = val + excl;
             uint8_t *co = col + excl;
+#ifdef GIST_SSDC_ABLATE_STORE  // timing experiment only: skip the global stores (wrong output)
+            lim = 0;
+#endif
 #pragma unroll 4
             for (int k = sl; k < (int)lim; k += 32 * kStoreWarps) {
-                vo[k] = vr[k];
-                co[k] = cr[k];
+                const uint32_t m = (rp + (uint32_t)k) & (kRing - 1);
+                vo[k] = S.vring[m];
+                co[k] = S.cring[m];
             }
             storers_sync();
             if (sl == 0) {
-                S.free_pos = S.ring_end[q];
-                S.stored = j + 1;
+                flag_st64(&S.free_pos, S.ring_end[q]);
+                flag_st(&S.stored, j + 1);
             }
         }
     }

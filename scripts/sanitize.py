@@ -1,0 +1,25 @@
+"""Small-shape run of every kernel for compute-sanitizer (memcheck / racecheck / synccheck)."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+import paper_conf_isca_jainpmtp18_b200 as gist  # noqa: E402
+import workloads as WL  # noqa: E402
+
+dev = torch.device("cuda:0")
+for g, shape in [(WL.P2S2, (2, 8, 16, 16)), (WL.P2S2, (1, 3, 14, 14)), (WL.P3S2, (2, 4, 13, 13)),
+                 (WL.P3S2C, (1, 4, 12, 12)), (WL.P3S1P1, (1, 4, 9, 9))]:
+    y = WL.relu_map(shape, 0.5, 1, dev)
+    out, arg, mask = gist.gist_maxpool_fwd_argmax(y, g, fuse_mask=True)
+    gist.gist_pool_relu_bwd(torch.randn_like(out), arg, mask, shape, g)
+for n in (1, 1000, 4096 * 3 + 5, 256 * 16 * 40 + 17):
+    x = WL.relu_map((n,), 0.7, n, dev)
+    gist.gist_binarize_encode(x)
+    row_end, col, val, nnz = gist.gist_ssdc_encode(x, trim=True)
+    gist.gist_ssdc_decode(row_end, col, val, n)
+    for b in (16, 10, 8):
+        gist.gist_dpr_decode(gist.gist_dpr_encode(x, b), n, b)
+torch.cuda.synchronize()
+print("sanitize workload done")
