@@ -13,6 +13,8 @@
 // result is deterministic and equal to the oracle's ascending-o scatter.
 #include <math_constants.h>
 
+#include <algorithm>
+
 #include "common.cuh"
 #include "kernels.h"
 
@@ -56,6 +58,19 @@ maxpool_fwd_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ 
             const float *plane = y + (int64_t)nc * a.H * a.W;
             float best = -CUDART_INF_F;
             int bi = -1;
+            if (KH && KW && h0 >= 0 && w0 >= 0 && h0 + KH <= a.H && w0 + KW <= a.W) {  // interior window
+                const float *wp = plane + h0 * a.W + w0;
+                float v[KH ? KH : 1][KW ? KW : 1];
+#pragma unroll
+                for (int dy = 0; dy < (KH ? KH : 1); ++dy)
+#pragma unroll
+                    for (int dx = 0; dx < (KW ? KW : 1); ++dx) v[dy][dx] = ld_ro(wp + dy * a.W + dx);
+                bi = 0;
+#pragma unroll
+                for (int dy = 0; dy < (KH ? KH : 1); ++dy)
+#pragma unroll
+                    for (int dx = 0; dx < (KW ? KW : 1); ++dx) take(v[dy][dx], dy * kw + dx, best, bi);
+            } else
             for (int dy = 0; dy < kh; ++dy) {
                 const int ih = h0 + dy;
                 if (ih < 0 || ih >= a.H) continue;
@@ -344,6 +359,369 @@ pool_bwd_k2s2_kernel(const float *__restrict__ dout, const uint32_t *__restrict_
     }
 }
 
+// ---- Generic geometry (any window <= 16 positions, stride, padding, ceil mode): shared-memory
+// tiles.  A tile is a band of output rows of one plane ("band") or several whole planes
+// ("multi"); its input rows are one contiguous range of the NCHW map, staged once with
+// coalesced float4 loads, so every window is read from shared memory.
+constexpr int kTileIn = 8192;   // staged floats per tile (32 KB)
+#ifndef GIST_POOL_K3S2_BLOCK
+#define GIST_POOL_K3S2_BLOCK 1
+#endif
+#ifndef GIST_POOL_FWD_TILED
+#define GIST_POOL_FWD_TILED 0
+#endif
+constexpr int kTileThreads = 256;
+
+struct TileSpec {
+    int32_t multi;   // 1: G whole planes per tile, 0: TR output rows of one plane
+    int32_t G, TR;
+    int32_t bands;   // band mode: tiles per plane
+    int64_t tiles;
+    int32_t NC;
+    FastDiv div_bands;
+};
+
+struct TileRange {
+    int64_t p0, np;    // first plane, planes
+    int32_t oh0, oh1;  // output rows [oh0, oh1) (multi: [0, Ho))
+};
+
+__device__ __forceinline__ TileRange tile_range(const TileSpec &T, const PoolArgs &a, int64_t tile) {
+    TileRange r;
+    if (T.multi) {
+        r.p0 = tile * T.G;
+        r.np = min((int64_t)T.G, (int64_t)T.NC - r.p0);
+        r.oh0 = 0;
+        r.oh1 = a.Ho;
+    } else {
+        uint32_t plane, band;
+        T.div_bands.divmod((uint32_t)tile, plane, band);
+        r.p0 = plane;
+        r.np = 1;
+        r.oh0 = (int)band * T.TR;
+        r.oh1 = min(a.Ho, r.oh0 + T.TR);
+    }
+    return r;
+}
+
+// Argmax of output o straight from global memory (boundary words only).
+__device__ int window_argmax_global(const float *__restrict__ y, const PoolArgs &a, int64_t o) {
+    uint32_t q, ow, nc, oh;
+    a.div_wo.divmod((uint32_t)o, q, ow);
+    a.div_ho.divmod(q, nc, oh);
+    const int h0 = (int)oh * a.sh - a.ph, w0 = (int)ow * a.sw - a.pw;
+    const float *plane = y + (int64_t)nc * a.H * a.W;
+    float best = -CUDART_INF_F;
+    int bi = -1;
+    for (int dy = 0; dy < a.kh; ++dy) {
+        const int ih = h0 + dy;
+        if (ih < 0 || ih >= a.H) continue;
+        for (int dx = 0; dx < a.kw; ++dx) {
+            const int iw = w0 + dx;
+            if (iw < 0 || iw >= a.W) continue;
+            if (bi < 0) bi = dy * a.kw + dx;
+            take(ld_ro(plane + ih * a.W + iw), dy * a.kw + dx, best, bi);
+        }
+    }
+    return bi;
+}
+
+// Stage global floats [g_lo, g_hi) into smem: s[g - base], base = g_lo & ~3 (16-B phase kept).
+__device__ __forceinline__ int64_t stage_range(float *s, const float *__restrict__ g, int64_t g_lo, int64_t g_hi,
+                                               int64_t n_total) {
+    const int64_t base = g_lo & ~3ll;
+    const int64_t q_end = (g_hi + 3) >> 2;
+    for (int64_t q4 = (base >> 2) + threadIdx.x; q4 < q_end; q4 += blockDim.x) {
+        const int64_t e = q4 * 4;
+        if (e + 4 <= n_total) {
+            reinterpret_cast<float4 *>(s)[q4 - (base >> 2)] = ld_stream_f4(reinterpret_cast<const float4 *>(g) + q4);
+        } else {
+            for (int k = 0; k < 4; ++k) s[e - base + k] = (e + k < n_total) ? g[e + k] : 0.0f;
+        }
+    }
+    return base;
+}
+
+template <int KH, int KW>
+__global__ void __launch_bounds__(kTileThreads)
+maxpool_fwd_tiled_kernel(const float *__restrict__ y, PoolArgs a, TileSpec T, float *__restrict__ out,
+                         uint32_t *__restrict__ arg) {
+    __shared__ __align__(16) float s_in[kTileIn + 8];
+    __shared__ uint8_t s_nib[kTileIn];
+    const int kh = KH ? KH : a.kh, kw = KW ? KW : a.kw;
+    const int64_t HW = (int64_t)a.H * a.W, HoWo = (int64_t)a.Ho * a.Wo;
+    for (int64_t tile = blockIdx.x; tile < T.tiles; tile += gridDim.x) {
+        const TileRange r = tile_range(T, a, tile);
+        const int ih_lo = T.multi ? 0 : max(0, r.oh0 * a.sh - a.ph);
+        const int ih_hi = T.multi ? a.H : min(a.H, (r.oh1 - 1) * a.sh - a.ph + kh);
+        const int64_t g_lo = r.p0 * HW + (int64_t)ih_lo * a.W;
+        const int64_t g_hi = (r.p0 + r.np - 1) * HW + (int64_t)ih_hi * a.W;
+        const int64_t base = stage_range(s_in, y, g_lo, g_hi, a.n_in);
+        const int64_t o_lo = r.p0 * HoWo + (int64_t)r.oh0 * a.Wo;
+        const int64_t o_hi = (r.p0 + r.np - 1) * HoWo + (int64_t)r.oh1 * a.Wo;
+        __syncthreads();
+        for (int64_t o = o_lo + threadIdx.x; o < o_hi; o += blockDim.x) {
+            uint32_t q, ow, nc, oh;
+            a.div_wo.divmod((uint32_t)o, q, ow);
+            a.div_ho.divmod(q, nc, oh);
+            const int h0 = (int)oh * a.sh - a.ph, w0 = (int)ow * a.sw - a.pw;
+            const float *pl = s_in + ((int64_t)nc * HW - base);
+            float best = -CUDART_INF_F;
+            int bi = -1;
+            if (KH && KW && h0 >= 0 && w0 >= 0 && h0 + KH <= a.H && w0 + KW <= a.W) {  // interior window
+                const float *wp = pl + h0 * a.W + w0;
+                bi = 0;
+#pragma unroll
+                for (int dy = 0; dy < (KH ? KH : 1); ++dy)
+#pragma unroll
+                    for (int dx = 0; dx < (KW ? KW : 1); ++dx) take(wp[dy * a.W + dx], dy * kw + dx, best, bi);
+            } else
+#pragma unroll
+            for (int dy = 0; dy < (KH ? KH : 4); ++dy) {
+                if (!KH && dy >= kh) break;
+                const int ih = h0 + dy;
+                if (ih < 0 || ih >= a.H) continue;
+#pragma unroll
+                for (int dx = 0; dx < (KW ? KW : 4); ++dx) {
+                    if (!KW && dx >= kw) break;
+                    const int iw = w0 + dx;
+                    if (iw < 0 || iw >= a.W) continue;
+                    if (bi < 0) bi = dy * kw + dx;  // first in-bounds position
+                    take(pl[ih * a.W + iw], dy * kw + dx, best, bi);
+                }
+            }
+            out[o] = best;
+            s_nib[o - o_lo] = (uint8_t)bi;
+        }
+        __syncthreads();
+        // argmax words starting inside [o_lo, o_hi); nibbles past o_hi (next tile) from global
+        for (int64_t w = ((o_lo + 7) >> 3) + threadIdx.x; w < ((o_hi + 7) >> 3); w += blockDim.x) {
+            uint32_t word = 0;
+            for (int j = 0; j < 8; ++j) {
+                const int64_t o = 8 * w + j;
+                uint32_t nib = 0;
+                if (o < o_hi) nib = s_nib[o - o_lo];
+                else if (o < a.n_out) nib = (uint32_t)window_argmax_global(y, a, o);
+                word |= nib << (4 * j);
+            }
+            arg[w] = word;
+        }
+        __syncthreads();
+    }
+}
+
+template <int KH, int KW, int SH, int SW>
+__global__ void __launch_bounds__(kTileThreads)
+pool_bwd_tiled_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
+                      const uint32_t *__restrict__ mask, PoolArgs a, TileSpec T, float *__restrict__ dx) {
+    __shared__ __align__(16) float s_dy[kTileIn + 8];
+    __shared__ uint32_t s_arg[kTileIn / 8 + 2];
+    const int kh = KH ? KH : a.kh, kw = KW ? KW : a.kw, sh = SH ? SH : a.sh, sw = SW ? SW : a.sw;
+    const int64_t HW = (int64_t)a.H * a.W, HoWo = (int64_t)a.Ho * a.Wo;
+    for (int64_t tile = blockIdx.x; tile < T.tiles; tile += gridDim.x) {
+        const TileRange r = tile_range(T, a, tile);
+        // owned input rows: a partition of [0, H) across the plane's bands
+        const int r_lo = (T.multi || r.oh0 == 0) ? 0 : min(a.H, max(0, r.oh0 * sh - a.ph));
+        const int r_hi = (T.multi || r.oh1 == a.Ho) ? a.H : min(a.H, max(0, r.oh1 * sh - a.ph));
+        // output rows whose windows cover them
+        const int t_lo = r_lo + a.ph - kh + 1;
+        const int os_lo = T.multi ? 0 : max(0, t_lo > 0 ? (t_lo + sh - 1) / sh : 0);
+        const int os_hi = T.multi ? a.Ho : min(a.Ho, r_hi > r_lo ? (r_hi - 1 + a.ph) / sh + 1 : os_lo);
+        const int64_t od_lo = r.p0 * HoWo + (int64_t)os_lo * a.Wo;
+        const int64_t od_hi = (r.p0 + r.np - 1) * HoWo + (int64_t)max(os_hi, os_lo) * a.Wo;
+        const int64_t dbase = stage_range(s_dy, dout, od_lo, od_hi, a.n_out);
+        const int64_t w_lo = od_lo >> 3;
+        for (int64_t w = w_lo + threadIdx.x; w < ((od_hi + 7) >> 3); w += blockDim.x) s_arg[w - w_lo] = ld_ro(arg + w);
+        __syncthreads();
+        const int64_t i_lo = r.p0 * HW + (int64_t)r_lo * a.W;
+        const int64_t i_hi = (r.p0 + r.np - 1) * HW + (int64_t)r_hi * a.W;
+        for (int64_t i = i_lo + threadIdx.x; i < i_hi; i += blockDim.x) {
+            uint32_t q, iw, nc, ih;
+            a.div_w.divmod((uint32_t)i, q, iw);
+            a.div_h.divmod(q, nc, ih);
+            float acc = 0.0f;  // R6: +0.0f, then ascending output order
+            if (mask == nullptr || ((ld_ro(mask + (i >> 5)) >> (i & 31)) & 1u)) {
+                const int th = (int)ih + a.ph, tw = (int)iw + a.pw;
+                const int oh_lo = th - kh + 1 > 0 ? (th - kh + 1 + sh - 1) / sh : 0;
+                const int oh_hi = min(a.Ho - 1, th / sh);
+                const int ow_lo = tw - kw + 1 > 0 ? (tw - kw + 1 + sw - 1) / sw : 0;
+                const int ow_hi = min(a.Wo - 1, tw / sw);
+                const int64_t ob = (int64_t)nc * HoWo;
+                for (int oh = oh_lo; oh <= oh_hi; ++oh) {
+                    const int ly = th - oh * sh;
+                    for (int ow = ow_lo; ow <= ow_hi; ++ow) {
+                        const int64_t o = ob + (int64_t)oh * a.Wo + ow;
+                        const uint32_t nib = (s_arg[(o >> 3) - w_lo] >> (4 * (o & 7))) & 0xfu;
+                        if (nib == (uint32_t)(ly * kw + (tw - ow * sw))) acc = acc + s_dy[o - dbase];
+                    }
+                }
+            }
+            dx[i] = acc;
+        }
+        __syncthreads();
+    }
+}
+
+// 3x3 stride 2, no padding (AlexNet, NiN, GoogLeNet stems; floor or ceil): one thread per 2x2
+// input block [2a, 2a+2) x [2b, 2b+2).  All four elements share the candidate windows
+// (oh, ow) in {a-1, a} x {b-1, b}; each window's nibble is decoded once and, visited in
+// ascending output order, routes +dY to the block element its argmax points at (R6).
+__global__ void __launch_bounds__(kTileThreads)
+pool_bwd_tiled_k3s2_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
+                           const uint32_t *__restrict__ mask, PoolArgs a, TileSpec T, FastDiv div_wb,
+                           FastDiv div_hb, float *__restrict__ dx) {
+    __shared__ __align__(16) float s_dy[kTileIn + 8];
+    __shared__ uint32_t s_arg[kTileIn / 8 + 2];
+    const int64_t HW = (int64_t)a.H * a.W, HoWo = (int64_t)a.Ho * a.Wo;
+    const int Wb = (a.W + 1) >> 1;
+    for (int64_t tile = blockIdx.x; tile < T.tiles; tile += gridDim.x) {
+        const TileRange r = tile_range(T, a, tile);
+        const int a_lo = T.multi ? 0 : r.oh0;                                      // block rows
+        const int a_hi = (T.multi || r.oh1 == a.Ho) ? (a.H + 1) >> 1 : r.oh1;
+        const int os_lo = T.multi ? 0 : max(0, r.oh0 - 1);
+        const int os_hi = T.multi ? a.Ho : min(a.Ho, a_hi);
+        const int64_t od_lo = r.p0 * HoWo + (int64_t)os_lo * a.Wo;
+        const int64_t od_hi = (r.p0 + r.np - 1) * HoWo + (int64_t)os_hi * a.Wo;
+        const int64_t dbase = stage_range(s_dy, dout, od_lo, od_hi, a.n_out);
+        const int64_t w_lo = od_lo >> 3;
+        for (int64_t w = w_lo + threadIdx.x; w < ((od_hi + 7) >> 3); w += blockDim.x) s_arg[w - w_lo] = ld_ro(arg + w);
+        __syncthreads();
+        const int64_t nblk = r.np * (int64_t)(a_hi - a_lo) * Wb;
+        for (int64_t t = threadIdx.x; t < nblk; t += blockDim.x) {
+            uint32_t q, b, pl, ar;
+            div_wb.divmod((uint32_t)t, q, b);
+            div_hb.divmod(q, pl, ar);  // div_hb divides by the tile's block-row count
+            const int A = a_lo + (int)ar;
+            const int64_t plane = r.p0 + pl;
+            const int64_t i00 = plane * HW + (int64_t)(2 * A) * a.W + 2 * (int)b;
+            float acc[2][2] = {{0.0f, 0.0f}, {0.0f, 0.0f}};
+#pragma unroll
+            for (int dwo = -1; dwo <= 0; ++dwo) {  // oh = A-1, A (ascending)
+                const int oh = A + dwo;
+                if (oh < 0 || oh >= a.Ho) continue;
+#pragma unroll
+                for (int dwc = -1; dwc <= 0; ++dwc) {  // ow = b-1, b (ascending)
+                    const int ow = (int)b + dwc;
+                    if (ow < 0 || ow >= a.Wo) continue;
+                    const int64_t o = plane * HoWo + (int64_t)oh * a.Wo + ow;
+                    const uint32_t nib = (s_arg[(o >> 3) - w_lo] >> (4 * (o & 7))) & 0xfu;
+                    const int ry = 2 * oh + (int)(nib / 3u) - 2 * A, rx = 2 * ow + (int)(nib % 3u) - 2 * (int)b;
+                    if (ry >= 0 && ry < 2 && rx >= 0 && rx < 2) {
+                        const float g = s_dy[o - dbase];
+                        if (ry == 0) {
+                            if (rx == 0) acc[0][0] = acc[0][0] + g; else acc[0][1] = acc[0][1] + g;
+                        } else {
+                            if (rx == 0) acc[1][0] = acc[1][0] + g; else acc[1][1] = acc[1][1] + g;
+                        }
+                    }
+                }
+            }
+#pragma unroll
+            for (int ry = 0; ry < 2; ++ry) {
+                if (2 * A + ry >= a.H) continue;
+#pragma unroll
+                for (int rx = 0; rx < 2; ++rx) {
+                    if (2 * (int)b + rx >= a.W) continue;
+                    const int64_t i = i00 + (int64_t)ry * a.W + rx;
+                    const bool on = mask == nullptr || ((ld_ro(mask + (i >> 5)) >> (i & 31)) & 1u);
+                    dx[i] = on ? acc[ry][rx] : 0.0f;
+                }
+            }
+        }
+        __syncthreads();
+    }
+}
+
+// Same 2x2-block formulation without tiles: candidate windows' dY and nibbles come straight
+// through L1 (neighbouring blocks share them), all loads issued before use.
+__global__ void __launch_bounds__(kPoolThreads)
+pool_bwd_k3s2_block_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
+                           const uint32_t *__restrict__ mask, PoolArgs a, FastDiv div_wb, FastDiv div_hb,
+                           int64_t nblk, float *__restrict__ dx) {
+    const int64_t HW = (int64_t)a.H * a.W, HoWo = (int64_t)a.Ho * a.Wo;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < nblk; t += stride) {
+        uint32_t q, b, plane, A;
+        div_wb.divmod((uint32_t)t, q, b);
+        div_hb.divmod(q, plane, A);
+        float g[2][2];
+        uint32_t nib[2][2];
+        bool ok[2][2];
+#pragma unroll
+        for (int u = 0; u < 2; ++u)
+#pragma unroll
+            for (int v = 0; v < 2; ++v) {
+                const int oh = (int)A - 1 + u, ow = (int)b - 1 + v;
+                ok[u][v] = oh >= 0 && oh < a.Ho && ow >= 0 && ow < a.Wo;
+                const int64_t o = (int64_t)plane * HoWo + (int64_t)(ok[u][v] ? oh : 0) * a.Wo + (ok[u][v] ? ow : 0);
+                g[u][v] = ld_ro(dout + o);
+                nib[u][v] = (ld_ro(arg + (o >> 3)) >> (4 * (o & 7))) & 0xfu;
+            }
+        const int64_t i00 = (int64_t)plane * HW + (int64_t)(2 * A) * a.W + 2 * (int)b;
+        uint32_t m[2] = {3u, 3u};
+        if (mask) {
+#pragma unroll
+            for (int ry = 0; ry < 2; ++ry) {
+                const int64_t i = i00 + (int64_t)ry * a.W;
+                const int64_t ic = (2 * (int)A + ry < a.H) ? i : i00;
+                const uint32_t w0 = ld_ro(mask + (ic >> 5)), w1 = ld_ro(mask + ((ic + 1) >> 5));
+                m[ry] = ((w0 >> (ic & 31)) & 1u) | (((w1 >> ((ic + 1) & 31)) & 1u) << 1);
+            }
+        }
+        float acc[2][2] = {{0.0f, 0.0f}, {0.0f, 0.0f}};
+#pragma unroll
+        for (int u = 0; u < 2; ++u)  // ascending output order: (A-1, b-1), (A-1, b), (A, b-1), (A, b)
+#pragma unroll
+            for (int v = 0; v < 2; ++v) {
+                if (!ok[u][v]) continue;
+                const int ry = 2 * (u - 1) + (int)(nib[u][v] / 3u), rx = 2 * (v - 1) + (int)(nib[u][v] % 3u);
+                if (ry == 0 && rx == 0) acc[0][0] = acc[0][0] + g[u][v];
+                if (ry == 0 && rx == 1) acc[0][1] = acc[0][1] + g[u][v];
+                if (ry == 1 && rx == 0) acc[1][0] = acc[1][0] + g[u][v];
+                if (ry == 1 && rx == 1) acc[1][1] = acc[1][1] + g[u][v];
+            }
+#pragma unroll
+        for (int ry = 0; ry < 2; ++ry) {
+            if (2 * (int)A + ry >= a.H) continue;
+#pragma unroll
+            for (int rx = 0; rx < 2; ++rx) {
+                if (2 * (int)b + rx >= a.W) continue;
+                dx[i00 + (int64_t)ry * a.W + rx] = ((m[ry] >> rx) & 1u) ? acc[ry][rx] : 0.0f;
+            }
+        }
+    }
+}
+
+// Host: tiles for the generic kernels.  Forward stages input rows (bounded by kTileIn floats);
+// backward stages dY rows (bounded likewise).
+TileSpec make_tiles(const PoolArgs &a, int32_t NC, bool backward) {
+    TileSpec T{};
+    T.NC = NC;
+    // forward stages input rows and keeps one nibble byte per output; backward stages dY rows
+    const int64_t plane = backward ? (int64_t)a.Ho * a.Wo : std::max((int64_t)a.H * a.W, (int64_t)a.Ho * a.Wo);
+    if (plane <= kTileIn) {
+        T.multi = 1;
+        T.G = (int32_t)(kTileIn / plane);
+        T.tiles = ceil_div(NC, T.G);
+        T.TR = a.Ho;
+        T.bands = 1;
+    } else {
+        T.multi = 0;
+        int64_t tr;
+        if (backward) {  // staged output rows = TR + floor((kh-1)/sh) <= kTileIn / Wo
+            tr = kTileIn / a.Wo - (a.kh - 1) / a.sh - 1;
+        } else {  // staged input rows (TR-1)*sh + kh <= kTileIn / W, and TR*Wo nibbles
+            tr = std::min<int64_t>((kTileIn / a.W - a.kh) / a.sh + 1, kTileIn / a.Wo);
+        }
+        T.TR = (int32_t)std::min<int64_t>(std::max<int64_t>(1, tr), a.Ho);
+        T.bands = (int32_t)ceil_div(a.Ho, T.TR);
+        T.tiles = (int64_t)NC * T.bands;
+        T.G = 1;
+    }
+    T.div_bands = FastDiv::make((uint32_t)std::max(1, T.bands));
+    return T;
+}
+
 PoolArgs make_args(int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo) {
     PoolArgs a;
     a.H = H;
@@ -363,6 +741,12 @@ PoolArgs make_args(int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d
     a.div_w = FastDiv::make((uint32_t)W);
     a.div_h = FastDiv::make((uint32_t)H);
     return a;
+}
+
+// The tiled kernels need a band of at least one output row's windows (fwd) / one staged output
+// row (bwd) to fit the tile, and windows of at most 4x4.
+bool tiled_ok(const PoolArgs &a) {
+    return a.kh <= 4 && a.kw <= 4 && (int64_t)a.kh * a.W <= kTileIn && (int64_t)(a.kh + 2) * a.Wo <= kTileIn;
 }
 
 bool is_k2s2_exact(const gist_pool2d &p, int32_t H, int32_t W, int32_t Ho, int32_t Wo) {
@@ -391,10 +775,17 @@ cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, 
         else maxpool_fwd_k2s2_pair_kernel<false><<<g2, kPoolThreads, 0, s>>>(y, a, out, argmax);
     } else if (is_k2s2_exact(p, H, W, Ho, Wo))
         maxpool_fwd_k2s2_kernel<<<grid_for(ceil_div(a.n_out, kFwdU), kPoolThreads, 8), kPoolThreads, 0, s>>>(y, a, out, argmax);
-    else if (p.kh == 3 && p.kw == 3)
+    else if (GIST_POOL_FWD_TILED && tiled_ok(a)) {
+        const TileSpec T = make_tiles(a, N * C, false);
+        const unsigned gt = (unsigned)std::min<int64_t>(T.tiles, (int64_t)num_sms() * 6);
+        if (p.kh == 3 && p.kw == 3)
+            maxpool_fwd_tiled_kernel<3, 3><<<gt, kTileThreads, 0, s>>>(y, a, T, out, argmax);
+        else if (p.kh == 2 && p.kw == 2)
+            maxpool_fwd_tiled_kernel<2, 2><<<gt, kTileThreads, 0, s>>>(y, a, T, out, argmax);
+        else
+            maxpool_fwd_tiled_kernel<0, 0><<<gt, kTileThreads, 0, s>>>(y, a, T, out, argmax);
+    } else if (p.kh == 3 && p.kw == 3)
         maxpool_fwd_kernel<3, 3><<<grid, kPoolThreads, 0, s>>>(y, a, out, argmax);
-    else if (p.kh == 2 && p.kw == 2)
-        maxpool_fwd_kernel<2, 2><<<grid, kPoolThreads, 0, s>>>(y, a, out, argmax);
     else
         maxpool_fwd_kernel<0, 0><<<grid, kPoolThreads, 0, s>>>(y, a, out, argmax);
     return cudaPeekAtLastError();
@@ -410,6 +801,26 @@ cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uin
         else pool_bwd_k2s2_pair_kernel<false><<<g2, kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
     } else if (is_k2s2_exact(p, H, W, Ho, Wo)) {
         pool_bwd_k2s2_kernel<<<grid_for(ceil_div(a.n_out, kBwdU), kPoolThreads, 8), kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+    } else if (GIST_POOL_K3S2_BLOCK && p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2 && p.ph == 0 && p.pw == 0) {
+        const int32_t hb = (H + 1) / 2, wb = (W + 1) / 2;
+        const int64_t nblk = (int64_t)N * C * hb * wb;
+        pool_bwd_k3s2_block_kernel<<<grid_for(nblk, kPoolThreads, 8), kPoolThreads, 0, s>>>(
+            dout, argmax, mask, a, FastDiv::make(wb), FastDiv::make(hb), nblk, dx);
+    } else if (tiled_ok(a)) {
+        const TileSpec T = make_tiles(a, N * C, true);
+        const unsigned gt = (unsigned)std::min<int64_t>(T.tiles, (int64_t)num_sms() * 6);
+        if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2 && p.ph == 0 && p.pw == 0) {
+            // block rows per tile: multi -> all (H+1)/2 of each plane; band -> TR (last band may be
+            // shorter: the kernel bounds t by its own count, the divisor only needs the stride)
+            const int32_t hb = T.multi ? (H + 1) / 2 : T.TR + 1;
+            pool_bwd_tiled_k3s2_kernel<<<gt, kTileThreads, 0, s>>>(dout, argmax, mask, a, T, FastDiv::make((W + 1) / 2),
+                                                                   FastDiv::make(hb), dx);
+        } else if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2)
+            pool_bwd_tiled_kernel<3, 3, 2, 2><<<gt, kTileThreads, 0, s>>>(dout, argmax, mask, a, T, dx);
+        else if (p.kh == 3 && p.kw == 3 && p.sh == 1 && p.sw == 1)
+            pool_bwd_tiled_kernel<3, 3, 1, 1><<<gt, kTileThreads, 0, s>>>(dout, argmax, mask, a, T, dx);
+        else
+            pool_bwd_tiled_kernel<0, 0, 0, 0><<<gt, kTileThreads, 0, s>>>(dout, argmax, mask, a, T, dx);
     } else {
         const unsigned grid = grid_for(a.n_in, kPoolThreads, 8);
         if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2)
