@@ -163,6 +163,20 @@ gist_status gist_ssdc_decode(const int32_t *row_end, const uint8_t *col, const f
 gist_status gist_dpr_encode(const float *x, int64_t n, int32_t bits, uint32_t *packed, cudaStream_t stream);
 gist_status gist_dpr_decode(const uint32_t *packed, int64_t n, int32_t bits, float *x, cudaStream_t stream);
 
+/* ---------------------------------------------------------------- f1: DPR over SSDC values
+ * P:169 §IV-A: "We also apply it [DPR] over SSDC encoding, compressing the non-zero values array
+ * in the CSR format.  We do not touch the meta array in CSR format".  Same conversion and
+ * packing as gist_dpr_encode/decode, applied to the first min(*nnz, capacity) entries of the
+ * CSR value array; *nnz is the DEVICE count written by gist_ssdc_encode, read on the device
+ * (no host synchronization).  Words past ceil(count/k) are left untouched.
+ *   encode: val [capacity] fp32 read, packed [gist_dpr_words(capacity, bits)] uint32 written.
+ *   decode: packed read, val [capacity] fp32 written (first count entries).
+ * Encoded footprint: 4*ceil(nnz/k) + nnz + 4*rows bytes (vs 5*nnz + 4*rows). */
+gist_status gist_ssdc_dpr_encode(const float *val, const int64_t *nnz, int64_t capacity, int32_t bits,
+                                 uint32_t *packed, cudaStream_t stream);
+gist_status gist_ssdc_dpr_decode(const uint32_t *packed, const int64_t *nnz, int64_t capacity, int32_t bits,
+                                 float *val, cudaStream_t stream);
+
 /* Number of SMs the launch heuristics use (cached on first call; for diagnostics). */
 int32_t gist_num_sms(void);
 

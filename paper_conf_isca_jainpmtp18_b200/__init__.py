@@ -23,6 +23,7 @@ __all__ = [
     "gist_ssdc_bytes", "gist_ssdc_workspace_bytes", "gist_dpr_words", "gist_num_sms", "gist_launch_count",
     "gist_binarize_encode", "gist_maxpool_fwd_argmax", "gist_pool_relu_bwd",
     "gist_ssdc_encode", "gist_ssdc_decode", "gist_dpr_encode", "gist_dpr_decode",
+    "gist_ssdc_dpr_encode", "gist_ssdc_dpr_decode",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -75,6 +76,8 @@ def _load() -> C.CDLL:
         "gist_ssdc_decode": (C.c_int, [p, p, p, i64, p, p]),
         "gist_dpr_encode": (C.c_int, [p, i64, i32, p, p]),
         "gist_dpr_decode": (C.c_int, [p, i64, i32, p, p]),
+        "gist_ssdc_dpr_encode": (C.c_int, [p, p, i64, i32, p, p]),
+        "gist_ssdc_dpr_decode": (C.c_int, [p, p, i64, i32, p, p]),
     }
     for name, (res, args) in sigs.items():
         fn = getattr(L, name)
@@ -247,3 +250,26 @@ def gist_dpr_decode(packed: torch.Tensor, n: int, bits: int, x: torch.Tensor | N
         x = torch.empty(n, dtype=torch.float32, device=packed.device)
     _check(lib.gist_dpr_decode(_ptr(packed), n, bits, _ptr(x), _stream(packed, stream)), "gist_dpr_decode")
     return x
+
+
+def gist_ssdc_dpr_encode(val: torch.Tensor, nnz: torch.Tensor, bits: int, capacity: int | None = None,
+                         packed: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """f1: DPR of the first min(nnz, capacity) CSR values; nnz is the device int64."""
+    cap = val.numel() if capacity is None else int(capacity)
+    words = gist_dpr_words(cap, bits)
+    if words < 0:
+        raise GistError(3, "gist_ssdc_dpr_encode")
+    packed = _words(words, val.device, packed)
+    _check(lib.gist_ssdc_dpr_encode(_ptr(val), _ptr(nnz), cap, bits, _ptr(packed), _stream(val, stream)),
+           "gist_ssdc_dpr_encode")
+    return packed
+
+
+def gist_ssdc_dpr_decode(packed: torch.Tensor, nnz: torch.Tensor, bits: int, capacity: int,
+                         val: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """f1: restore the first min(nnz, capacity) CSR values to fp32."""
+    if val is None:
+        val = torch.empty(max(capacity, 1), dtype=torch.float32, device=packed.device)
+    _check(lib.gist_ssdc_dpr_decode(_ptr(packed), _ptr(nnz), int(capacity), bits, _ptr(val), _stream(packed, stream)),
+           "gist_ssdc_dpr_decode")
+    return val

@@ -212,4 +212,28 @@ gist_status gist_dpr_decode(const uint32_t *packed, int64_t n, int32_t bits, flo
     return launched(gist::launch_dpr_decode(packed, n, bits, x, stream), 1);
 }
 
+gist_status gist_ssdc_dpr_encode(const float *val, const int64_t *nnz, int64_t capacity, int32_t bits,
+                                 uint32_t *packed, cudaStream_t stream) {
+    if (bits != 8 && bits != 10 && bits != 16) return GIST_ERR_UNSUPPORTED;
+    if (capacity < 0) return GIST_ERR_INVALID_ARGUMENT;
+    if (capacity == 0) return GIST_OK;
+    if (!val || !nnz || !packed) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(val) || misaligned(packed) || (reinterpret_cast<uintptr_t>(nnz) & 7u)) return GIST_ERR_MISALIGNED;
+    if (any_overlap({{val, 4 * capacity}, {nnz, 8}}, {{packed, 4 * gist_dpr_words(capacity, bits)}}))
+        return GIST_ERR_INVALID_ARGUMENT;
+    return launched(gist::launch_dpr_encode(val, capacity, bits, packed, stream, nnz), 1);
+}
+
+gist_status gist_ssdc_dpr_decode(const uint32_t *packed, const int64_t *nnz, int64_t capacity, int32_t bits,
+                                 float *val, cudaStream_t stream) {
+    if (bits != 8 && bits != 10 && bits != 16) return GIST_ERR_UNSUPPORTED;
+    if (capacity < 0) return GIST_ERR_INVALID_ARGUMENT;
+    if (capacity == 0) return GIST_OK;
+    if (!val || !nnz || !packed) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(val) || misaligned(packed) || (reinterpret_cast<uintptr_t>(nnz) & 7u)) return GIST_ERR_MISALIGNED;
+    if (any_overlap({{packed, 4 * gist_dpr_words(capacity, bits)}, {nnz, 8}}, {{val, 4 * capacity}}))
+        return GIST_ERR_INVALID_ARGUMENT;
+    return launched(gist::launch_dpr_decode(packed, capacity, bits, val, stream, nnz), 1);
+}
+
 }  // extern "C"

@@ -22,7 +22,10 @@ cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint
                                int64_t capacity, int64_t *nnz, void *workspace, cudaStream_t s);
 cudaError_t launch_ssdc_decode(const int32_t *row_end, const uint8_t *col, const float *val, int64_t n, float *x,
                                cudaStream_t s);
-cudaError_t launch_dpr_encode(const float *x, int64_t n, int bits, uint32_t *packed, cudaStream_t s);
-cudaError_t launch_dpr_decode(const uint32_t *packed, int64_t n, int bits, float *x, cudaStream_t s);
+// n_dev != nullptr: the element count is min(n, *n_dev), read on the device.
+cudaError_t launch_dpr_encode(const float *x, int64_t n, int bits, uint32_t *packed, cudaStream_t s,
+                              const int64_t *n_dev = nullptr);
+cudaError_t launch_dpr_decode(const uint32_t *packed, int64_t n, int bits, float *x, cudaStream_t s,
+                              const int64_t *n_dev = nullptr);
 
 }  // namespace gist

@@ -110,3 +110,8 @@ def test_validation_without_gpu(gist):
     assert L.gist_ssdc_encode(A, 1 << 20, B, B + (1 << 24), B + (1 << 26), 1 << 20, B + (1 << 28), B + (1 << 29),
                               8, None) == INVALID  # workspace too small
     assert L.gist_ssdc_encode(A, 1024, B, None, None, 0, B + 4100, B + 8192, 4096, None) == MISALIGNED  # nnz
+    # f1: DPR over SSDC values (device count)
+    assert L.gist_ssdc_dpr_encode(A, B, 0, 16, B + 64, None) == OK
+    assert L.gist_ssdc_dpr_encode(A, B, 100, 12, B + 64, None) == UNSUPPORTED
+    assert L.gist_ssdc_dpr_encode(A, None, 100, 8, B + 64, None) == INVALID
+    assert L.gist_ssdc_dpr_decode(A, B + 4, 100, 8, B + 64, None) == MISALIGNED

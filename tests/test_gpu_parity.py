@@ -260,3 +260,22 @@ def test_full_size_vgg16_ssdc_and_dpr(gist, ref, cuda):
     for bits in (16, 10, 8):
         packed = gist.gist_dpr_encode(x, bits)
         assert_bits_equal(host(packed), ref.dpr_encode(xh, bits), f"fp{bits}")
+
+
+# ------------------------------------------------------------------------ f1: DPR over SSDC values
+@pytest.mark.parametrize("bits", [16, 10, 8])
+@pytest.mark.parametrize("n", [1000, 256 * 16 * 33 + 7])
+def test_ssdc_values_dpr(gist, ref, cuda, bits, n):
+    # DPR of the CSR value array only; the count comes from the device nnz.
+    x = WL.relu_map((n,), 0.7, n + bits, cuda) * torch.exp2(torch.randint(-8, 8, (n,), device=cuda).float())
+    row_end, col, val, nnz = gist.gist_ssdc_encode(x)
+    k = int(nnz.item())
+    packed = gist.gist_ssdc_dpr_encode(val, nnz, bits)
+    r_row_end, r_col, r_val = ref.ssdc_encode(host(x))
+    r_packed = ref.dpr_encode(r_val, bits)
+    assert_bits_equal(host(packed)[:r_packed.size], r_packed, "dpr(val)")
+    back = gist.gist_ssdc_dpr_decode(packed, nnz, bits, n)
+    assert_bits_equal(host(back)[:k], ref.dpr_decode(r_packed, k, bits), "dpr^-1")
+    dense = gist.gist_ssdc_decode(row_end, col, back[:max(k, 1)], n)
+    expect = ref.ssdc_decode(r_row_end, r_col, ref.dpr_decode(r_packed, k, bits), n)
+    assert_bits_equal(host(dense), expect, "ssdc_decode(dpr^-1(dpr(val)))")
