@@ -53,6 +53,24 @@ __device__ __forceinline__ void st_relaxed(uint64_t *p, uint64_t v) {
 }
 
 
+#ifdef GIST_SSDC_TRACE
+// Timing experiment only: per-tile hand-off timestamps (%globaltimer, ns) for the first
+// kTraceCtas CTAs: [cta][j][event], events 0 claim, 1 landed, 2 counted, 3 resolved,
+// 4 compacted, 5 stored.
+constexpr int kTraceCtas = 4, kTraceTiles = 256;
+__device__ uint64_t *g_trace = nullptr;
+__device__ __forceinline__ void trace(int j, int ev) {
+    if (g_trace && blockIdx.x < kTraceCtas && j < kTraceTiles) {
+        uint64_t t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        g_trace[((int64_t)blockIdx.x * kTraceTiles + j) * 8 + ev] = t;
+    }
+}
+#define TRACE(j, ev) trace(j, ev)
+#else
+#define TRACE(j, ev)
+#endif
+
 __global__ void ssdc_ws_init(uint64_t *ws, int64_t words) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += (int64_t)gridDim.x * blockDim.x)
         ws[i] = 0ull;
@@ -138,9 +156,14 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
 
 // Decoupled look-back by one warp: lane i reads tile base-i.  Sums aggregates up to and
 // including the nearest inclusive prefix, re-polling only needed unpublished descriptors.
-__device__ __forceinline__ int64_t look_back(const Workspace *ws, int64_t tile, int lane) {
+// On reaching that prefix the warp also publishes the inclusive prefixes of the aggregate-only
+// tiles it summed over in that round (their values follow from it; every writer writes the same
+// value), so the prefix frontier advances by up to 31 tiles per look-back.
+__device__ __forceinline__ int64_t look_back(Workspace *ws, int64_t tile, int lane, int *rounds = nullptr,
+                                             int *polls = nullptr) {
     int64_t excl = 0;
     for (int64_t base = tile - 1;; base -= 32) {
+        if (rounds) ++*rounds;
         const int64_t idx = base - lane;
         uint64_t d = (idx >= 0) ? ld_relaxed(&ws->desc[idx]) : kStatusP;  // virtual P(0)
         uint32_t pm, need;
@@ -149,13 +172,25 @@ __device__ __forceinline__ int64_t look_back(const Workspace *ws, int64_t tile, 
             const uint32_t xm = __ballot_sync(kFull, (d >> 62) == 0);
             need = pm ? (((pm & (0u - pm)) << 1) - 1u) : kFull;
             if (!(xm & need)) break;
+            if (polls) ++*polls;
             if ((d >> 62) == 0) d = ld_relaxed(&ws->desc[idx]);
         }
-        uint64_t v = ((need >> lane) & 1u) ? (d & kValueMask) : 0ull;
+        const uint64_t v = ((need >> lane) & 1u) ? (d & kValueMask) : 0ull;
+        if (pm) {
+            uint64_t suf = v;  // suffix sum over lanes [lane, first P]: inclusive prefix of tile base-lane
 #pragma unroll
-        for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
-        excl += (int64_t)v;
-        if (pm) return excl;
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint64_t t = __shfl_down_sync(kFull, suf, o);
+                if (lane + o < 32) suf += t;
+            }
+            const int first_p = __ffs(pm) - 1;
+            if (lane < first_p && idx >= 0) st_relaxed(&ws->desc[idx], kStatusP | suf);
+            return excl + (int64_t)__shfl_sync(kFull, suf, 0);
+        }
+        uint64_t w = v;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) w += __shfl_xor_sync(kFull, w, o);
+        excl += (int64_t)w;
     }
 }
 
@@ -218,6 +253,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
             for (int j = 0;; ++j) {
                 const int s = j % kStages;
                 if (j >= kStages) mbar_wait(&S.empty[s], (uint32_t)(j / kStages - 1) & 1u);
+                TRACE(j, 0);
                 load_tile(S, s, t, x, n, tiles);
                 if (t >= tiles) break;
                 t = atomicAdd(&ws->ticket, 1u);
@@ -232,9 +268,11 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
             while (!(ready = mbar_try(&S.full[s], (uint32_t)(j / kStages) & 1u, 1000)))
                 if (flag_ld(&S.last_j) < j) break;
             if (!ready) break;
+            if (lane == 0) TRACE(j, 1);
             while (j - flag_ld(&S.stored) >= kQ) __nanosleep(64);  // queue slot still held by an unstored tile
             const int64_t tile = S.st_ticket[s];
             if (lane == 0) S.q_ticket[q] = tile;
+
             if (tile < tiles) {
                 float *T = S.tile[s];
                 if (tile == tiles - 1) {  // ragged last tile: tail the TMA could not copy, zeros
@@ -275,6 +313,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
             __syncwarp();
             if (lane == 0) {
                 if (tile >= tiles) flag_st(&S.last_j, j);  // before the arrival
+                TRACE(j, 2);
                 mbar_arrive(&S.counted[q]);
             }
             if (tile >= tiles) break;
@@ -293,7 +332,15 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
 #ifdef GIST_SSDC_ABLATE_LOOKBACK  // timing experiment only: no look-back (wrong output)
                 const int64_t excl = 0;
 #else
+#ifdef GIST_SSDC_TRACE
+                int rounds = 0, polls = 0;
+                if (lane == 0) TRACE(j, 6);
+                const int64_t excl = (tile == 0) ? 0 : look_back(ws, tile, lane, &rounds, &polls);
+                if (lane == 0 && g_trace && blockIdx.x < kTraceCtas && j < kTraceTiles)
+                    g_trace[((int64_t)blockIdx.x * kTraceTiles + j) * 8 + 7] = (uint64_t)rounds * 1000000 + polls;
+#else
                 const int64_t excl = (tile == 0) ? 0 : look_back(ws, tile, lane);
+#endif
 #endif
                 const uint32_t total = S.total[q];
                 if (lane == 0) {
@@ -305,7 +352,10 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                 if (lane < kTileRows && r < rows) row_end[r] = (int32_t)(excl + S.row_excl[q][lane] + S.row_cnt[q][lane]);
             }
             __syncwarp();
-            if (lane == 0) mbar_arrive(&S.resolved[q]);
+            if (lane == 0) {
+                TRACE(j, 3);
+                mbar_arrive(&S.resolved[q]);
+            }
             if (tile >= tiles) break;
         }
     } else if (warp < kWarps) {
@@ -377,6 +427,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
             fence_proxy_async_smem();  // our reads of the raw stage precede the next TMA write
             __syncwarp();
             if (lane == 0) {
+                if (warp == 0) TRACE(j, 4);
                 mbar_arrive(&S.empty[s]);
                 mbar_arrive(&S.compacted[q]);
             }
@@ -409,6 +460,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
             }
             storers_sync();
             if (sl == 0) {
+                TRACE(j, 5);
                 flag_st64(&S.free_pos, S.ring_end[q]);
                 flag_st(&S.stored, j + 1);
             }
@@ -465,6 +517,12 @@ ssdc_decode_kernel(const int32_t *__restrict__ row_end, const uint8_t *__restric
 }
 
 }  // namespace
+
+#ifdef GIST_SSDC_TRACE
+extern "C" int gist_debug_ssdc_trace(void *buf) {
+    return (int)cudaMemcpyToSymbol(g_trace, &buf, sizeof(void *));
+}
+#endif
 
 size_t ssdc_workspace_bytes(int64_t n) {
     const int64_t rows = (n + kRow - 1) / kRow;
