@@ -398,7 +398,8 @@ def main():
     ap.add_argument("--batch", type=int, default=None, help="per-GPU batch (default: the config's)")
     ap.add_argument("--sparsity", type=float, default=None)
     ap.add_argument("--dpr-bits", type=int, default=None)
-    ap.add_argument("--fuse-mask", action="store_true", help="a1 inside the a2 call")
+    ap.add_argument("--no-fuse-mask", dest="fuse_mask", action="store_false",
+                    help="call a1 separately instead of passing the mask to the a2 call")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=8.0)
     ap.add_argument("--kernels-out", default=None, help="write the per-kernel breakdown JSON here")

@@ -103,7 +103,8 @@ gist_status gist_binarize_encode(const float *y, int64_t n, uint32_t *mask, cuda
  *   out    [N,C,Ho,Wo] fp32, written (the pool output, still consumed in forward).
  *   argmax [gist_argmax_words(N*C*Ho*Wo)] uint32, written.
  *   mask   NULL, or [gist_binarize_words(N*C*H*W)] uint32: if non-NULL the a1 mask of y is
- *          written in the same pass (fused Binarize; saves one read of y).
+ *          written too — in the same pass (one read of y) for 2x2/s2 unpadded pools with
+ *          W % 16 == 0 and H even, otherwise by a second kernel over y.
  * TOO_LARGE if N*C*H*W >= 2^31. */
 gist_status gist_maxpool_fwd_argmax(const float *y, int32_t N, int32_t C, int32_t H, int32_t W,
                                     const gist_pool2d *p, float *out, uint32_t *argmax,

@@ -137,9 +137,11 @@ gist_status gist_maxpool_fwd_argmax(const float *y, int32_t N, int32_t C, int32_
     if (any_overlap({{y, 4 * n}},
                     {{out, 4 * n_out}, {argmax, 4 * gist_argmax_words(n_out)}, {mask, mask ? 4 * gist_binarize_words(n) : 0}}))
         return GIST_ERR_INVALID_ARGUMENT;
-    cudaError_t e = gist::launch_maxpool_fwd(y, N, C, H, W, *p, Ho, Wo, out, argmax, stream);
-    if (e == cudaSuccess && mask) e = gist::launch_binarize(y, n, mask, stream);
-    return launched(e, mask ? 2 : 1);
+    bool fused = false;
+    cudaError_t e = gist::launch_maxpool_fwd(y, N, C, H, W, *p, Ho, Wo, out, argmax, stream, mask, &fused);
+    const bool separate = mask && !fused;  // geometry the fused kernel does not cover
+    if (e == cudaSuccess && separate) e = gist::launch_binarize(y, n, mask, stream);
+    return launched(e, separate ? 2 : 1);
 }
 
 gist_status gist_pool_relu_bwd(const float *dout, const uint32_t *argmax, const uint32_t *mask, int32_t N, int32_t C,

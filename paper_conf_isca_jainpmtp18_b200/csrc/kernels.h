@@ -12,8 +12,11 @@ int num_sms();
 void count_launches(int k);  // bookkeeping for gist_launch_count()
 
 cudaError_t launch_binarize(const float *y, int64_t n, uint32_t *mask, cudaStream_t s);
+// mask != nullptr: write the a1 mask in the same pass when the geometry allows it
+// (*mask_fused = true); otherwise the caller launches binarize separately.
 cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p,
-                               int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, cudaStream_t s);
+                               int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, cudaStream_t s,
+                               uint32_t *mask = nullptr, bool *mask_fused = nullptr);
 cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uint32_t *mask, int32_t N, int32_t C,
                             int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo, float *dx,
                             cudaStream_t s);

@@ -209,6 +209,55 @@ maxpool_fwd_k2s2_pair_kernel(const float *__restrict__ y, PoolArgs a, float *__r
     }
 }
 
+// 2x2/s2 forward with the a1 mask fused (W % 16 == 0, H even): one warp per output row R owns
+// the word-aligned input block [2R*W, 2R*W + 2W) (rows 2R, 2R+1), so it can assemble every
+// mask word of that block itself: nibbles are OR-ed into a per-warp shared-memory row of words
+// and stored once — the ReLU output is read a single time for pool output, argmax and mask.
+constexpr int kMaskRowWords = 64;  // 2W/32 <= 64  ->  W <= 1024
+
+__global__ void __launch_bounds__(kPoolThreads)
+maxpool_fwd_k2s2_rowmask_kernel(const float *__restrict__ y, PoolArgs a, int64_t out_rows, float *__restrict__ out,
+                                uint32_t *__restrict__ arg, uint32_t *__restrict__ mask) {
+    __shared__ uint32_t s_mask[kPoolThreads / 32][kMaskRowWords];
+    const int lane = threadIdx.x & 31;
+    uint32_t *mw = s_mask[threadIdx.x >> 5];
+    const int pairs = a.Wo >> 1, words = (2 * a.W) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * kPoolThreads) >> 5;
+    for (int64_t R = ((int64_t)blockIdx.x * kPoolThreads + threadIdx.x) >> 5; R < out_rows; R += nwarps) {
+        for (int w = lane; w < words; w += 32) mw[w] = 0u;
+        __syncwarp();
+        const int64_t blk = R * 2 * a.W;  // first input element of the row block (H even)
+        for (int p0 = 0; p0 < pairs; p0 += 32) {
+            const int p = p0 + lane;
+            uint32_t byte = 0;
+            if (p < pairs) {
+                const float4 t = ld_stream_f4(reinterpret_cast<const float4 *>(y + blk + 4 * p));
+                const float4 b = ld_stream_f4(reinterpret_cast<const float4 *>(y + blk + a.W + 4 * p));
+                float m0, m1;
+                uint32_t k0, k1;
+                win4(t.x, t.y, b.x, b.y, m0, k0);
+                win4(t.z, t.w, b.z, b.w, m1, k1);
+                reinterpret_cast<float2 *>(out + R * a.Wo)[p] = make_float2(m0, m1);
+                byte = (k0 | (k1 << 4)) << (8 * (lane & 3));
+                // R1: bit = (y > 0); top quad at block offset 4p, bottom at W + 4p
+                const uint32_t nt = (uint32_t)(t.x > 0.0f) | ((uint32_t)(t.y > 0.0f) << 1) |
+                                    ((uint32_t)(t.z > 0.0f) << 2) | ((uint32_t)(t.w > 0.0f) << 3);
+                const uint32_t nb = (uint32_t)(b.x > 0.0f) | ((uint32_t)(b.y > 0.0f) << 1) |
+                                    ((uint32_t)(b.z > 0.0f) << 2) | ((uint32_t)(b.w > 0.0f) << 3);
+                const int ot = 4 * p, ob = a.W + 4 * p;
+                if (nt) atomicOr(&mw[ot >> 5], nt << (ot & 31));
+                if (nb) atomicOr(&mw[ob >> 5], nb << (ob & 31));
+            }
+            byte |= __shfl_xor_sync(kFull, byte, 1);
+            byte |= __shfl_xor_sync(kFull, byte, 2);
+            if ((lane & 3) == 0 && p < pairs) arg[(R * a.Wo + 2 * p) >> 3] = byte;
+        }
+        __syncwarp();
+        for (int w = lane; w < words; w += 32) mask[(blk >> 5) + w] = mw[w];
+        __syncwarp();
+    }
+}
+
 template <bool EVEN_H>
 __global__ void __launch_bounds__(kPoolThreads)
 pool_bwd_k2s2_pair_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
@@ -766,8 +815,17 @@ unsigned grid_for(int64_t work_items, int64_t items_per_block, int per_sm) {
 }  // namespace
 
 cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p,
-                               int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, cudaStream_t s) {
+                               int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, cudaStream_t s, uint32_t *mask,
+                               bool *mask_fused) {
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
+    if (mask_fused) *mask_fused = false;
+    if (mask && is_k2s2_exact(p, H, W, Ho, Wo) && W % 16 == 0 && H == 2 * Ho && 2 * W / 32 <= kMaskRowWords) {
+        const int64_t rows = (int64_t)N * C * Ho;
+        maxpool_fwd_k2s2_rowmask_kernel<<<grid_for(rows, kPoolThreads / 32, 8), kPoolThreads, 0, s>>>(y, a, rows, out,
+                                                                                                   argmax, mask);
+        if (mask_fused) *mask_fused = true;
+        return cudaPeekAtLastError();
+    }
     const unsigned grid = grid_for(a.n_out, kPoolThreads, 8);
     if (is_k2s2_exact(p, H, W, Ho, Wo) && W % 4 == 0) {
         const unsigned g2 = grid_for(ceil_div(a.n_out / 2, 32 * kPairU), kPoolThreads / 32, 8);

@@ -76,7 +76,7 @@ def pool_case(shape, g, seed, cuda, ties=True):
 
 
 SHAPES = [(1, 1, 5, 7), (2, 3, 13, 13), (1, 64, 56, 56), (2, 5, 27, 27), (1, 7, 14, 14), (3, 2, 55, 55),
-          (1, 3, 9, 16), (2, 4, 12, 24), (1, 1, 1, 1)]
+          (1, 3, 9, 16), (2, 4, 12, 24), (1, 1, 1, 1), (2, 3, 8, 32), (1, 5, 6, 16), (1, 2, 10, 112)]
 
 
 @pytest.mark.parametrize("g", GEOMS, ids=gid)
@@ -231,8 +231,8 @@ def test_full_size_vgg16_relu_pool(gist, ref, cuda, site):
     s = _vgg_site(site)
     shape = (64,) + s.chw
     y = WL.relu_map(shape, 0.8, 3_000_000 + 1, cuda)
-    out, arg, mask = gist.gist_maxpool_fwd_argmax(y, s.pool)
-    mask = gist.gist_binarize_encode(y)
+    out, arg, mask = gist.gist_maxpool_fwd_argmax(y, s.pool, fuse_mask=True)  # fused a1 where possible
+    assert torch.equal(mask, gist.gist_binarize_encode(y))
     dout = WL.grad_map(tuple(out.shape), 17, cuda)
     dx = gist.gist_pool_relu_bwd(dout, arg, mask, shape, s.pool)
     yh = host(y)
