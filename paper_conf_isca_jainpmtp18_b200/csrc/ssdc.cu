@@ -40,8 +40,15 @@ constexpr uint64_t kValueMask = (1ull << 62) - 1;
 struct Workspace {
     uint32_t ticket;
     uint32_t pad;
-    uint64_t desc[1];  // [tiles]
+    uint64_t desc[1];  // [tiles * kDescStride]
 };
+
+#ifndef GIST_SSDC_DESC_STRIDE
+#define GIST_SSDC_DESC_STRIDE 1
+#endif
+// Descriptor spacing in 64-bit words (1: 16 tiles per 128-B L2 line).
+constexpr int kDescStride = GIST_SSDC_DESC_STRIDE;
+__device__ __forceinline__ uint64_t *desc_at(Workspace *ws, int64_t tile) { return &ws->desc[tile * kDescStride]; }
 
 __device__ __forceinline__ uint64_t ld_relaxed(const uint64_t *p) {
     uint64_t v;
@@ -165,7 +172,7 @@ __device__ __forceinline__ int64_t look_back(Workspace *ws, int64_t tile, int la
     for (int64_t base = tile - 1;; base -= 32) {
         if (rounds) ++*rounds;
         const int64_t idx = base - lane;
-        uint64_t d = (idx >= 0) ? ld_relaxed(&ws->desc[idx]) : kStatusP;  // virtual P(0)
+        uint64_t d = (idx >= 0) ? ld_relaxed(desc_at(ws, idx)) : kStatusP;  // virtual P(0)
         uint32_t pm, need;
         for (;;) {
             pm = __ballot_sync(kFull, (d >> 62) == 2);
@@ -173,7 +180,7 @@ __device__ __forceinline__ int64_t look_back(Workspace *ws, int64_t tile, int la
             need = pm ? (((pm & (0u - pm)) << 1) - 1u) : kFull;
             if (!(xm & need)) break;
             if (polls) ++*polls;
-            if ((d >> 62) == 0) d = ld_relaxed(&ws->desc[idx]);
+            if ((d >> 62) == 0) d = ld_relaxed(desc_at(ws, idx));
         }
         const uint64_t v = ((need >> lane) & 1u) ? (d & kValueMask) : 0ull;
         if (pm) {
@@ -184,7 +191,7 @@ __device__ __forceinline__ int64_t look_back(Workspace *ws, int64_t tile, int la
                 if (lane + o < 32) suf += t;
             }
             const int first_p = __ffs(pm) - 1;
-            if (lane < first_p && idx >= 0) st_relaxed(&ws->desc[idx], kStatusP | suf);
+            if (lane < first_p && idx >= 0) st_relaxed(desc_at(ws, idx), kStatusP | suf);
             return excl + (int64_t)__shfl_sync(kFull, suf, 0);
         }
         uint64_t w = v;
@@ -307,7 +314,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                 }
                 if (lane == 31) {
                     S.total[q] = inc;
-                    st_relaxed(&ws->desc[tile], (tile == 0 ? kStatusP : kStatusA) | (uint64_t)inc);
+                    st_relaxed(desc_at(ws, tile), (tile == 0 ? kStatusP : kStatusA) | (uint64_t)inc);
                 }
             }
             __syncwarp();
@@ -345,7 +352,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                 const uint32_t total = S.total[q];
                 if (lane == 0) {
                     S.excl[q] = excl;
-                    if (tile > 0) st_relaxed(&ws->desc[tile], kStatusP | (uint64_t)(excl + total));
+                    if (tile > 0) st_relaxed(desc_at(ws, tile), kStatusP | (uint64_t)(excl + total));
                     if (tile == tiles - 1) *nnz_out = excl + total;
                 }
                 const int64_t r = tile * kTileRows + lane;
@@ -527,7 +534,7 @@ extern "C" int gist_debug_ssdc_trace(void *buf) {
 size_t ssdc_workspace_bytes(int64_t n) {
     const int64_t rows = (n + kRow - 1) / kRow;
     const int64_t tiles = (rows + kTileRows - 1) / kTileRows;
-    return 8 + 8 * (size_t)(tiles > 0 ? tiles : 1);
+    return 8 + 8 * (size_t)kDescStride * (size_t)(tiles > 0 ? tiles : 1);
 }
 
 cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val,
