@@ -1,0 +1,147 @@
+"""Stash-time integration with PyTorch autograd (§IV-B).
+
+Gist's Schedule Builder inserts an encode after a feature map's last
+forward use and a decode before its backward use, so only the encoding lives through the
+long forward->backward gap (Fig 2).  Here the same schedule is expressed with autograd:
+
+* `relu_maxpool(x, pool)` — ReLU->MaxPool pair (Binarize): the forward runs the
+  a2 kernel with the a1 mask fused; autograd saves ONLY the 1-bit mask and the 4-bit argmax
+  map (neither the ReLU output nor the pool output), and the backward is the a3 kernel.
+* `relu_conv(x, conv)` / `stashed_conv(y, conv)` — ReLU->Conv and Pool->Conv (SSDC,
+  P:158-164): the conv input is stashed as exact-size 256-column CSR (a4) and densified just
+  before the conv backward (a5); the dense math stays in cuDNN ("dense compute").
+* `dpr_saved_tensors(bits, params)` — every other stashed activation (DPR,
+  "applicable to any layer combination") is packed to FP16/FP10/FP8 by the a6 kernel when
+  autograd saves it and restored by a7 when the backward unpacks it.
+
+Everything on the encode/decode path is a libgist kernel; torch supplies the dense layers.
+"""
+from __future__ import annotations
+
+import contextlib
+
+import torch
+import torch.nn.functional as F
+
+from . import (gist_dpr_decode, gist_dpr_encode, gist_maxpool_fwd_argmax, gist_pool_relu_bwd,
+               gist_ssdc_decode, gist_ssdc_encode, gist_ssdc_rows, gist_ssdc_workspace_bytes)
+
+
+def _pool_tuple(kernel_size, stride, padding, ceil_mode):
+    k = (kernel_size, kernel_size) if isinstance(kernel_size, int) else tuple(kernel_size)
+    s = k if stride is None else ((stride, stride) if isinstance(stride, int) else tuple(stride))
+    p = (padding, padding) if isinstance(padding, int) else tuple(padding)
+    return (k[0], k[1], s[0], s[1], p[0], p[1], int(bool(ceil_mode)))
+
+
+class _ReLUMaxPool(torch.autograd.Function):
+    @staticmethod
+    def forward(ctx, x, pool):
+        y = torch.relu(x)
+        out, arg, mask = gist_maxpool_fwd_argmax(y.contiguous(), pool, fuse_mask=True)
+        del y  # the fp32 ReLU output is not stashed
+        ctx.save_for_backward(arg, mask)
+        ctx.shape, ctx.pool = tuple(x.shape), pool
+        return out
+
+    @staticmethod
+    def backward(ctx, dout):
+        arg, mask = ctx.saved_tensors
+        return gist_pool_relu_bwd(dout.contiguous(), arg, mask, ctx.shape, ctx.pool), None
+
+
+def relu_maxpool(x, kernel_size, stride=None, padding=0, ceil_mode=False):
+    """max_pool2d(relu(x)) whose stash is the Binarize encoding (mask + argmax map)."""
+    return _ReLUMaxPool.apply(x, _pool_tuple(kernel_size, stride, padding, ceil_mode))
+
+
+class CSRStash:
+    """Exact-size SSDC encoding of a dense fp32 map (one count pass, one encode pass)."""
+
+    def __init__(self, y: torch.Tensor):
+        y = y.contiguous()
+        self.shape, self.n = tuple(y.shape), y.numel()
+        ws = torch.empty(gist_ssdc_workspace_bytes(self.n), dtype=torch.uint8, device=y.device)
+        nnz = torch.empty(1, dtype=torch.int64, device=y.device)
+        row_end = torch.empty(gist_ssdc_rows(self.n), dtype=torch.int32, device=y.device)
+        gist_ssdc_encode(y, capacity=0, row_end=row_end, nnz=nnz, workspace=ws)  # count only
+        k = int(nnz.item())
+        col = torch.empty(max(k, 1), dtype=torch.uint8, device=y.device)
+        val = torch.empty(max(k, 1), dtype=torch.float32, device=y.device)
+        gist_ssdc_encode(y, capacity=k, row_end=row_end, col=col, val=val, nnz=nnz, workspace=ws)
+        self.row_end, self.col, self.val, self.nnz = row_end, col, val, k
+
+    def nbytes(self) -> int:
+        return 5 * self.nnz + 4 * self.row_end.numel()
+
+    def dense(self) -> torch.Tensor:
+        return gist_ssdc_decode(self.row_end, self.col, self.val, self.n).view(self.shape)
+
+
+class _StashedConv(torch.autograd.Function):
+    """conv2d whose saved input is SSDC-encoded; relu=True also applies the preceding ReLU
+    (its backward mask is recovered from the decoded input: y > 0)."""
+
+    @staticmethod
+    def forward(ctx, x, weight, bias, stride, padding, dilation, groups, relu):
+        y = torch.relu(x) if relu else x
+        out = F.conv2d(y, weight, bias, stride, padding, dilation, groups)
+        ctx.csr = CSRStash(y)
+        del y
+        ctx.save_for_backward(weight)
+        ctx.conf = (stride, padding, dilation, groups, relu, bias is not None)
+        return out
+
+    @staticmethod
+    def backward(ctx, dout):
+        (weight,) = ctx.saved_tensors
+        stride, padding, dilation, groups, relu, has_bias = ctx.conf
+        y = ctx.csr.dense()  # decoded just before its backward use
+        ctx.csr = None
+        gx, gw, gb = torch.ops.aten.convolution_backward(
+            dout.contiguous(), y, weight, [weight.shape[0]] if has_bias else None, stride, padding, dilation, False,
+            [0, 0], groups, [True, True, has_bias])
+        if relu:
+            gx.masked_fill_(y == 0, 0.0)  # ReLU backward: y = relu(x) is 0 exactly where x <= 0
+        del y
+        return gx, gw, gb, None, None, None, None, None
+
+
+def relu_conv(x, conv: torch.nn.Conv2d):
+    """conv(relu(x)) with the ReLU output stashed as SSDC (ReLU->Conv)."""
+    return _StashedConv.apply(x, conv.weight, conv.bias, conv.stride, conv.padding, conv.dilation, conv.groups, True)
+
+
+def stashed_conv(y, conv: torch.nn.Conv2d):
+    """conv(y) with its input stashed as SSDC (Pool->Conv)."""
+    return _StashedConv.apply(y, conv.weight, conv.bias, conv.stride, conv.padding, conv.dilation, conv.groups, False)
+
+
+class _DPRPacked:
+    __slots__ = ("words", "n", "shape", "bits")
+
+    def __init__(self, t: torch.Tensor, bits: int):
+        t = t.contiguous()
+        self.n, self.shape, self.bits = t.numel(), tuple(t.shape), bits
+        self.words = gist_dpr_encode(t, bits)
+
+
+@contextlib.contextmanager
+def dpr_saved_tensors(bits: int, params=(), min_numel: int = 4096):
+    """Inside this context, fp32 CUDA activations saved by autograd (not parameters, not tiny
+    tensors) are stored as DPR words and restored to fp32 when the backward unpacks them."""
+    skip = {p.data_ptr() for p in params}
+
+    def pack(t):
+        if (t.is_cuda and t.dtype == torch.float32 and t.numel() >= min_numel and t.data_ptr() not in skip
+                and t.is_contiguous()):
+            return _DPRPacked(t, bits)
+        return t
+
+    def unpack(p):
+        if isinstance(p, _DPRPacked):
+            return gist_dpr_decode(p.words, p.n, p.bits).view(p.shape)
+        return p
+
+    with torch.autograd.graph.saved_tensors_hooks(pack, unpack):
+        yield

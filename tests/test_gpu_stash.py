@@ -1,0 +1,73 @@
+"""f2: stash-time encodings inside PyTorch autograd (paper_conf_isca_jainpmtp18_b200.stash).
+The Binarize and SSDC paths are lossless, so a training step's gradients match
+plain PyTorch up to the dense-layer backward's own rounding; DPR is lossy and stays
+within its format's relative error."""
+import pytest
+import torch
+import torch.nn as nn
+import torch.nn.functional as F
+
+pytestmark = pytest.mark.gpu
+
+
+class TinyVGG(nn.Module):
+    def __init__(self):
+        super().__init__()
+        self.c1, self.c2 = nn.Conv2d(3, 16, 3, padding=1), nn.Conv2d(16, 16, 3, padding=1)
+        self.c3, self.c4 = nn.Conv2d(16, 32, 3, padding=1), nn.Conv2d(32, 32, 3, padding=1)
+        self.fc = nn.Linear(32 * 8 * 8, 10)
+
+    def base(self, x):
+        x = F.max_pool2d(F.relu(self.c2(F.relu(self.c1(x)))), 2)
+        x = F.max_pool2d(F.relu(self.c4(F.relu(self.c3(x)))), 2)
+        return self.fc(torch.flatten(x, 1))
+
+    def gist(self, x, stash):
+        z = stash.relu_conv(self.c1(x), self.c2)
+        z = stash.relu_maxpool(z, 2)
+        z = stash.relu_conv(stash.stashed_conv(z, self.c3), self.c4)
+        z = stash.relu_maxpool(z, 2)
+        return self.fc(torch.flatten(z, 1))
+
+
+def grads(model, fwd, x, y):
+    model.zero_grad(set_to_none=True)
+    F.cross_entropy(fwd(x), y).backward()
+    return [p.grad.clone() for p in model.parameters()]
+
+
+def test_lossless_stash_matches_pytorch(gist, cuda):
+    from paper_conf_isca_jainpmtp18_b200 import stash
+    torch.manual_seed(0)
+    m = TinyVGG().to(cuda)
+    x = torch.randn(8, 3, 32, 32, device=cuda)
+    y = torch.randint(0, 10, (8,), device=cuda)
+    g0 = grads(m, m.base, x, y)
+    g1 = grads(m, lambda t: m.gist(t, stash), x, y)
+    for a, b in zip(g0, g1):
+        torch.testing.assert_close(b, a, rtol=1e-4, atol=1e-5)
+
+
+def test_dpr_saved_tensors_hooks(gist, cuda):
+    from paper_conf_isca_jainpmtp18_b200 import stash
+    torch.manual_seed(1)
+    lin = nn.Linear(4096, 256).to(cuda)
+    x = torch.randn(64, 4096, device=cuda, requires_grad=True)
+    out0 = lin(x)
+    out0.sum().backward()
+    gw0 = lin.weight.grad.clone()
+    lin.weight.grad = None
+    with stash.dpr_saved_tensors(16, lin.parameters()):
+        out1 = lin(x)
+    out1.sum().backward()
+    # the saved input went through FP16: weight grad within fp16 relative error
+    torch.testing.assert_close(lin.weight.grad, gw0, rtol=2e-3, atol=2e-2)
+    assert not torch.equal(lin.weight.grad, gw0)  # the stash really was reduced
+
+
+def test_csr_stash_is_exact_and_small(gist, cuda):
+    from paper_conf_isca_jainpmtp18_b200 import stash
+    y = torch.relu(torch.randn(4, 64, 56, 56, device=cuda) - 0.84)  # ~80% zeros
+    s = stash.CSRStash(y)
+    assert torch.equal(s.dense().view(torch.int32), y.view(torch.int32))
+    assert s.nbytes() < 0.3 * 4 * y.numel()
