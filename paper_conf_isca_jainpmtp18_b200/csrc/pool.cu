@@ -58,14 +58,31 @@ maxpool_fwd_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ 
             const float *plane = y + (int64_t)nc * a.H * a.W;
             float best = -CUDART_INF_F;
             int bi = -1;
-            if (KH && KW && h0 >= 0 && w0 >= 0 && h0 + KH <= a.H && w0 + KW <= a.W) {  // interior window
-                const float *wp = plane + h0 * a.W + w0;
+            if (KH && KW) {
+                // branch-free: out-of-bounds taps read as -inf (never selected under the strict '>'
+                // rule, R3) and the argmax starts at the first in-bounds position, so border and
+                // interior windows run the same instructions (no warp divergence).
+                // When every active lane's window is interior (warp-uniform vote) the bounds
+                // tests are skipped altogether.
                 float v[KH ? KH : 1][KW ? KW : 1];
+                const bool interior = h0 >= 0 && w0 >= 0 && h0 + kh <= a.H && w0 + kw <= a.W;
+                if (__all_sync(__activemask(), interior)) {
 #pragma unroll
-                for (int dy = 0; dy < (KH ? KH : 1); ++dy)
+                    for (int dy = 0; dy < (KH ? KH : 1); ++dy)
 #pragma unroll
-                    for (int dx = 0; dx < (KW ? KW : 1); ++dx) v[dy][dx] = ld_ro(wp + dy * a.W + dx);
-                bi = 0;
+                        for (int dx = 0; dx < (KW ? KW : 1); ++dx) v[dy][dx] = ld_ro(plane + (h0 + dy) * a.W + w0 + dx);
+                    bi = 0;
+                } else {
+#pragma unroll
+                    for (int dy = 0; dy < (KH ? KH : 1); ++dy)
+#pragma unroll
+                        for (int dx = 0; dx < (KW ? KW : 1); ++dx) {
+                            const int ih = h0 + dy, iw = w0 + dx;
+                            const bool in = ih >= 0 && ih < a.H && iw >= 0 && iw < a.W;
+                            v[dy][dx] = in ? ld_ro(plane + ih * a.W + iw) : -CUDART_INF_F;
+                        }
+                    bi = max(0, -h0) * kw + max(0, -w0);
+                }
 #pragma unroll
                 for (int dy = 0; dy < (KH ? KH : 1); ++dy)
 #pragma unroll
@@ -682,7 +699,11 @@ pool_bwd_tiled_k3s2_kernel(const float *__restrict__ dout, const uint32_t *__res
 }
 
 // Same 2x2-block formulation without tiles: candidate windows' dY and nibbles come straight
-// through L1 (neighbouring blocks share them), all loads issued before use.
+// through L1 (neighbouring blocks share them), all loads issued before use.  For 3x3 stride 2
+// each window can only hit block (A, b) = rows 2A..2A+1 x cols 2b..2b+1 through fixed nibbles
+// (nibble = 3*dy + dx):  (A-1,b-1): 8 -> (0,0);  (A-1,b): 6 -> (0,0), 7 -> (0,1);
+// (A,b-1): 2 -> (0,0), 5 -> (1,0);  (A,b): 0 -> (0,0), 1 -> (0,1), 3 -> (1,0), 4 -> (1,1).
+// Windows are visited in ascending output order (R6).
 __global__ void __launch_bounds__(kPoolThreads)
 pool_bwd_k3s2_block_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
                            const uint32_t *__restrict__ mask, PoolArgs a, FastDiv div_wb, FastDiv div_hb,
@@ -693,50 +714,46 @@ pool_bwd_k3s2_block_kernel(const float *__restrict__ dout, const uint32_t *__res
         uint32_t q, b, plane, A;
         div_wb.divmod((uint32_t)t, q, b);
         div_hb.divmod(q, plane, A);
-        float g[2][2];
-        uint32_t nib[2][2];
-        bool ok[2][2];
+        const bool up = A >= 1, left = b >= 1;             // windows (A-1, .) / (., b-1) exist
+        const bool here_r = (int)A < a.Ho, here_c = (int)b < a.Wo;  // windows (A, .) / (., b) exist
+        const int64_t o11 = (int64_t)plane * HoWo + (int64_t)A * a.Wo + b;  // window (A, b)
+        float g[4] = {0.f, 0.f, 0.f, 0.f};
+        uint32_t nb[4] = {15u, 15u, 15u, 15u};  // 15: no window / no hit
+        const bool ok[4] = {up && left, up && here_c, here_r && left, here_r && here_c};
+        const int64_t os[4] = {o11 - a.Wo - 1, o11 - a.Wo, o11 - 1, o11};
 #pragma unroll
-        for (int u = 0; u < 2; ++u)
-#pragma unroll
-            for (int v = 0; v < 2; ++v) {
-                const int oh = (int)A - 1 + u, ow = (int)b - 1 + v;
-                ok[u][v] = oh >= 0 && oh < a.Ho && ow >= 0 && ow < a.Wo;
-                const int64_t o = (int64_t)plane * HoWo + (int64_t)(ok[u][v] ? oh : 0) * a.Wo + (ok[u][v] ? ow : 0);
-                g[u][v] = ld_ro(dout + o);
-                nib[u][v] = (ld_ro(arg + (o >> 3)) >> (4 * (o & 7))) & 0xfu;
+        for (int k = 0; k < 4; ++k)
+            if (ok[k]) {
+                g[k] = ld_ro(dout + os[k]);
+                nb[k] = (ld_ro(arg + (os[k] >> 3)) >> (4 * (os[k] & 7))) & 0xfu;
             }
         const int64_t i00 = (int64_t)plane * HW + (int64_t)(2 * A) * a.W + 2 * (int)b;
-        uint32_t m[2] = {3u, 3u};
+        const bool r1 = 2 * (int)A + 1 < a.H, c1 = 2 * (int)b + 1 < a.W;
+        uint32_t m0 = 3u, m1 = 3u;
         if (mask) {
-#pragma unroll
-            for (int ry = 0; ry < 2; ++ry) {
-                const int64_t i = i00 + (int64_t)ry * a.W;
-                const int64_t ic = (2 * (int)A + ry < a.H) ? i : i00;
-                const uint32_t w0 = ld_ro(mask + (ic >> 5)), w1 = ld_ro(mask + ((ic + 1) >> 5));
-                m[ry] = ((w0 >> (ic & 31)) & 1u) | (((w1 >> ((ic + 1) & 31)) & 1u) << 1);
+            const uint32_t w0 = ld_ro(mask + (i00 >> 5)), w0b = ld_ro(mask + ((i00 + 1) >> 5));
+            m0 = ((w0 >> (i00 & 31)) & 1u) | (((w0b >> ((i00 + 1) & 31)) & 1u) << 1);
+            if (r1) {
+                const int64_t i10 = i00 + a.W;
+                const uint32_t w1 = ld_ro(mask + (i10 >> 5)), w1b = ld_ro(mask + ((i10 + 1) >> 5));
+                m1 = ((w1 >> (i10 & 31)) & 1u) | (((w1b >> ((i10 + 1) & 31)) & 1u) << 1);
             }
         }
-        float acc[2][2] = {{0.0f, 0.0f}, {0.0f, 0.0f}};
-#pragma unroll
-        for (int u = 0; u < 2; ++u)  // ascending output order: (A-1, b-1), (A-1, b), (A, b-1), (A, b)
-#pragma unroll
-            for (int v = 0; v < 2; ++v) {
-                if (!ok[u][v]) continue;
-                const int ry = 2 * (u - 1) + (int)(nib[u][v] / 3u), rx = 2 * (v - 1) + (int)(nib[u][v] % 3u);
-                if (ry == 0 && rx == 0) acc[0][0] = acc[0][0] + g[u][v];
-                if (ry == 0 && rx == 1) acc[0][1] = acc[0][1] + g[u][v];
-                if (ry == 1 && rx == 0) acc[1][0] = acc[1][0] + g[u][v];
-                if (ry == 1 && rx == 1) acc[1][1] = acc[1][1] + g[u][v];
-            }
-#pragma unroll
-        for (int ry = 0; ry < 2; ++ry) {
-            if (2 * (int)A + ry >= a.H) continue;
-#pragma unroll
-            for (int rx = 0; rx < 2; ++rx) {
-                if (2 * (int)b + rx >= a.W) continue;
-                dx[i00 + (int64_t)ry * a.W + rx] = ((m[ry] >> rx) & 1u) ? acc[ry][rx] : 0.0f;
-            }
+        float a00 = 0.0f, a01 = 0.0f, a10 = 0.0f, a11 = 0.0f;  // +0.0f, then ascending o
+        if (nb[0] == 8u) a00 = a00 + g[0];
+        if (nb[1] == 6u) a00 = a00 + g[1];
+        if (nb[1] == 7u) a01 = a01 + g[1];
+        if (nb[2] == 2u) a00 = a00 + g[2];
+        if (nb[2] == 5u) a10 = a10 + g[2];
+        if (nb[3] == 0u) a00 = a00 + g[3];
+        if (nb[3] == 1u) a01 = a01 + g[3];
+        if (nb[3] == 3u) a10 = a10 + g[3];
+        if (nb[3] == 4u) a11 = a11 + g[3];
+        dx[i00] = (m0 & 1u) ? a00 : 0.0f;
+        if (c1) dx[i00 + 1] = (m0 & 2u) ? a01 : 0.0f;
+        if (r1) {
+            dx[i00 + a.W] = (m1 & 1u) ? a10 : 0.0f;
+            if (c1) dx[i00 + a.W + 1] = (m1 & 2u) ? a11 : 0.0f;
         }
     }
 }

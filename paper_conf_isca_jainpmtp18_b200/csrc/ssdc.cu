@@ -100,7 +100,10 @@ __global__ void ssdc_ws_init(uint64_t *ws, int64_t words) {
 #endif
 constexpr int kStages = GIST_SSDC_STAGES;         // raw TMA ring (16 KB tiles)
 constexpr int kRing = GIST_SSDC_RING;            // pending ring entries (compacted, awaiting offset)
-constexpr int kQ = 16;                           // per-CTA tile queue slots (counted .. stored)
+#ifndef GIST_SSDC_QUEUE
+#define GIST_SSDC_QUEUE 16
+#endif
+constexpr int kQ = GIST_SSDC_QUEUE;              // per-CTA tile queue slots (counted .. stored)
 constexpr int kCtasPerSm = GIST_SSDC_CTAS;
 constexpr int kTileElems = kTileRows * kRow;     // 4096 elements
 constexpr uint32_t kTileBytes = kTileElems * 4;  // 16 KB
