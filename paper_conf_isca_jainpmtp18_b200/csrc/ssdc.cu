@@ -78,6 +78,19 @@ __device__ __forceinline__ void trace(int j, int ev) {
 #define TRACE(j, ev)
 #endif
 
+// WAR between generic-proxy reads of a TMA stage and the next TMA write into it: the
+// consumer's mbarrier arrive -> producer's wait already orders them (as in CUTLASS pipelines);
+// fence.proxy.async there stalls until the CTA's in-flight bulk copies land, so it is a
+// measured variant only (GIST_PROXY_FENCE=1).
+#ifndef GIST_PROXY_FENCE
+#define GIST_PROXY_FENCE 0
+#endif
+__device__ __forceinline__ void ring_release_fence() {
+#if GIST_PROXY_FENCE
+    fence_proxy_async_smem();
+#endif
+}
+
 __global__ void ssdc_ws_init(uint64_t *ws, int64_t words) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += (int64_t)gridDim.x * blockDim.x)
         ws[i] = 0ull;
@@ -155,7 +168,7 @@ __device__ __forceinline__ void load_tile(EncSmem &S, int s, int64_t t, const fl
         const int64_t avail = n - t * kTileElems;
         bytes = avail >= kTileElems ? kTileBytes : (uint32_t)((avail * 4) & ~15ll);
     }
-    fence_proxy_async_smem();
+    ring_release_fence();
     mbar_arrive_expect_tx(&S.full[s], bytes);
     if (bytes) tma_load_1d(S.tile[s], x + t * kTileElems, bytes, &S.full[s]);
 }
@@ -290,6 +303,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                     const int from = avail >= kTileElems ? kTileElems : (int)(((avail * 4) & ~15ll) / 4);
                     for (int i = from + lane; i < kTileElems; i += 32)
                         T[i] = (i < avail) ? x[tile * kTileElems + i] : 0.0f;
+                    fence_proxy_async_smem();  // generic writes into a TMA stage (once per call)
                     __syncwarp();
                 }
                 uint32_t mine = 0;  // lane r ends up with row r's count
@@ -434,7 +448,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                     p_hi += on;
                 }
             }
-            fence_proxy_async_smem();  // our reads of the raw stage precede the next TMA write
+            ring_release_fence();  // (variant knob; the mbarrier hand-off orders the reads)
             __syncwarp();
             if (lane == 0) {
                 if (warp == 0) TRACE(j, 4);
@@ -473,6 +487,750 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                 TRACE(j, 5);
                 flag_st64(&S.free_pos, S.ring_end[q]);
                 flag_st(&S.stored, j + 1);
+            }
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
+// Encode v3: count, then compact from a second read served by L2; every CTA keeps its own
+// running prefix over ALL tile totals, so there is no serial look-back chain.
+//
+// Tiles are slices of kSliceRows = 32 rows (32 KB), claimed in ticket order by persistent CTAs
+// (one per SM).  The global offset of tile t is sum(tot[0..t)); a CTA's gatherer sums the
+// published totals from where it stopped for its previous tile up to t-1 — about one grid's
+// worth of totals per tile, loaded in one coalesced round trip — so offsets never wait on
+// another CTA's look-back, only on the (recent) predecessors' counts.  Warp roles per CTA,
+// linked by mbarriers:
+//   * producer (1 lane): claims tiles (pre-claiming the next ticket) and streams each tile's
+//     four 8 KB parts into a kStages3-deep shared-memory ring with 1-D TMA bulk copies
+//     (HBM -> smem; the lines stay in L2 for the second read);
+//   * 4 counter warps (one per part): per-row nonzero bit-pattern counts (R8), stage released;
+//   * publisher warp: tile-local row scan -> rinc[], tile total published (flag | count in one
+//     word) to tot[tile];
+//   * gatherer warp: running prefix over tot[] -> the tile's global offset;
+//   * 8 writer warps (4 rows each): re-read their rows with 128-bit loads (L2 hits; issued one
+//     tile ahead for memory-level parallelism), rank nonzeros with warp ballots, stage them in
+//     shared memory congruent to the output mod 4 and store val/col with 128-/32-bit stores,
+//     plus row_end.
+// A CTA holds at most kQ3 tiles between claim and write-out (bounded L2 footprint).  HBM sees
+// the algorithmic traffic: 4n read once, 5*nnz + 4*rows written.
+#ifndef GIST_SSDC_ALGO
+#define GIST_SSDC_ALGO 4
+#endif
+#ifndef GIST_SSDC3_STAGES
+#define GIST_SSDC3_STAGES 16
+#endif
+#ifndef GIST_SSDC3_Q
+#define GIST_SSDC3_Q 8
+#endif
+#ifndef GIST_SSDC3_KEEP
+#define GIST_SSDC3_KEEP 0
+#endif
+#ifndef GIST_SSDC3_PARTS
+#define GIST_SSDC3_PARTS 4
+#endif
+constexpr int k3Writers = 8;
+constexpr int k2RowsPerWarp = 4;
+constexpr int kSliceRows = k3Writers * k2RowsPerWarp;  // 32 rows = 8192 elements = 32 KB
+constexpr int kParts = GIST_SSDC3_PARTS;               // counter warps = TMA stages per tile
+constexpr int kPartRows = kSliceRows / kParts;
+constexpr int kPartElems = kPartRows * kRow;           // 8 KB per TMA stage (4 parts)
+constexpr int kStages3 = GIST_SSDC3_STAGES;
+constexpr int kQ3 = GIST_SSDC3_Q;
+constexpr int k3Prod = 0, k3Count = 1, k3Pub = k3Count + kParts, k3Gather = k3Pub + 1, k3Writer0 = k3Gather + 1;
+constexpr int k3Threads = 32 * (k3Writer0 + k3Writers);  // 480
+constexpr uint32_t kTotFlag = 0x80000000u;
+constexpr int kStage = k2RowsPerWarp * kRow + 4;  // staged entries per writer warp (+ alignment pad)
+constexpr int kGatherPer = 8;                     // totals per lane per gather round (256 per warp)
+constexpr int kTotOffset = 32;                    // tot[] after the ticket, one 128-B line apart
+static_assert(kStages3 % kParts == 0, "each counter warp owns the stages of its part");
+static_assert(kPartRows % 2 == 0, "counters reduce two rows at a time");
+
+struct __align__(128) Enc3Smem {
+    float raw[kStages3][kPartElems];  // TMA ring (parts of tiles)
+    float vst[k3Writers][kStage];     // per-writer compacted values (congruent to the output mod 4)
+    uint8_t cst[k3Writers][kStage];   // per-writer compacted column bytes
+    uint32_t rcnt[kQ3][kSliceRows];   // per-row nonzero counts
+    uint32_t rinc[kQ3][kSliceRows];   // tile-local inclusive row ends
+    int64_t base[kQ3];                // global offset of the tile
+    int64_t tile[kQ3];                // tile claimed in this slot (>= tiles: no more work)
+    uint64_t full[kStages3], empty[kStages3];
+    uint64_t counted[kQ3], published[kQ3], resolved[kQ3], freed[kQ3];
+};
+
+// The tile totals are self-contained words (flag | count) and nothing else is published with
+// them, so relaxed gpu-scope accesses suffice (no fences, no L1 invalidation).
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t *p) {
+    uint32_t v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed_u32(uint32_t *p, uint32_t v) {
+    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive1(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+// Rows [4w, 4w+4) of tile t: lane l gets cols [4l, 4l+4) in lo[r] and [128+4l, 128+4l+4) in
+// hi[r].  Last use of the data: L2 evict-first.  Elements past n read as zeros (never counted).
+__device__ __forceinline__ void load_rows(const float *__restrict__ x, int64_t n, int64_t t, int w, int lane,
+                                          uint4 (&lo)[k2RowsPerWarp], uint4 (&hi)[k2RowsPerWarp]) {
+#pragma unroll
+    for (int r = 0; r < k2RowsPerWarp; ++r) {
+        const int64_t e0 = (t * kSliceRows + w * k2RowsPerWarp + r) * kRow;
+        const uint4 *p = reinterpret_cast<const uint4 *>(x + e0);
+        if (e0 + kRow <= n) {
+            lo[r] = __ldcs(p + lane);
+            hi[r] = __ldcs(p + 32 + lane);
+        } else {
+            uint32_t v[8];
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                const int64_t e = e0 + (k < 4 ? 4 * lane + k : 128 + 4 * lane + k - 4);
+                v[k] = e < n ? __float_as_uint(x[e]) : 0u;
+            }
+            lo[r] = make_uint4(v[0], v[1], v[2], v[3]);
+            hi[r] = make_uint4(v[4], v[5], v[6], v[7]);
+        }
+    }
+}
+
+__device__ __forceinline__ uint32_t nz4(const uint4 &a) {  // nonzero bit patterns among 4 words
+    return umin(a.x, 1u) + umin(a.y, 1u) + umin(a.z, 1u) + umin(a.w, 1u);
+}
+
+// Writer: compact the 4 rows held in lo/hi (tile t, queue slot q) to val/col, and row_end.
+__device__ __forceinline__ void write_rows(Enc3Smem &S, int q, int64_t t, int64_t rows, int w, int lane,
+                                           const uint4 (&lo)[k2RowsPerWarp], const uint4 (&hi)[k2RowsPerWarp],
+                                           int32_t *__restrict__ row_end, uint8_t *__restrict__ col,
+                                           float *__restrict__ val, int64_t capacity) {
+    const uint32_t lt = (1u << lane) - 1u;
+    const int rw = w * k2RowsPerWarp;
+    const int64_t tile_base = S.base[q];
+    const uint32_t w_excl = rw ? S.rinc[q][rw - 1] : 0u;
+    const uint32_t w_cnt = S.rinc[q][rw + k2RowsPerWarp - 1] - w_excl;
+    const int64_t off = tile_base + w_excl;  // global index of the warp's first entry
+    if (w_cnt) {
+        const int a = (int)(off & 3);  // staging index = a + local index
+        float *vs = S.vst[w];
+        uint8_t *cs = S.cst[w];
+#pragma unroll
+        for (int r = 0; r < k2RowsPerWarp; ++r) {
+            const uint32_t v[8] = {lo[r].x, lo[r].y, lo[r].z, lo[r].w, hi[r].x, hi[r].y, hi[r].z, hi[r].w};
+            uint32_t bal[8];
+#pragma unroll
+            for (int k = 0; k < 8; ++k) bal[k] = __ballot_sync(kFull, v[k] != 0u);
+            const uint32_t q0 = a + (rw + r ? S.rinc[q][rw + r - 1] : 0u) - w_excl;
+            uint32_t p_lo = q0 + __popc(bal[0] & lt) + __popc(bal[1] & lt) + __popc(bal[2] & lt) + __popc(bal[3] & lt);
+            uint32_t p_hi = q0 + __popc(bal[0]) + __popc(bal[1]) + __popc(bal[2]) + __popc(bal[3]) +
+                            __popc(bal[4] & lt) + __popc(bal[5] & lt) + __popc(bal[6] & lt) + __popc(bal[7] & lt);
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                if (v[k]) {
+                    vs[p_lo] = __uint_as_float(v[k]);
+                    cs[p_lo] = (uint8_t)(4 * lane + k);
+                    ++p_lo;
+                }
+            }
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                if (v[4 + k]) {
+                    vs[p_hi] = __uint_as_float(v[4 + k]);
+                    cs[p_hi] = (uint8_t)(128 + 4 * lane + k);
+                    ++p_hi;
+                }
+            }
+        }
+        __syncwarp();
+        // global entries [off, lim) in 4-entry groups g = [4g, 4g+4); staging index 4g - (off & ~3)
+        const int64_t lim = (off + w_cnt < capacity) ? off + w_cnt : capacity;
+        const int64_t g_lo = off >> 2, g_hi = (lim + 3) >> 2;
+        for (int64_t g = g_lo + lane; g < g_hi; g += 32) {
+            const int si = (int)(4 * (g - g_lo));
+            const int64_t e = 4 * g;
+            if (e >= off && e + 4 <= lim) {
+                *reinterpret_cast<float4 *>(val + e) = *reinterpret_cast<const float4 *>(vs + si);
+                *reinterpret_cast<uint32_t *>(col + e) = *reinterpret_cast<const uint32_t *>(cs + si);
+            } else {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    if (e + j >= off && e + j < lim) {
+                        val[e + j] = vs[si + j];
+                        col[e + j] = cs[si + j];
+                    }
+                }
+            }
+        }
+        __syncwarp();
+    }
+    if (lane < k2RowsPerWarp) {
+        const int64_t r = t * kSliceRows + rw + lane;
+        if (r < rows) row_end[r] = (int32_t)(tile_base + S.rinc[q][rw + lane]);
+    }
+}
+
+#ifdef GIST_SSDC3_TRACE
+// Timing experiment only: per (CTA, local tile j) timestamps (%globaltimer, ns): 0 producer
+// issues the tile, 1 tile total published, 2 tile offset resolved, 3 writer 0 done.
+constexpr int kTrace3Tiles = 256;
+__device__ uint64_t *g_trace3 = nullptr;
+__device__ __forceinline__ void trace3(int64_t j, int ev) {
+    if (g_trace3 && j < kTrace3Tiles - 1) {
+        uint64_t t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        g_trace3[((int64_t)blockIdx.x * kTrace3Tiles + j) * 4 + ev] = t;
+    }
+}
+#define TRACE3(j, ev) trace3(j, ev)
+#else
+#define TRACE3(j, ev)
+#endif
+
+__global__ void __launch_bounds__(k3Threads, 1)
+ssdc_encode3_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t tiles,
+                    int32_t *__restrict__ row_end, uint8_t *__restrict__ col, float *__restrict__ val,
+                    int64_t capacity, int64_t *__restrict__ nnz_out, uint32_t *__restrict__ ws) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    Enc3Smem &S = *reinterpret_cast<Enc3Smem *>(smem_raw);
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    uint32_t *ticket = ws;
+    uint32_t *tot = ws + kTotOffset;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kStages3; ++s) {
+            mbar_init(&S.full[s], 1);
+            mbar_init(&S.empty[s], 1);
+        }
+        for (int q = 0; q < kQ3; ++q) {
+            mbar_init(&S.counted[q], kParts);
+            mbar_init(&S.published[q], 1);
+            mbar_init(&S.resolved[q], 1);
+            mbar_init(&S.freed[q], k3Writers);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+
+    if (warp == k3Prod) {
+        // ---- producer: claim tiles in ticket order (next one pre-claimed), stream their parts.
+        // The end ("no more tiles") is a slot whose tile is >= tiles; its parts arrive with 0 bytes.
+        if (lane == 0) {
+#ifdef GIST_SSDC3_TRACE
+            if (g_trace3) {
+                uint32_t smid;
+                asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+                g_trace3[((int64_t)blockIdx.x * kTrace3Tiles + kTrace3Tiles - 1) * 4 + 3] = smid;
+            }
+#endif
+            int64_t t = atomicAdd(ticket, 1u);
+            for (int64_t j = 0;; ++j) {
+                const int q = (int)(j % kQ3);
+                if (j >= kQ3) mbar_wait(&S.freed[q], (uint32_t)(j / kQ3 - 1) & 1u);
+                S.tile[q] = t;
+                TRACE3(j, 0);
+                const int64_t e_tile = t * (int64_t)(kSliceRows * kRow);
+                for (int h = 0; h < kParts; ++h) {
+                    const int64_t js = kParts * j + h;
+                    const int s = (int)(js % kStages3);
+                    if (js >= kStages3) mbar_wait(&S.empty[s], (uint32_t)(js / kStages3 - 1) & 1u);
+                    const int64_t e0 = e_tile + h * kPartElems;
+                    const int64_t avail = t < tiles ? n - e0 : 0;
+                    const uint32_t bytes =
+                        avail >= kPartElems ? kPartElems * 4u : (avail > 0 ? (uint32_t)((avail * 4) & ~15ll) : 0u);
+                    ring_release_fence();
+                    mbar_arrive_expect_tx(&S.full[s], bytes);  // also publishes S.tile[q] to the counter
+                    if (bytes) {
+#if GIST_SSDC3_KEEP
+                        tma_load_1d_keep(S.raw[s], x + e0, bytes, &S.full[s]);
+#else
+                        tma_load_1d_normal(S.raw[s], x + e0, bytes, &S.full[s]);
+#endif
+                    }
+                }
+                if (t >= tiles) break;
+                t = atomicAdd(ticket, 1u);
+            }
+        }
+    } else if (warp >= k3Count && warp < k3Count + kParts) {
+        // ---- counters: part h of every tile; lane r ends up with row r's count
+        const int h = warp - k3Count;
+        for (int64_t j = 0;; ++j) {
+            const int64_t js = kParts * j + h;
+            const int s = (int)(js % kStages3);
+            const int q = (int)(j % kQ3);
+            mbar_wait(&S.full[s], (uint32_t)(js / kStages3) & 1u);
+            const int64_t t = S.tile[q];
+            if (t < tiles) {
+                float *T = S.raw[s];
+                const int64_t e0 = t * (int64_t)(kSliceRows * kRow) + h * kPartElems;
+                const int64_t avail = n - e0;
+                if (avail < kPartElems) {  // ragged end of the map: the part the TMA could not copy, zeros
+                    const int from = avail > 0 ? (int)(((avail * 4) & ~15ll) / 4) : 0;
+                    for (int i = from + lane; i < kPartElems; i += 32) T[i] = (i < avail) ? x[e0 + i] : 0.0f;
+                    fence_proxy_async_smem();  // generic writes into a TMA stage (once per call)
+                    __syncwarp();
+                }
+                uint32_t mine = 0;
+#pragma unroll
+                for (int r = 0; r < kPartRows; r += 2) {  // two rows per reduction (16-bit fields)
+                    const uint4 *row4 = reinterpret_cast<const uint4 *>(T + r * kRow);
+                    const uint4 a0 = row4[lane], b0 = row4[32 + lane], c0 = row4[64 + lane], d0 = row4[96 + lane];
+                    const uint32_t u = __reduce_add_sync(kFull, (nz4(a0) + nz4(b0)) | ((nz4(c0) + nz4(d0)) << 16));
+                    if (lane == r) mine = u & 0xffffu;
+                    if (lane == r + 1) mine = u >> 16;
+                }
+                if (lane < kPartRows) S.rcnt[q][h * kPartRows + lane] = mine;
+            }
+            ring_release_fence();  // (variant knob; the mbarrier hand-off orders the reads)
+            __syncwarp();
+            if (lane == 0) {
+                mbar_arrive1(&S.empty[s]);
+                mbar_arrive1(&S.counted[q]);
+            }
+            if (t >= tiles) break;
+        }
+    } else if (warp == k3Pub) {
+        // ---- publisher: tile-local row scan, tile total -> tot[tile]
+        for (int64_t j = 0;; ++j) {
+            const int q = (int)(j % kQ3);
+            mbar_wait(&S.counted[q], (uint32_t)(j / kQ3) & 1u);
+            const int64_t t = S.tile[q];
+            if (t < tiles) {
+                uint32_t inc = S.rcnt[q][lane];
+#pragma unroll
+                for (int d = 1; d < 32; d <<= 1) {
+                    const uint32_t u = __shfl_up_sync(kFull, inc, d);
+                    if (lane >= d) inc += u;
+                }
+                S.rinc[q][lane] = inc;
+                if (lane == 31) st_relaxed_u32(&tot[t], kTotFlag | inc);
+            }
+            __syncwarp();
+            if (lane == 0) {
+                TRACE3(j, 1);
+                mbar_arrive1(&S.published[q]);
+            }
+            if (t >= tiles) break;
+        }
+    } else if (warp == k3Gather) {
+        // ---- gatherer: running prefix over all tile totals, in tile order.  For each of this
+        // CTA's tiles t: sum tot[pos .. t) (up to 256 totals per coalesced round trip; re-poll
+        // until all are published), base(t) = sum.
+        int64_t pos = 0, sum = 0;
+        for (int64_t j = 0;; ++j) {
+            const int q = (int)(j % kQ3);
+            mbar_wait(&S.published[q], (uint32_t)(j / kQ3) & 1u);
+            const int64_t t = S.tile[q];
+            const int64_t upto = t < tiles ? t : 0;
+            while (pos < upto) {
+                uint32_t v[kGatherPer];
+#pragma unroll
+                for (int i = 0; i < kGatherPer; ++i) {
+                    const int64_t idx = pos + 32 * i + lane;
+                    v[i] = idx < upto ? ld_relaxed_u32(&tot[idx]) : kTotFlag;  // past upto: ready, 0
+                }
+                // the longest fully published prefix of the window
+                int64_t ready = 32 * kGatherPer;
+#pragma unroll
+                for (int i = kGatherPer - 1; i >= 0; --i) {
+                    const uint32_t miss = __ballot_sync(kFull, !(v[i] & kTotFlag));
+                    if (miss) ready = 32 * i + __ffs(miss) - 1;
+                }
+                uint32_t add = 0;
+#pragma unroll
+                for (int i = 0; i < kGatherPer; ++i)
+                    if (32 * i + lane < ready) add += v[i] & ~kTotFlag;
+                sum += (int64_t)__reduce_add_sync(kFull, add);
+                pos += ready;
+                if (pos > upto) pos = upto;
+                if (ready < 32 * kGatherPer && pos < upto) __nanosleep(32);
+            }
+            if (t < tiles) {
+                if (lane == 0) S.base[q] = sum;
+                if (t == tiles - 1 && lane == 0) *nnz_out = sum + S.rinc[q][kSliceRows - 1];
+            }
+            __syncwarp();
+            if (lane == 0) {
+                TRACE3(j, 2);
+                mbar_arrive1(&S.resolved[q]);
+            }
+            if (t >= tiles) break;
+        }
+    } else {
+        // ---- writers: rows [4w, 4w+4) of each tile; the next tile's loads are in flight while
+        // the current one is compacted (two register sets, manual 2x unroll)
+        const int w = warp - k3Writer0;
+        uint4 lo0[k2RowsPerWarp], hi0[k2RowsPerWarp], lo1[k2RowsPerWarp], hi1[k2RowsPerWarp];
+        mbar_wait(&S.published[0], 0u);
+        int64_t t0 = S.tile[0], t1 = tiles;
+        if (t0 < tiles) load_rows(x, n, t0, w, lane, lo0, hi0);
+        for (int64_t j = 0; t0 < tiles; j += 2) {
+            // even j: data in set 0, prefetch j+1 into set 1
+            mbar_wait(&S.published[(j + 1) % kQ3], (uint32_t)((j + 1) / kQ3) & 1u);
+            t1 = S.tile[(j + 1) % kQ3];
+            if (t1 < tiles) load_rows(x, n, t1, w, lane, lo1, hi1);
+            {
+                const int q = (int)(j % kQ3);
+                mbar_wait(&S.resolved[q], (uint32_t)(j / kQ3) & 1u);
+                write_rows(S, q, t0, rows, w, lane, lo0, hi0, row_end, col, val, capacity);
+                __syncwarp();
+                if (lane == 0) {
+                    if (w == 0) TRACE3(j, 3);
+                    mbar_arrive1(&S.freed[q]);
+                }
+            }
+            if (t1 >= tiles) break;
+            // odd j+1: data in set 1, prefetch j+2 into set 0
+            mbar_wait(&S.published[(j + 2) % kQ3], (uint32_t)((j + 2) / kQ3) & 1u);
+            t0 = S.tile[(j + 2) % kQ3];
+            if (t0 < tiles) load_rows(x, n, t0, w, lane, lo0, hi0);
+            {
+                const int q = (int)((j + 1) % kQ3);
+                mbar_wait(&S.resolved[q], (uint32_t)((j + 1) / kQ3) & 1u);
+                write_rows(S, q, t1, rows, w, lane, lo1, hi1, row_end, col, val, capacity);
+                __syncwarp();
+                if (lane == 0) {
+                    if (w == 0) TRACE3(j + 1, 3);
+                    mbar_arrive1(&S.freed[q]);
+                }
+            }
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
+// Encode v4: one pass — compact straight from the TMA stage into a pending ring, publish the
+// tile count at once, and resolve offsets with a per-CTA running prefix over all tile totals.
+//
+// Tiles are kTile4Rows = 16 rows (16 KB); tickets hand out groups of kGroup4 consecutive tiles
+// (32 KB) to persistent CTAs (one per SM) in ticket order.  The global offset of tile t is
+// sum(tot[0..t)).  Warp roles per CTA, linked by mbarriers:
+//   * producer (1 lane): claims groups (next one pre-claimed) and streams each tile into a
+//     kStages4-deep shared-memory ring with one 1-D TMA bulk copy (cp.async.bulk);
+//   * kComp4 compactor warps (tile j goes to warp j % kComp4): warp ballots rank the nonzero bit
+//     patterns (R8) of each row; the tile total is published to tot[tile] (flag | count, one
+//     word) before anything else, then the tile's (value, column) pairs are scattered in
+//     tile-local order into a wrapping pending ring (one 64-bit store per entry) and the stage
+//     is released;
+//   * gatherer warp: running prefix over tot[] (up to 512 totals per coalesced round trip) ->
+//     each of the CTA's tiles gets its global offset as soon as all earlier tiles are counted;
+//   * kStore4 storer warps: copy each resolved tile from the ring to val/col (coalesced) and
+//     write its row_end, in order, then free its ring space and slot.
+// No tile waits on another CTA's look-back; HBM sees the algorithmic traffic only (4n read
+// once, 5*nnz + 4*rows written).
+#ifndef GIST_SSDC4_STAGES
+#define GIST_SSDC4_STAGES 8
+#endif
+#ifndef GIST_SSDC4_COMP
+#define GIST_SSDC4_COMP 4
+#endif
+#ifndef GIST_SSDC4_STORE
+#define GIST_SSDC4_STORE 2
+#endif
+#ifndef GIST_SSDC4_RING
+#define GIST_SSDC4_RING 8192
+#endif
+constexpr int kTile4Rows = 16;
+constexpr int kTile4Elems = kTile4Rows * kRow;    // 4096 elements = 16 KB
+constexpr int kGroup4 = 2;                        // tiles per ticket (32 KB)
+constexpr int kStages4 = GIST_SSDC4_STAGES;
+constexpr int kComp4 = GIST_SSDC4_COMP;
+constexpr int kStore4 = GIST_SSDC4_STORE;
+constexpr int kRing4 = GIST_SSDC4_RING;           // pending (value, column) pairs
+constexpr int kQ4 = 32;                           // tiles in flight per CTA (claim .. stored)
+constexpr int k4Prod = 0, k4Comp = 1, k4Gather = k4Comp + kComp4, k4Store = k4Gather + 1;
+constexpr int k4Threads = 32 * (k4Store + kStore4);
+constexpr uint32_t kTot4Flag = 0x80000000u;
+constexpr int kGather4Per = 16;                   // totals per lane per gather round (512 per warp)
+constexpr int kTot4Offset = 32;                   // tot[] after the ticket, one 128-B line apart
+static_assert(kStages4 % kComp4 == 0, "each compactor owns the stages of its tiles");
+static_assert((kRing4 & (kRing4 - 1)) == 0 && kRing4 >= kTile4Elems, "ring: power of two >= one tile");
+
+struct __align__(128) Enc4Smem {
+    float raw[kStages4][kTile4Elems];   // TMA ring
+    uint2 pend[kRing4];                 // pending (value bits, column) pairs, tile-local order
+    int64_t tile[kQ4];                  // tile of each slot (>= tiles: no more work)
+    int64_t base[kQ4];                  // global offset of the tile (gatherer)
+    int64_t ring_end[kQ4];              // monotonic ring position after the tile
+    uint32_t rinc[kQ4][kTile4Rows];     // tile-local inclusive row ends
+    uint32_t pos[kQ4];                  // ring start of the tile (masked)
+    uint64_t full[kStages4], empty[kStages4];
+    uint64_t counted[kQ4], compacted[kQ4], resolved[kQ4], freed[kQ4];
+    int64_t alloc_pos;                  // monotonic ring allocation cursor (compactors, in tile order)
+    unsigned long long free_pos;        // monotonic ring release cursor (storers; atomic access)
+    int32_t alloc_turn;                 // local tile index allowed to allocate next (atomic access)
+    int32_t last_j;                     // local index of the end marker (atomic access)
+};
+
+#ifdef GIST_SSDC4_TRACE
+// Timing experiment only: per (CTA, local tile j) timestamps (%globaltimer, ns): 0 issued,
+// 1 landed, 2 counted, 3 allocated, 4 compacted, 5 resolved, 6 stored.
+constexpr int kTrace4Tiles = 512;
+__device__ uint64_t *g_trace4 = nullptr;
+__device__ __forceinline__ void trace4(int64_t j, int ev) {
+    if (g_trace4 && j < kTrace4Tiles) {
+        uint64_t t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        g_trace4[((int64_t)blockIdx.x * kTrace4Tiles + j) * 8 + ev] = t;
+    }
+}
+#define TRACE4(j, ev) trace4(j, ev)
+#else
+#define TRACE4(j, ev)
+#endif
+
+__global__ void __launch_bounds__(k4Threads, 1)
+ssdc_encode4_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t tiles,
+                    int32_t *__restrict__ row_end, uint8_t *__restrict__ col, float *__restrict__ val,
+                    int64_t capacity, int64_t *__restrict__ nnz_out, uint32_t *__restrict__ ws) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    Enc4Smem &S = *reinterpret_cast<Enc4Smem *>(smem_raw);
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    uint32_t *ticket = ws;
+    uint32_t *tot = ws + kTot4Offset;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kStages4; ++s) {
+            mbar_init(&S.full[s], 1);
+            mbar_init(&S.empty[s], 1);
+        }
+        for (int q = 0; q < kQ4; ++q) {
+            mbar_init(&S.counted[q], 1);
+            mbar_init(&S.compacted[q], 1);
+            mbar_init(&S.resolved[q], 1);
+            mbar_init(&S.freed[q], 1);
+        }
+        S.alloc_pos = 0;
+        S.free_pos = 0;
+        S.alloc_turn = 0;
+        S.last_j = 0x7fffffff;
+        fence_mbar_init();
+    }
+    __syncthreads();
+
+    if (warp == k4Prod) {
+        // ---- producer: claim groups of tiles in ticket order (next group pre-claimed) and
+        // stream each tile.  The end is a slot whose tile is >= tiles (0-byte arrival).
+        if (lane == 0) {
+            int64_t g = atomicAdd(ticket, 1u);
+            for (int64_t j = 0;; ++j) {
+                const int64_t t = (g < (tiles + kGroup4 - 1) / kGroup4) ? g * kGroup4 + j % kGroup4 : tiles;
+                const int q = (int)(j % kQ4);
+                const int s = (int)(j % kStages4);
+                if (j >= kQ4) mbar_wait_sleep(&S.freed[q], (uint32_t)(j / kQ4 - 1) & 1u);
+                if (j >= kStages4) mbar_wait_sleep(&S.empty[s], (uint32_t)(j / kStages4 - 1) & 1u);
+                const int64_t tt = t < tiles ? t : tiles;
+                S.tile[q] = tt;
+                const int64_t e0 = tt * (int64_t)kTile4Elems;
+                const int64_t avail = tt < tiles ? n - e0 : 0;
+                const uint32_t bytes =
+                    avail >= kTile4Elems ? kTile4Elems * 4u : (avail > 0 ? (uint32_t)((avail * 4) & ~15ll) : 0u);
+                ring_release_fence();
+                TRACE4(j, 0);
+                mbar_arrive_expect_tx(&S.full[s], bytes);  // also publishes S.tile[q] to the compactor
+                if (bytes) tma_load_1d(S.raw[s], x + e0, bytes, &S.full[s]);
+                if (tt >= tiles) break;
+                if (j % kGroup4 == kGroup4 - 1) g = atomicAdd(ticket, 1u);
+            }
+        }
+    } else if (warp >= k4Comp && warp < k4Comp + kComp4) {
+        // ---- compactors: tile j = c, c + kComp4, ... of this CTA.  Lane l holds columns
+        // [4l, 4l+4) ("lo") and [128+4l, 128+4l+4) ("hi") of each row.
+        const int c = warp - k4Comp;
+        const uint32_t lt = (1u << lane) - 1u;
+        for (int64_t j = c;; j += kComp4) {
+            const int s = (int)(j % kStages4);
+            const int q = (int)(j % kQ4);
+            bool ready;  // past the end marker no arrival ever comes for this j
+            while (!(ready = mbar_try(&S.full[s], (uint32_t)(j / kStages4) & 1u, 1000)))
+                if (atomicAdd(&S.last_j, 0) < j) break;
+            if (!ready) break;
+            if (lane == 0) TRACE4(j, 1);
+            const int64_t t = S.tile[q];
+            if (t >= tiles) {  // end marker: tell the other compactors, the gatherer and the storers
+                if (lane == 0) atomicExch(&S.last_j, (int32_t)j);
+                __syncwarp();
+                if (lane == 0) {
+                    mbar_arrive1(&S.counted[q]);
+                    mbar_arrive1(&S.compacted[q]);
+                }
+                break;
+            }
+            float *T = S.raw[s];
+            const int64_t e0 = t * (int64_t)kTile4Elems;
+            const int64_t avail = n - e0;
+            if (avail < kTile4Elems) {  // ragged end of the map: the part the TMA could not copy, zeros
+                const int from = (int)(((avail * 4) & ~15ll) / 4);
+                for (int i = from + lane; i < kTile4Elems; i += 32) T[i] = (i < avail) ? x[e0 + i] : 0.0f;
+                fence_proxy_async_smem();  // generic writes into a TMA stage (once per call)
+                __syncwarp();
+            }
+            // pass 1: ballots -> per-row counts -> tile-local row ends; publish the total
+            uint32_t mine = 0;  // lane r: row r's count
+#pragma unroll
+            for (int r = 0; r < kTile4Rows; ++r) {
+                const uint4 *row4 = reinterpret_cast<const uint4 *>(T + r * kRow);
+                const uint4 a = row4[lane], b2 = row4[32 + lane];
+                const uint32_t cnt = __reduce_add_sync(kFull, nz4(a) + nz4(b2));
+                if (lane == r) mine = cnt;
+            }
+            uint32_t inc = mine;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t u = __shfl_up_sync(kFull, inc, d);
+                if (lane >= d) inc += u;
+            }
+            const uint32_t total = __shfl_sync(kFull, inc, kTile4Rows - 1);
+            if (lane == 0) st_relaxed_u32(&tot[t], kTot4Flag | total);
+            if (lane < kTile4Rows) S.rinc[q][lane] = inc;
+            __syncwarp();
+            if (lane == 0) {
+                TRACE4(j, 2);
+                mbar_arrive1(&S.counted[q]);
+            }
+            // ring space, allocated in local tile order
+            if (lane == 0) {
+                while (atomicAdd(&S.alloc_turn, 0) != (int32_t)j) __nanosleep(32);
+                const int64_t p = S.alloc_pos;
+                while (p + total - (int64_t)atomicAdd(&S.free_pos, 0ull) > kRing4) __nanosleep(64);
+                S.pos[q] = (uint32_t)(p & (kRing4 - 1));
+                S.ring_end[q] = p + total;
+                S.alloc_pos = p + total;
+                __threadfence_block();
+                atomicExch(&S.alloc_turn, (int32_t)(j + 1));
+                TRACE4(j, 3);
+            }
+            __syncwarp();
+            // pass 2: scatter (value, column) pairs in tile-local order
+            const uint32_t rp = S.pos[q];
+            uint2 *ring = S.pend;
+#pragma unroll 4
+            for (int r = 0; r < kTile4Rows; ++r) {
+                const uint4 *row4 = reinterpret_cast<const uint4 *>(T + r * kRow);
+                const uint4 a = row4[lane], b2 = row4[32 + lane];
+                const uint32_t v[8] = {a.x, a.y, a.z, a.w, b2.x, b2.y, b2.z, b2.w};
+                uint32_t bal[8];
+#pragma unroll
+                for (int k = 0; k < 8; ++k) bal[k] = __ballot_sync(kFull, v[k] != 0u);
+                const uint32_t q0 = rp + (r ? S.rinc[q][r - 1] : 0u);
+                uint32_t p_lo = q0 + __popc(bal[0] & lt) + __popc(bal[1] & lt) + __popc(bal[2] & lt) + __popc(bal[3] & lt);
+                uint32_t p_hi = q0 + __popc(bal[0]) + __popc(bal[1]) + __popc(bal[2]) + __popc(bal[3]) +
+                                __popc(bal[4] & lt) + __popc(bal[5] & lt) + __popc(bal[6] & lt) + __popc(bal[7] & lt);
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    if (v[k]) ring[p_lo & (kRing4 - 1)] = make_uint2(v[k], 4u * lane + k);
+                    p_lo += v[k] != 0u;
+                }
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    if (v[4 + k]) ring[p_hi & (kRing4 - 1)] = make_uint2(v[4 + k], 128u + 4u * lane + k);
+                    p_hi += v[4 + k] != 0u;
+                }
+            }
+            ring_release_fence();  // (variant knob; the mbarrier hand-off orders the reads)
+            __syncwarp();
+            if (lane == 0) {
+                TRACE4(j, 4);
+                mbar_arrive1(&S.empty[s]);
+                mbar_arrive1(&S.compacted[q]);
+            }
+        }
+    } else if (warp == k4Gather) {
+        // ---- gatherer: running prefix over all tile totals, in tile order.
+        int64_t pos = 0, sum = 0;
+        for (int64_t j = 0;; ++j) {
+            const int q = (int)(j % kQ4);
+            mbar_wait_sleep(&S.counted[q], (uint32_t)(j / kQ4) & 1u);
+            const int64_t t = S.tile[q];
+            const int64_t upto = t < tiles ? t : 0;
+            while (pos < upto) {
+                uint32_t v[kGather4Per];
+#pragma unroll
+                for (int i = 0; i < kGather4Per; ++i) {
+                    const int64_t idx = pos + 32 * i + lane;
+                    v[i] = idx < upto ? ld_relaxed_u32(&tot[idx]) : kTot4Flag;  // past upto: ready, 0
+                }
+                int64_t ready = 32 * kGather4Per;  // longest fully published prefix of the window
+#pragma unroll
+                for (int i = kGather4Per - 1; i >= 0; --i) {
+                    const uint32_t miss = __ballot_sync(kFull, !(v[i] & kTot4Flag));
+                    if (miss) ready = 32 * i + __ffs(miss) - 1;
+                }
+                uint32_t add = 0;
+#pragma unroll
+                for (int i = 0; i < kGather4Per; ++i)
+                    if (32 * i + lane < ready) add += v[i] & ~kTot4Flag;
+                sum += (int64_t)__reduce_add_sync(kFull, add);
+                pos += ready;
+                if (pos > upto) pos = upto;
+                if (ready < 32 * kGather4Per && pos < upto) __nanosleep(32);
+            }
+            if (t < tiles) {
+                if (lane == 0) S.base[q] = sum;
+                if (t == tiles - 1 && lane == 0) *nnz_out = sum + S.rinc[q][kTile4Rows - 1];
+            }
+            __syncwarp();
+            if (lane == 0) {
+                TRACE4(j, 5);
+                mbar_arrive1(&S.resolved[q]);
+            }
+            if (t >= tiles) break;
+        }
+    } else {
+        // ---- storers: in tile order, copy resolved tiles from the ring to val/col (coalesced)
+        // and write row_end; then free ring space and the slot.
+        const int sl = threadIdx.x - 32 * k4Store;
+        constexpr int kST = 32 * kStore4;
+        for (int64_t j = 0;; ++j) {
+            const int q = (int)(j % kQ4);
+            const uint32_t par = (uint32_t)(j / kQ4) & 1u;
+            mbar_wait_sleep(&S.resolved[q], par);
+            const int64_t t = S.tile[q];
+            if (t >= tiles) break;
+            mbar_wait_sleep(&S.compacted[q], par);
+            const int64_t base = S.base[q];
+            const uint32_t total = S.rinc[q][kTile4Rows - 1];
+            const uint32_t rp = S.pos[q];
+            if (sl < kTile4Rows) {
+                const int64_t r = t * kTile4Rows + sl;
+                if (r < rows) row_end[r] = (int32_t)(base + S.rinc[q][sl]);
+            }
+            int64_t lim = (base + total < capacity) ? base + total : capacity;
+            // output entries [base, lim): aligned groups of 4 with 128-bit / 32-bit stores
+            const int64_t g_lo = base >> 2, g_hi = (lim + 3) >> 2;
+            for (int64_t g = g_lo + sl; g < g_hi; g += kST) {
+                const int64_t e = 4 * g;
+                uint2 pr[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const int64_t ek = e + k;
+                    pr[k] = (ek >= base && ek < lim) ? S.pend[(rp + (uint32_t)(ek - base)) & (kRing4 - 1)]
+                                                     : make_uint2(0u, 0u);
+                }
+                if (e >= base && e + 4 <= lim) {
+                    *reinterpret_cast<uint4 *>(val + e) = make_uint4(pr[0].x, pr[1].x, pr[2].x, pr[3].x);
+                    *reinterpret_cast<uint32_t *>(col + e) =
+                        __byte_perm(__byte_perm(pr[0].y, pr[1].y, 0x0040), __byte_perm(pr[2].y, pr[3].y, 0x0040), 0x5410);
+                } else {
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) {
+                        if (e + k >= base && e + k < lim) {
+                            val[e + k] = __uint_as_float(pr[k].x);
+                            col[e + k] = (uint8_t)pr[k].y;
+                        }
+                    }
+                }
+            }
+            asm volatile("bar.sync 1, %0;" ::"n"(kST) : "memory");
+            if (sl == 0) {
+                __threadfence_block();
+                atomicExch(&S.free_pos, (unsigned long long)S.ring_end[q]);
+                TRACE4(j, 6);
+                mbar_arrive1(&S.freed[q]);
             }
         }
     }
@@ -528,6 +1286,16 @@ ssdc_decode_kernel(const int32_t *__restrict__ row_end, const uint8_t *__restric
 
 }  // namespace
 
+#ifdef GIST_SSDC4_TRACE
+extern "C" int gist_debug_ssdc4_trace(void *buf) {
+    return (int)cudaMemcpyToSymbol(g_trace4, &buf, sizeof(void *));
+}
+#endif
+#ifdef GIST_SSDC3_TRACE
+extern "C" int gist_debug_ssdc3_trace(void *buf) {
+    return (int)cudaMemcpyToSymbol(g_trace3, &buf, sizeof(void *));
+}
+#endif
 #ifdef GIST_SSDC_TRACE
 extern "C" int gist_debug_ssdc_trace(void *buf) {
     return (int)cudaMemcpyToSymbol(g_trace, &buf, sizeof(void *));
@@ -536,18 +1304,48 @@ extern "C" int gist_debug_ssdc_trace(void *buf) {
 
 size_t ssdc_workspace_bytes(int64_t n) {
     const int64_t rows = (n + kRow - 1) / kRow;
+#if GIST_SSDC_ALGO == 4
+    const int64_t tiles = (rows + kTile4Rows - 1) / kTile4Rows;
+    return 4 * (size_t)kTot4Offset + 8 * (size_t)((tiles + 1) / 2);  // ticket line + tot[tiles] uint32
+#elif GIST_SSDC_ALGO == 3
+    const int64_t tiles = (rows + kSliceRows - 1) / kSliceRows;
+    return 4 * (size_t)kTotOffset + 8 * (size_t)((tiles + 1) / 2);  // ticket line + tot[tiles] uint32
+#else
     const int64_t tiles = (rows + kTileRows - 1) / kTileRows;
     return 8 + 8 * (size_t)kDescStride * (size_t)(tiles > 0 ? tiles : 1);
+#endif
 }
 
 cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val,
                                int64_t capacity, int64_t *nnz, void *workspace, cudaStream_t s) {
     const int64_t rows = (n + kRow - 1) / kRow;
-    const int64_t tiles = (rows + kTileRows - 1) / kTileRows;
     const int64_t ws_words = (int64_t)ssdc_workspace_bytes(n) / 8;
     int64_t iblocks = ceil_div(ws_words, 256);
     if (iblocks > 1024) iblocks = 1024;
     ssdc_ws_init<<<(unsigned)iblocks, 256, 0, s>>>(reinterpret_cast<uint64_t *>(workspace), ws_words);
+#if GIST_SSDC_ALGO == 4
+    static std::once_flag attr_once;
+    std::call_once(attr_once, [] {
+        cudaFuncSetAttribute(ssdc_encode4_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(Enc4Smem));
+    });
+    const int64_t tiles = (rows + kTile4Rows - 1) / kTile4Rows;
+    const int64_t groups = (tiles + kGroup4 - 1) / kGroup4;
+    const int64_t grid = groups < num_sms() ? groups : num_sms();
+    ssdc_encode4_kernel<<<(unsigned)grid, k4Threads, sizeof(Enc4Smem), s>>>(
+        x, n, rows, tiles, row_end, col, val, capacity, nnz, reinterpret_cast<uint32_t *>(workspace));
+#elif GIST_SSDC_ALGO == 3
+    // A tile's offset waits for the totals of all earlier tiles, claimed in ticket order by
+    // running CTAs: one persistent CTA per SM (the shared-memory ring allows no more).
+    static std::once_flag attr_once;
+    std::call_once(attr_once, [] {
+        cudaFuncSetAttribute(ssdc_encode3_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(Enc3Smem));
+    });
+    const int64_t tiles = (rows + kSliceRows - 1) / kSliceRows;
+    const int64_t grid = tiles < num_sms() ? tiles : num_sms();
+    ssdc_encode3_kernel<<<(unsigned)grid, k3Threads, sizeof(Enc3Smem), s>>>(
+        x, n, rows, tiles, row_end, col, val, capacity, nnz, reinterpret_cast<uint32_t *>(workspace));
+#else
+    const int64_t tiles = (rows + kTileRows - 1) / kTileRows;
     static std::once_flag attr_once;
     std::call_once(attr_once, [] {
         cudaFuncSetAttribute(ssdc_encode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(EncSmem));
@@ -556,6 +1354,7 @@ cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint
     if (grid > tiles) grid = tiles;
     ssdc_encode_kernel<<<(unsigned)grid, kCtaThreads, sizeof(EncSmem), s>>>(
         x, n, rows, tiles, row_end, col, val, capacity, nnz, reinterpret_cast<Workspace *>(workspace));
+#endif
     return cudaPeekAtLastError();
 }
 

@@ -33,6 +33,23 @@ __device__ __forceinline__ void tma_load_1d(void *dst, const void *src, uint32_t
         : "memory");
 }
 
+// As tma_load_1d, default L2 policy.
+__device__ __forceinline__ void tma_load_1d_normal(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+
+// As tma_load_1d, but L2 evict-last: the data is read again soon (SSDC encode's second pass).
+__device__ __forceinline__ void tma_load_1d_keep(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    asm volatile(
+        "{\n\t.reg .b64 pol;\n\t"
+        "createpolicy.fractional.L2::evict_last.b64 pol, 1.0;\n\t"
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], pol;\n\t}"
+        ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+
 // 1-D bulk copy shared -> global (bytes % 16 == 0, both addresses 16-B aligned), tracked by the
 // issuing thread's bulk async-group.
 __device__ __forceinline__ void tma_store_1d(void *dst, const void *src, uint32_t bytes) {
@@ -71,6 +88,31 @@ __device__ __forceinline__ bool mbar_try(uint64_t *bar, uint32_t parity, uint32_
         : "r"(smem_u32(bar)), "r"(parity), "r"(ns)
         : "memory");
     return ok != 0;
+}
+
+// Wait with the thread suspended in try_wait (time-limit hint, ns) instead of spinning on issue
+// slots; GIST_MBAR_SLEEP_NS = 0 falls back to the plain try_wait loop.
+#ifndef GIST_MBAR_SLEEP_NS
+#define GIST_MBAR_SLEEP_NS 0
+#endif
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) {
+#if GIST_MBAR_SLEEP_NS
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAITS_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
+        "@!p bra WAITS_%=;\n\t}"
+        ::"r"(smem_u32(bar)), "r"(parity), "r"((uint32_t)GIST_MBAR_SLEEP_NS)
+        : "memory");
+#else
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAITS_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAITS_%=;\n\t}"
+        ::"r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+#endif
 }
 
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {

@@ -50,7 +50,7 @@ def test_size_helpers(gist):
     for bits, k in ((16, 2), (10, 3), (8, 4)):
         assert gist.gist_dpr_words(10, bits) == -(-10 // k)
     assert gist.gist_dpr_words(10, 12) == -1
-    assert gist.gist_ssdc_workspace_bytes(1 << 20) >= 8 + 8 * ((1 << 20) // 8192)
+    assert gist.gist_ssdc_workspace_bytes(1 << 20) >= 4 * ((1 << 20) // 8192)  # one flagged total per 32-row slice
     assert gist.gist_pool2d_out_dims(56, 56, (3, 3, 2, 2, 0, 0, 0)) == (27, 27)
     assert gist.gist_pool2d_out_dims(54, 54, (3, 3, 2, 2, 0, 0, 1)) == (27, 27)  # NiN ceil
     assert gist.gist_pool2d_out_dims(112, 112, (3, 3, 2, 2, 0, 0, 1)) == (56, 56)  # GoogLeNet

@@ -130,6 +130,25 @@ def test_ssdc_round_trip(gist, ref, cuda, n, s):
     assert_bits_equal(host(back), ref.ssdc_decode(r_row_end, r_col, r_val, n), "decode vs oracle")
 
 
+# Several encode chunks (one chunk = grid x 8192 elements, ~2.4 M on 148 SMs) with ragged ends.
+@pytest.mark.parametrize("n", [148 * 2 * 8192 + 1, 7_777_777, 25_000_001])
+@pytest.mark.parametrize("s", [0.0, 0.5, 0.9])
+def test_ssdc_multi_chunk(gist, ref, cuda, n, s):
+    x = WL.relu_map((n,), s, n + 17, cuda, negative_zero=True)
+    row_end, col, val, nnz = gist.gist_ssdc_encode(x, trim=True)
+    r_row_end, r_col, r_val = ref.ssdc_encode(host(x))
+    assert int(nnz.item()) == r_col.size
+    assert_bits_equal(host(row_end), r_row_end, "row_end")
+    assert_bits_equal(host(col), r_col, "col")
+    assert_bits_equal(host(val), r_val, "val")
+    cap = r_col.size // 3 + 5
+    row_end2, col2, val2, nnz2 = gist.gist_ssdc_encode(x, capacity=cap)
+    assert int(nnz2.item()) == r_col.size
+    assert_bits_equal(host(row_end2), r_row_end, "row_end (capacity)")
+    assert_bits_equal(host(col2)[:cap], r_col[:cap], "col prefix")
+    assert_bits_equal(host(val2)[:cap], r_val[:cap], "val prefix")
+
+
 def test_ssdc_structured_sparsity(gist, ref, cuda):
     x = WL.relu_map((2, 64, 56, 56), 0.8, 11, cuda, structured=True)
     row_end, col, val, nnz = gist.gist_ssdc_encode(x, trim=True)
