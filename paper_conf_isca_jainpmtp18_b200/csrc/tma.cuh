@@ -33,21 +33,11 @@ __device__ __forceinline__ void tma_load_1d(void *dst, const void *src, uint32_t
         : "memory");
 }
 
-// As tma_load_1d, default L2 policy.
+// As tma_load_1d, default L2 policy (the data is read again soon: SSDC encode's second pass).
 __device__ __forceinline__ void tma_load_1d_normal(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                  ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
                  : "memory");
-}
-
-// As tma_load_1d, but L2 evict-last: the data is read again soon (SSDC encode's second pass).
-__device__ __forceinline__ void tma_load_1d_keep(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
-    asm volatile(
-        "{\n\t.reg .b64 pol;\n\t"
-        "createpolicy.fractional.L2::evict_last.b64 pol, 1.0;\n\t"
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], pol;\n\t}"
-        ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
-        : "memory");
 }
 
 // 1-D bulk copy shared -> global (bytes % 16 == 0, both addresses 16-B aligned), tracked by the
@@ -95,8 +85,24 @@ __device__ __forceinline__ bool mbar_try(uint64_t *bar, uint32_t parity, uint32_
 #ifndef GIST_MBAR_SLEEP_NS
 #define GIST_MBAR_SLEEP_NS 0
 #endif
+#ifndef GIST_MBAR_BACKOFF_NS
+#define GIST_MBAR_BACKOFF_NS 0
+#endif
 __device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) {
-#if GIST_MBAR_SLEEP_NS
+#if GIST_MBAR_BACKOFF_NS
+    uint32_t ok;
+    for (;;) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(ok)
+            : "r"(smem_u32(bar)), "r"(parity)
+            : "memory");
+        if (ok) break;
+        __nanosleep(GIST_MBAR_BACKOFF_NS);
+    }
+#elif GIST_MBAR_SLEEP_NS
     asm volatile(
         "{\n\t.reg .pred p;\n"
         "WAITS_%=:\n\t"

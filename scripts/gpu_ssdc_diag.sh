@@ -1,2 +1,3 @@
 set -x
-timeout 200 python scripts/ssdc4_trace.py 0.8 2>&1 | tail -45
+timeout 900 python -m pytest tests -x -q -m "gpu and not slow" -k "ssdc" 2>&1 | tail -2
+bash scripts/gpu_ssdc_ncu.sh
