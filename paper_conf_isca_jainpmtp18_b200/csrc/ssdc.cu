@@ -133,8 +133,13 @@ __device__ __forceinline__ void load_rows(const float *__restrict__ x, int64_t n
     }
 }
 
+__device__ __forceinline__ uint32_t min1(uint32_t v) {  // 1 if the bit pattern is nonzero (one IMNMX)
+    uint32_t r;
+    asm("min.u32 %0, %1, 1;" : "=r"(r) : "r"(v));
+    return r;
+}
 __device__ __forceinline__ uint32_t nz4(const uint4 &a) {  // nonzero bit patterns among 4 words
-    return umin(a.x, 1u) + umin(a.y, 1u) + umin(a.z, 1u) + umin(a.w, 1u);
+    return min1(a.x) + min1(a.y) + min1(a.z) + min1(a.w);
 }
 
 // Writer: compact the rows held in lo/hi (tile t, queue slot q) to val/col, and row_end.
@@ -163,14 +168,21 @@ __device__ __forceinline__ void write_rows(EncSmem &S, int q, int64_t t, int64_t
             const uint32_t b2 = __ballot_sync(kFull, c & 4u), b3 = __ballot_sync(kFull, c & 8u);
             uint32_t i = p + __popc(b0 & lt) + 2 * __popc(b1 & lt) + 4 * __popc(b2 & lt) + 8 * __popc(b3 & lt);
             p += __popc(b0) + 2 * __popc(b1) + 4 * __popc(b2) + 8 * __popc(b3);
+            // predicated scatter with a running shared-memory address: per element one compare,
+            // two predicated stores (value, column at the same index) and one predicated add
+            uint32_t addr = smem_u32(vs + i);
             const uint32_t c0 = 8u * lane;
 #pragma unroll
             for (int k = 0; k < 8; ++k) {
-                if (v[k]) {
-                    vs[i] = v[k];
-                    cs[i] = c0 + k;
-                }
-                i += v[k] != 0u;
+                asm volatile(
+                    "{\n\t.reg .pred p;\n\t"
+                    "setp.ne.u32 p, %1, 0;\n\t"
+                    "@p st.shared.u32 [%0], %1;\n\t"
+                    "@p st.shared.u32 [%0+%3], %2;\n\t"
+                    "@p add.u32 %0, %0, 4;\n\t}"
+                    : "+r"(addr)
+                    : "r"(v[k]), "r"(c0 + k), "n"(kWriters * kStage * 4)
+                    : "memory");
             }
         }
         __syncwarp();
