@@ -21,6 +21,7 @@ __device__ __forceinline__ uint32_t nib4(float4 v) {
 
 __global__ void __launch_bounds__(kBinThreads)
 binarize_kernel(const float *__restrict__ y, int64_t n, uint32_t *__restrict__ mask) {
+    pdl_enter();
     const int lane = threadIdx.x & 31;
     const int64_t warp = ((int64_t)blockIdx.x * kBinThreads + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * kBinThreads) >> 5;
@@ -69,7 +70,7 @@ cudaError_t launch_binarize(const float *y, int64_t n, uint32_t *mask, cudaStrea
     int64_t blocks = ceil_div(chunks, per_block);
     const int64_t cap = (int64_t)num_sms() * 8;  // 8 resident 256-thread CTAs per SM
     if (blocks > cap) blocks = cap;
-    binarize_kernel<<<(unsigned)blocks, kBinThreads, 0, stream>>>(y, n, mask);
+    launch_k(binarize_kernel, (unsigned)blocks, kBinThreads, 0, stream, y, n, mask);
     return cudaPeekAtLastError();
 }
 

@@ -4,6 +4,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <utility>
+
 namespace gist {
 
 constexpr int kWarp = 32;
@@ -45,6 +47,42 @@ struct FastDiv {
         r = n - q * d;
     }
 };
+
+// Programmatic dependent launch (PDL): every libgist kernel is launched with programmatic
+// stream serialization and starts with pdl_enter(): it lets the next kernel in the stream be
+// scheduled at once (its CTAs' launch and prologue overlap this kernel's tail) and then waits
+// until the previous kernel has completed and its memory is visible (griddepcontrol.wait) before
+// touching global memory.  Stream order of the results is unchanged.  GIST_PDL=0 builds plain
+// <<<>>> launches (A/B knob).
+#ifndef GIST_PDL
+#define GIST_PDL 1
+#endif
+__device__ __forceinline__ void pdl_enter() {
+#if GIST_PDL
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+#endif
+}
+
+template <typename... K, typename... A>
+inline cudaError_t launch_k(void (*kern)(K...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, A &&...args) {
+#if GIST_PDL
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, std::forward<A>(args)...);
+#else
+    kern<<<grid, block, smem, s>>>(std::forward<A>(args)...);
+    return cudaPeekAtLastError();
+#endif
+}
 
 __host__ __device__ __forceinline__ int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 

@@ -116,6 +116,7 @@ __device__ uint32_t encode_word_scalar(const float *x, int64_t n, int64_t w) {
 template <int BITS>
 __global__ void __launch_bounds__(kDprThreads)
 dpr_encode_kernel(const float *__restrict__ x, int64_t n, uint32_t *__restrict__ packed, const int64_t *__restrict__ n_dev) {
+    pdl_enter();
     if (n_dev) n = min(n, *n_dev);  // count known only on the device (DPR over SSDC values)
     constexpr int K = Fmt<BITS>::K;
     constexpr int GF = (BITS == 10) ? 12 : 4;  // floats per group
@@ -170,6 +171,7 @@ dpr_encode_kernel(const float *__restrict__ x, int64_t n, uint32_t *__restrict__
 template <int BITS>
 __global__ void __launch_bounds__(kDprThreads)
 dpr_decode_kernel(const uint32_t *__restrict__ packed, int64_t n, float *__restrict__ x, const int64_t *__restrict__ n_dev) {
+    pdl_enter();
     if (n_dev) n = min(n, *n_dev);  // count known only on the device (DPR over SSDC values)
     constexpr int K = Fmt<BITS>::K;
     constexpr uint32_t FIELD = (1u << BITS) - 1u;
@@ -252,9 +254,9 @@ int64_t dpr_blocks(int64_t n) {
 cudaError_t launch_dpr_encode(const float *x, int64_t n, int bits, uint32_t *packed, cudaStream_t s,
                               const int64_t *n_dev) {
     switch (bits) {
-        case 16: dpr_encode_kernel<16><<<(unsigned)dpr_blocks<16>(n), kDprThreads, 0, s>>>(x, n, packed, n_dev); break;
-        case 10: dpr_encode_kernel<10><<<(unsigned)dpr_blocks<10>(n), kDprThreads, 0, s>>>(x, n, packed, n_dev); break;
-        case 8: dpr_encode_kernel<8><<<(unsigned)dpr_blocks<8>(n), kDprThreads, 0, s>>>(x, n, packed, n_dev); break;
+        case 16: launch_k(dpr_encode_kernel<16>, (unsigned)dpr_blocks<16>(n), kDprThreads, 0, s, x, n, packed, n_dev); break;
+        case 10: launch_k(dpr_encode_kernel<10>, (unsigned)dpr_blocks<10>(n), kDprThreads, 0, s, x, n, packed, n_dev); break;
+        case 8: launch_k(dpr_encode_kernel<8>, (unsigned)dpr_blocks<8>(n), kDprThreads, 0, s, x, n, packed, n_dev); break;
         default: return cudaErrorInvalidValue;
     }
     return cudaPeekAtLastError();
@@ -263,9 +265,9 @@ cudaError_t launch_dpr_encode(const float *x, int64_t n, int bits, uint32_t *pac
 cudaError_t launch_dpr_decode(const uint32_t *packed, int64_t n, int bits, float *x, cudaStream_t s,
                               const int64_t *n_dev) {
     switch (bits) {
-        case 16: dpr_decode_kernel<16><<<(unsigned)dpr_blocks<16>(n), kDprThreads, 0, s>>>(packed, n, x, n_dev); break;
-        case 10: dpr_decode_kernel<10><<<(unsigned)dpr_blocks<10>(n), kDprThreads, 0, s>>>(packed, n, x, n_dev); break;
-        case 8: dpr_decode_kernel<8><<<(unsigned)dpr_blocks<8>(n), kDprThreads, 0, s>>>(packed, n, x, n_dev); break;
+        case 16: launch_k(dpr_decode_kernel<16>, (unsigned)dpr_blocks<16>(n), kDprThreads, 0, s, packed, n, x, n_dev); break;
+        case 10: launch_k(dpr_decode_kernel<10>, (unsigned)dpr_blocks<10>(n), kDprThreads, 0, s, packed, n, x, n_dev); break;
+        case 8: launch_k(dpr_decode_kernel<8>, (unsigned)dpr_blocks<8>(n), kDprThreads, 0, s, packed, n, x, n_dev); break;
         default: return cudaErrorInvalidValue;
     }
     return cudaPeekAtLastError();

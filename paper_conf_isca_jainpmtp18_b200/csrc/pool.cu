@@ -43,6 +43,7 @@ __device__ __forceinline__ void take(float v, int idx, float &best, int &bi) {
 template <int KH, int KW>
 __global__ void __launch_bounds__(kPoolThreads)
 maxpool_fwd_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ out, uint32_t *__restrict__ arg) {
+    pdl_enter();
     const int kh = KH ? KH : a.kh, kw = KW ? KW : a.kw;
     const int lane = threadIdx.x & 31;
     const int64_t chunks = ((int64_t)a.n_out + 31) / 32;
@@ -117,6 +118,7 @@ constexpr int kFwdU = 4;
 __global__ void __launch_bounds__(kPoolThreads)
 maxpool_fwd_k2s2_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ out,
                         uint32_t *__restrict__ arg) {
+    pdl_enter();
     const int lane = threadIdx.x & 31;
     const int64_t chunks = ((int64_t)a.n_out + 31) / 32;
     const int64_t nwarps = ((int64_t)gridDim.x * kPoolThreads) >> 5;
@@ -190,6 +192,7 @@ template <bool EVEN_H>
 __global__ void __launch_bounds__(kPoolThreads)
 maxpool_fwd_k2s2_pair_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ out,
                              uint32_t *__restrict__ arg) {
+    pdl_enter();
     const int lane = threadIdx.x & 31;
     const int64_t pairs = (int64_t)a.n_out / 2;
     const int64_t chunks = (pairs + 31) / 32;
@@ -235,6 +238,7 @@ constexpr int kMaskRowWords = 64;  // 2W/32 <= 64  ->  W <= 1024
 __global__ void __launch_bounds__(kPoolThreads)
 maxpool_fwd_k2s2_rowmask_kernel(const float *__restrict__ y, PoolArgs a, int64_t out_rows, float *__restrict__ out,
                                 uint32_t *__restrict__ arg, uint32_t *__restrict__ mask) {
+    pdl_enter();
     __shared__ uint32_t s_mask[kPoolThreads / 32][kMaskRowWords];
     const int lane = threadIdx.x & 31;
     uint32_t *mw = s_mask[threadIdx.x >> 5];
@@ -279,6 +283,7 @@ template <bool EVEN_H>
 __global__ void __launch_bounds__(kPoolThreads)
 pool_bwd_k2s2_pair_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
                           const uint32_t *__restrict__ mask, PoolArgs a, float *__restrict__ dx) {
+    pdl_enter();
     const int64_t pairs = (int64_t)a.n_out / 2;
     const int64_t stride = (int64_t)gridDim.x * kPoolThreads;
     for (int64_t q0 = (int64_t)blockIdx.x * kPoolThreads + threadIdx.x; q0 < pairs; q0 += stride * kPairU) {
@@ -340,6 +345,7 @@ template <int KH, int KW, int SH, int SW>
 __global__ void __launch_bounds__(kPoolThreads)
 pool_bwd_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg, const uint32_t *__restrict__ mask,
                 PoolArgs a, float *__restrict__ dx) {
+    pdl_enter();
     const int kh = KH ? KH : a.kh, kw = KW ? KW : a.kw;
     const int sh = SH ? SH : a.sh, sw = SW ? SW : a.sw;
     const int64_t stride = (int64_t)gridDim.x * kPoolThreads;
@@ -377,6 +383,7 @@ constexpr int kBwdU = 4;
 __global__ void __launch_bounds__(kPoolThreads)
 pool_bwd_k2s2_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
                      const uint32_t *__restrict__ mask, PoolArgs a, float *__restrict__ dx) {
+    pdl_enter();
     const int64_t stride = (int64_t)gridDim.x * kPoolThreads;
     const bool odd_h = (a.H & 1) != 0;
     for (int64_t o0 = (int64_t)blockIdx.x * kPoolThreads + threadIdx.x; o0 < a.n_out; o0 += stride * kBwdU) {
@@ -512,6 +519,7 @@ template <int KH, int KW>
 __global__ void __launch_bounds__(kTileThreads)
 maxpool_fwd_tiled_kernel(const float *__restrict__ y, PoolArgs a, TileSpec T, float *__restrict__ out,
                          uint32_t *__restrict__ arg) {
+    pdl_enter();
     __shared__ __align__(16) float s_in[kTileIn + 8];
     __shared__ uint8_t s_nib[kTileIn];
     const int kh = KH ? KH : a.kh, kw = KW ? KW : a.kw;
@@ -580,6 +588,7 @@ template <int KH, int KW, int SH, int SW>
 __global__ void __launch_bounds__(kTileThreads)
 pool_bwd_tiled_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
                       const uint32_t *__restrict__ mask, PoolArgs a, TileSpec T, float *__restrict__ dx) {
+    pdl_enter();
     __shared__ __align__(16) float s_dy[kTileIn + 8];
     __shared__ uint32_t s_arg[kTileIn / 8 + 2];
     const int kh = KH ? KH : a.kh, kw = KW ? KW : a.kw, sh = SH ? SH : a.sh, sw = SW ? SW : a.sw;
@@ -636,6 +645,7 @@ __global__ void __launch_bounds__(kTileThreads)
 pool_bwd_tiled_k3s2_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
                            const uint32_t *__restrict__ mask, PoolArgs a, TileSpec T, FastDiv div_wb,
                            FastDiv div_hb, float *__restrict__ dx) {
+    pdl_enter();
     __shared__ __align__(16) float s_dy[kTileIn + 8];
     __shared__ uint32_t s_arg[kTileIn / 8 + 2];
     const int64_t HW = (int64_t)a.H * a.W, HoWo = (int64_t)a.Ho * a.Wo;
@@ -708,6 +718,7 @@ __global__ void __launch_bounds__(kPoolThreads)
 pool_bwd_k3s2_block_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
                            const uint32_t *__restrict__ mask, PoolArgs a, FastDiv div_wb, FastDiv div_hb,
                            int64_t nblk, float *__restrict__ dx) {
+    pdl_enter();
     const int64_t HW = (int64_t)a.H * a.W, HoWo = (int64_t)a.Ho * a.Wo;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < nblk; t += stride) {
@@ -838,7 +849,7 @@ cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, 
     if (mask_fused) *mask_fused = false;
     if (mask && is_k2s2_exact(p, H, W, Ho, Wo) && W % 16 == 0 && H == 2 * Ho && 2 * W / 32 <= kMaskRowWords) {
         const int64_t rows = (int64_t)N * C * Ho;
-        maxpool_fwd_k2s2_rowmask_kernel<<<grid_for(rows, kPoolThreads / 32, 8), kPoolThreads, 0, s>>>(y, a, rows, out,
+        launch_k(maxpool_fwd_k2s2_rowmask_kernel, grid_for(rows, kPoolThreads / 32, 8), kPoolThreads, 0, s, y, a, rows, out,
                                                                                                    argmax, mask);
         if (mask_fused) *mask_fused = true;
         return cudaPeekAtLastError();
@@ -846,23 +857,23 @@ cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, 
     const unsigned grid = grid_for(a.n_out, kPoolThreads, 8);
     if (is_k2s2_exact(p, H, W, Ho, Wo) && W % 4 == 0) {
         const unsigned g2 = grid_for(ceil_div(a.n_out / 2, 32 * kPairU), kPoolThreads / 32, 8);
-        if (H == 2 * Ho) maxpool_fwd_k2s2_pair_kernel<true><<<g2, kPoolThreads, 0, s>>>(y, a, out, argmax);
-        else maxpool_fwd_k2s2_pair_kernel<false><<<g2, kPoolThreads, 0, s>>>(y, a, out, argmax);
+        if (H == 2 * Ho) launch_k(maxpool_fwd_k2s2_pair_kernel<true>, g2, kPoolThreads, 0, s, y, a, out, argmax);
+        else launch_k(maxpool_fwd_k2s2_pair_kernel<false>, g2, kPoolThreads, 0, s, y, a, out, argmax);
     } else if (is_k2s2_exact(p, H, W, Ho, Wo))
-        maxpool_fwd_k2s2_kernel<<<grid_for(ceil_div(a.n_out, kFwdU), kPoolThreads, 8), kPoolThreads, 0, s>>>(y, a, out, argmax);
+        launch_k(maxpool_fwd_k2s2_kernel, grid_for(ceil_div(a.n_out, kFwdU), kPoolThreads, 8), kPoolThreads, 0, s, y, a, out, argmax);
     else if (GIST_POOL_FWD_TILED && tiled_ok(a)) {
         const TileSpec T = make_tiles(a, N * C, false);
         const unsigned gt = (unsigned)std::min<int64_t>(T.tiles, (int64_t)num_sms() * 6);
         if (p.kh == 3 && p.kw == 3)
-            maxpool_fwd_tiled_kernel<3, 3><<<gt, kTileThreads, 0, s>>>(y, a, T, out, argmax);
+            launch_k(maxpool_fwd_tiled_kernel<3, 3>, gt, kTileThreads, 0, s, y, a, T, out, argmax);
         else if (p.kh == 2 && p.kw == 2)
-            maxpool_fwd_tiled_kernel<2, 2><<<gt, kTileThreads, 0, s>>>(y, a, T, out, argmax);
+            launch_k(maxpool_fwd_tiled_kernel<2, 2>, gt, kTileThreads, 0, s, y, a, T, out, argmax);
         else
-            maxpool_fwd_tiled_kernel<0, 0><<<gt, kTileThreads, 0, s>>>(y, a, T, out, argmax);
+            launch_k(maxpool_fwd_tiled_kernel<0, 0>, gt, kTileThreads, 0, s, y, a, T, out, argmax);
     } else if (p.kh == 3 && p.kw == 3)
-        maxpool_fwd_kernel<3, 3><<<grid, kPoolThreads, 0, s>>>(y, a, out, argmax);
+        launch_k(maxpool_fwd_kernel<3, 3>, grid, kPoolThreads, 0, s, y, a, out, argmax);
     else
-        maxpool_fwd_kernel<0, 0><<<grid, kPoolThreads, 0, s>>>(y, a, out, argmax);
+        launch_k(maxpool_fwd_kernel<0, 0>, grid, kPoolThreads, 0, s, y, a, out, argmax);
     return cudaPeekAtLastError();
 }
 
@@ -872,14 +883,14 @@ cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uin
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
     if (is_k2s2_exact(p, H, W, Ho, Wo) && W % 4 == 0) {
         const unsigned g2 = grid_for(ceil_div(a.n_out / 2, kPairU), kPoolThreads, 8);
-        if (H == 2 * Ho) pool_bwd_k2s2_pair_kernel<true><<<g2, kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
-        else pool_bwd_k2s2_pair_kernel<false><<<g2, kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+        if (H == 2 * Ho) launch_k(pool_bwd_k2s2_pair_kernel<true>, g2, kPoolThreads, 0, s, dout, argmax, mask, a, dx);
+        else launch_k(pool_bwd_k2s2_pair_kernel<false>, g2, kPoolThreads, 0, s, dout, argmax, mask, a, dx);
     } else if (is_k2s2_exact(p, H, W, Ho, Wo)) {
-        pool_bwd_k2s2_kernel<<<grid_for(ceil_div(a.n_out, kBwdU), kPoolThreads, 8), kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+        launch_k(pool_bwd_k2s2_kernel, grid_for(ceil_div(a.n_out, kBwdU), kPoolThreads, 8), kPoolThreads, 0, s, dout, argmax, mask, a, dx);
     } else if (GIST_POOL_K3S2_BLOCK && p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2 && p.ph == 0 && p.pw == 0) {
         const int32_t hb = (H + 1) / 2, wb = (W + 1) / 2;
         const int64_t nblk = (int64_t)N * C * hb * wb;
-        pool_bwd_k3s2_block_kernel<<<grid_for(nblk, kPoolThreads, 8), kPoolThreads, 0, s>>>(
+        launch_k(pool_bwd_k3s2_block_kernel, grid_for(nblk, kPoolThreads, 8), kPoolThreads, 0, s, 
             dout, argmax, mask, a, FastDiv::make(wb), FastDiv::make(hb), nblk, dx);
     } else if (tiled_ok(a)) {
         const TileSpec T = make_tiles(a, N * C, true);
@@ -888,22 +899,22 @@ cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uin
             // block rows per tile: multi -> all (H+1)/2 of each plane; band -> TR (last band may be
             // shorter: the kernel bounds t by its own count, the divisor only needs the stride)
             const int32_t hb = T.multi ? (H + 1) / 2 : T.TR + 1;
-            pool_bwd_tiled_k3s2_kernel<<<gt, kTileThreads, 0, s>>>(dout, argmax, mask, a, T, FastDiv::make((W + 1) / 2),
+            launch_k(pool_bwd_tiled_k3s2_kernel, gt, kTileThreads, 0, s, dout, argmax, mask, a, T, FastDiv::make((W + 1) / 2),
                                                                    FastDiv::make(hb), dx);
         } else if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2)
-            pool_bwd_tiled_kernel<3, 3, 2, 2><<<gt, kTileThreads, 0, s>>>(dout, argmax, mask, a, T, dx);
+            launch_k(pool_bwd_tiled_kernel<3, 3, 2, 2>, gt, kTileThreads, 0, s, dout, argmax, mask, a, T, dx);
         else if (p.kh == 3 && p.kw == 3 && p.sh == 1 && p.sw == 1)
-            pool_bwd_tiled_kernel<3, 3, 1, 1><<<gt, kTileThreads, 0, s>>>(dout, argmax, mask, a, T, dx);
+            launch_k(pool_bwd_tiled_kernel<3, 3, 1, 1>, gt, kTileThreads, 0, s, dout, argmax, mask, a, T, dx);
         else
-            pool_bwd_tiled_kernel<0, 0, 0, 0><<<gt, kTileThreads, 0, s>>>(dout, argmax, mask, a, T, dx);
+            launch_k(pool_bwd_tiled_kernel<0, 0, 0, 0>, gt, kTileThreads, 0, s, dout, argmax, mask, a, T, dx);
     } else {
         const unsigned grid = grid_for(a.n_in, kPoolThreads, 8);
         if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2)
-            pool_bwd_kernel<3, 3, 2, 2><<<grid, kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+            launch_k(pool_bwd_kernel<3, 3, 2, 2>, grid, kPoolThreads, 0, s, dout, argmax, mask, a, dx);
         else if (p.kh == 3 && p.kw == 3 && p.sh == 1 && p.sw == 1)
-            pool_bwd_kernel<3, 3, 1, 1><<<grid, kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+            launch_k(pool_bwd_kernel<3, 3, 1, 1>, grid, kPoolThreads, 0, s, dout, argmax, mask, a, dx);
         else
-            pool_bwd_kernel<0, 0, 0, 0><<<grid, kPoolThreads, 0, s>>>(dout, argmax, mask, a, dx);
+            launch_k(pool_bwd_kernel<0, 0, 0, 0>, grid, kPoolThreads, 0, s, dout, argmax, mask, a, dx);
     }
     return cudaPeekAtLastError();
 }

@@ -43,6 +43,7 @@ namespace {
 constexpr int kRow = 256;
 
 __global__ void ssdc_ws_init(uint64_t *ws, int64_t words) {
+    pdl_enter();
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += (int64_t)gridDim.x * blockDim.x)
         ws[i] = 0ull;
 }
@@ -238,6 +239,7 @@ __global__ void __launch_bounds__(kEncThreads, 1)
 ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t tiles,
                     int32_t *__restrict__ row_end, uint8_t *__restrict__ col, float *__restrict__ val,
                     int64_t capacity, int64_t *__restrict__ nnz_out, uint32_t *__restrict__ ws) {
+    pdl_enter();
     extern __shared__ __align__(128) unsigned char smem_raw[];
     EncSmem &S = *reinterpret_cast<EncSmem *>(smem_raw);
     const int lane = threadIdx.x & 31;
@@ -449,6 +451,7 @@ constexpr int kDecRows = 4;  // rows per warp iteration
 __global__ void __launch_bounds__(kDecThreads)
 ssdc_decode_kernel(const int32_t *__restrict__ row_end, const uint8_t *__restrict__ col,
                    const float *__restrict__ val, int64_t n, int64_t rows, float *__restrict__ x) {
+    pdl_enter();
     __shared__ __align__(16) float s_buf[kDecThreads / 32][kDecRows * kRow];
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
@@ -511,7 +514,7 @@ cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint
     const int64_t ws_words = (int64_t)ssdc_workspace_bytes(n) / 8;
     int64_t iblocks = ceil_div(ws_words, 256);
     if (iblocks > 1024) iblocks = 1024;
-    ssdc_ws_init<<<(unsigned)iblocks, 256, 0, s>>>(reinterpret_cast<uint64_t *>(workspace), ws_words);
+    launch_k(ssdc_ws_init, (unsigned)iblocks, 256, 0, s, reinterpret_cast<uint64_t *>(workspace), ws_words);
     // A tile's offset waits for the totals of all earlier tiles, claimed in ticket order by
     // running CTAs: one persistent CTA per SM (the shared-memory ring allows no more).
     static std::once_flag attr_once;
@@ -520,7 +523,7 @@ cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint
     });
     const int64_t tiles = (rows + kTileRows - 1) / kTileRows;
     const int64_t grid = tiles < num_sms() ? tiles : num_sms();
-    ssdc_encode_kernel<<<(unsigned)grid, kEncThreads, sizeof(EncSmem), s>>>(
+    launch_k(ssdc_encode_kernel, (unsigned)grid, kEncThreads, sizeof(EncSmem), s, 
         x, n, rows, tiles, row_end, col, val, capacity, nnz, reinterpret_cast<uint32_t *>(workspace));
     return cudaPeekAtLastError();
 }
@@ -532,7 +535,7 @@ cudaError_t launch_ssdc_decode(const int32_t *row_end, const uint8_t *col, const
     int64_t blocks = ceil_div(groups, kDecThreads / 32);
     const int64_t cap = (int64_t)num_sms() * 6;
     if (blocks > cap) blocks = cap;
-    ssdc_decode_kernel<<<(unsigned)blocks, kDecThreads, 0, s>>>(row_end, col, val, n, rows, x);
+    launch_k(ssdc_decode_kernel, (unsigned)blocks, kDecThreads, 0, s, row_end, col, val, n, rows, x);
     return cudaPeekAtLastError();
 }
 
