@@ -14,6 +14,7 @@
 #include <math_constants.h>
 
 #include <algorithm>
+#include <type_traits>
 
 #include "common.cuh"
 #include "kernels.h"
@@ -229,52 +230,105 @@ maxpool_fwd_k2s2_pair_kernel(const float *__restrict__ y, PoolArgs a, float *__r
     }
 }
 
-// 2x2/s2 forward with the a1 mask fused (W % 16 == 0, H even): one warp per output row R owns
-// the word-aligned input block [2R*W, 2R*W + 2W) (rows 2R, 2R+1), so it can assemble every
-// mask word of that block itself: nibbles are OR-ed into a per-warp shared-memory row of words
-// and stored once — the ReLU output is read a single time for pool output, argmax and mask.
-constexpr int kMaskRowWords = 64;  // 2W/32 <= 64  ->  W <= 1024
+// ---- 2x2/s2 forward with the a1 mask fused, any even W, H even: the map is a sequence of
+// row blocks (input rows 2R, 2R+1 = output row R) that are contiguous in NCHW, so a run of
+// whole blocks is one contiguous range of y, out, argmax nibbles and mask bits.  Runs ("units")
+// of BR blocks with BR*W = 0 mod 16 start on argmax-word and mask-word boundaries, so a warp
+// owns every word of its unit.  Items: V = 4 columns (an output pair, float4 rows, W % 4 == 0)
+// or V = 2 (one output, float2 rows).  Each item's V top and V bottom mask bits go to a per-warp
+// byte buffer (one byte per V-bit unit, in memory order: a block's top units, then its bottom
+// units), which the warp packs into whole mask words at the end of the unit.  y is read once.
+constexpr int kFusedUnitItems = 512;  // items per unit (upper bound; host picks BR)
+constexpr int kFusedU = 4;            // items per lane in flight
 
+template <int V>
 __global__ void __launch_bounds__(kPoolThreads)
-maxpool_fwd_k2s2_rowmask_kernel(const float *__restrict__ y, PoolArgs a, int64_t out_rows, float *__restrict__ out,
-                                uint32_t *__restrict__ arg, uint32_t *__restrict__ mask) {
+maxpool_fwd_k2s2_fused_kernel(const float *__restrict__ y, PoolArgs a, int64_t blocks, int32_t BR, FastDiv div_ipr,
+                              float *__restrict__ out, uint32_t *__restrict__ arg, uint32_t *__restrict__ mask) {
     pdl_enter();
-    __shared__ uint32_t s_mask[kPoolThreads / 32][kMaskRowWords];
+    __shared__ __align__(16) uint8_t s_units[kPoolThreads / 32][2 * kFusedUnitItems + 32];
+    using VecT = typename std::conditional<V == 4, float4, float2>::type;
     const int lane = threadIdx.x & 31;
-    uint32_t *mw = s_mask[threadIdx.x >> 5];
-    const int pairs = a.Wo >> 1, words = (2 * a.W) >> 5;
+    uint8_t *ub = s_units[threadIdx.x >> 5];
+    const int ipr = a.W / V;                      // items per row
+    const int64_t units = (blocks + BR - 1) / BR;
     const int64_t nwarps = ((int64_t)gridDim.x * kPoolThreads) >> 5;
-    for (int64_t R = ((int64_t)blockIdx.x * kPoolThreads + threadIdx.x) >> 5; R < out_rows; R += nwarps) {
-        for (int w = lane; w < words; w += 32) mw[w] = 0u;
-        __syncwarp();
-        const int64_t blk = R * 2 * a.W;  // first input element of the row block (H even)
-        for (int p0 = 0; p0 < pairs; p0 += 32) {
-            const int p = p0 + lane;
-            uint32_t byte = 0;
-            if (p < pairs) {
-                const float4 t = ld_stream_f4(reinterpret_cast<const float4 *>(y + blk + 4 * p));
-                const float4 b = ld_stream_f4(reinterpret_cast<const float4 *>(y + blk + a.W + 4 * p));
-                float m0, m1;
-                uint32_t k0, k1;
-                win4(t.x, t.y, b.x, b.y, m0, k0);
-                win4(t.z, t.w, b.z, b.w, m1, k1);
-                reinterpret_cast<float2 *>(out + R * a.Wo)[p] = make_float2(m0, m1);
-                byte = (k0 | (k1 << 4)) << (8 * (lane & 3));
-                // R1: bit = (y > 0); top quad at block offset 4p, bottom at W + 4p
-                const uint32_t nt = (uint32_t)(t.x > 0.0f) | ((uint32_t)(t.y > 0.0f) << 1) |
-                                    ((uint32_t)(t.z > 0.0f) << 2) | ((uint32_t)(t.w > 0.0f) << 3);
-                const uint32_t nb = (uint32_t)(b.x > 0.0f) | ((uint32_t)(b.y > 0.0f) << 1) |
-                                    ((uint32_t)(b.z > 0.0f) << 2) | ((uint32_t)(b.w > 0.0f) << 3);
-                const int ot = 4 * p, ob = a.W + 4 * p;
-                if (nt) atomicOr(&mw[ot >> 5], nt << (ot & 31));
-                if (nb) atomicOr(&mw[ob >> 5], nb << (ob & 31));
+    for (int64_t u = ((int64_t)blockIdx.x * kPoolThreads + threadIdx.x) >> 5; u < units; u += nwarps) {
+        const int64_t R0 = u * BR;
+        const int nb = (int)((R0 + BR <= blocks) ? BR : blocks - R0);
+        const int ni = nb * ipr;                  // items in this unit
+        const int64_t e0 = R0 * 2 * a.W;          // first input element (word aligned)
+        const int64_t o0 = R0 * a.Wo;             // first output (argmax-word aligned)
+        for (int jb = 0; jb < ni; jb += 32 * kFusedU) {
+            VecT t[kFusedU], bt[kFusedU];
+            uint32_t rb[kFusedU], rp[kFusedU];
+#pragma unroll
+            for (int k = 0; k < kFusedU; ++k) {
+                const int j = jb + 32 * k + lane;
+                if (j < ni) {
+                    div_ipr.divmod((uint32_t)j, rb[k], rp[k]);
+                    const float *p = y + e0 + (int64_t)rb[k] * 2 * a.W + V * rp[k];
+                    t[k] = *reinterpret_cast<const VecT *>(p);   // (streamed: read once)
+                    bt[k] = *reinterpret_cast<const VecT *>(p + a.W);
+                }
             }
-            byte |= __shfl_xor_sync(kFull, byte, 1);
-            byte |= __shfl_xor_sync(kFull, byte, 2);
-            if ((lane & 3) == 0 && p < pairs) arg[(R * a.Wo + 2 * p) >> 3] = byte;
+#pragma unroll
+            for (int k = 0; k < kFusedU; ++k) {
+                const int j = jb + 32 * k + lane;
+                uint32_t part = 0;
+                if (j < ni) {
+                    uint32_t nt, nbm;
+                    if constexpr (V == 4) {
+                        float m0, m1;
+                        uint32_t k0, k1;
+                        win4(t[k].x, t[k].y, bt[k].x, bt[k].y, m0, k0);
+                        win4(t[k].z, t[k].w, bt[k].z, bt[k].w, m1, k1);
+                        reinterpret_cast<float2 *>(out + o0)[j] = make_float2(m0, m1);
+                        part = (k0 | (k1 << 4)) << (8 * (lane & 3));
+                        nt = (uint32_t)(t[k].x > 0.0f) | ((uint32_t)(t[k].y > 0.0f) << 1) |
+                             ((uint32_t)(t[k].z > 0.0f) << 2) | ((uint32_t)(t[k].w > 0.0f) << 3);
+                        nbm = (uint32_t)(bt[k].x > 0.0f) | ((uint32_t)(bt[k].y > 0.0f) << 1) |
+                              ((uint32_t)(bt[k].z > 0.0f) << 2) | ((uint32_t)(bt[k].w > 0.0f) << 3);
+                    } else {
+                        float m;
+                        uint32_t kk;
+                        win4(t[k].x, t[k].y, bt[k].x, bt[k].y, m, kk);
+                        out[o0 + j] = m;
+                        part = kk << (4 * (lane & 7));
+                        nt = (uint32_t)(t[k].x > 0.0f) | ((uint32_t)(t[k].y > 0.0f) << 1);
+                        nbm = (uint32_t)(bt[k].x > 0.0f) | ((uint32_t)(bt[k].y > 0.0f) << 1);
+                    }
+                    // R1 bits of the item's top and bottom units, in memory order
+                    const int ut = (int)rb[k] * 2 * ipr + (int)rp[k];
+                    ub[ut] = (uint8_t)nt;
+                    ub[ut + ipr] = (uint8_t)nbm;
+                }
+                if constexpr (V == 4) {  // 4 items (8 nibbles) per argmax word
+                    part |= __shfl_xor_sync(kFull, part, 1);
+                    part |= __shfl_xor_sync(kFull, part, 2);
+                    if ((lane & 3) == 0 && j < ni) arg[((o0 >> 1) + j) >> 2] = part;
+                } else {                 // 8 items per argmax word
+                    part |= __shfl_xor_sync(kFull, part, 1);
+                    part |= __shfl_xor_sync(kFull, part, 2);
+                    part |= __shfl_xor_sync(kFull, part, 4);
+                    if ((lane & 7) == 0 && j < ni) arg[(o0 + j) >> 3] = part;
+                }
+            }
         }
         __syncwarp();
-        for (int w = lane; w < words; w += 32) mask[(blk >> 5) + w] = mw[w];
+        // pack the unit's mask words: 32 / V units of V bits each
+        constexpr int kPer = 32 / V;
+        const int nu = 2 * ni;
+        const int nw = (nu + kPer - 1) / kPer;
+        for (int w = lane; w < nw; w += 32) {
+            uint32_t word = 0;
+#pragma unroll
+            for (int i = 0; i < kPer; ++i) {
+                const int x = w * kPer + i;
+                if (x < nu) word |= (uint32_t)ub[x] << (V * i);
+            }
+            mask[(e0 >> 5) + w] = word;
+        }
         __syncwarp();
     }
 }
@@ -847,12 +901,24 @@ cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, 
                                bool *mask_fused) {
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
     if (mask_fused) *mask_fused = false;
-    if (mask && is_k2s2_exact(p, H, W, Ho, Wo) && W % 16 == 0 && H == 2 * Ho && 2 * W / 32 <= kMaskRowWords) {
-        const int64_t rows = (int64_t)N * C * Ho;
-        launch_k(maxpool_fwd_k2s2_rowmask_kernel, grid_for(rows, kPoolThreads / 32, 8), kPoolThreads, 0, s, y, a, rows, out,
-                                                                                                   argmax, mask);
-        if (mask_fused) *mask_fused = true;
-        return cudaPeekAtLastError();
+    if (mask && is_k2s2_exact(p, H, W, Ho, Wo) && H == 2 * Ho) {
+        // units of BR whole row blocks with BR*W = 0 mod 16 (word-aligned), ~256 items each
+        const int V = (W % 4 == 0) ? 4 : 2;
+        const int ipr = W / V;
+        int align = 16;
+        for (int g = W; g % 2 == 0 && align > 1; g /= 2) align /= 2;  // 16 / gcd(W, 16)
+        const int64_t blocks = (int64_t)N * C * Ho;
+        int64_t BR = align * std::max<int64_t>(1, 256 / ((int64_t)align * ipr));
+        if (BR * ipr <= kFusedUnitItems) {
+            const unsigned g = grid_for(ceil_div(blocks, BR), kPoolThreads / 32, 8);
+            const FastDiv d = FastDiv::make((uint32_t)ipr);
+            if (V == 4)
+                launch_k(maxpool_fwd_k2s2_fused_kernel<4>, g, kPoolThreads, 0, s, y, a, blocks, (int32_t)BR, d, out, argmax, mask);
+            else
+                launch_k(maxpool_fwd_k2s2_fused_kernel<2>, g, kPoolThreads, 0, s, y, a, blocks, (int32_t)BR, d, out, argmax, mask);
+            if (mask_fused) *mask_fused = true;
+            return cudaPeekAtLastError();
+        }
     }
     const unsigned grid = grid_for(a.n_out, kPoolThreads, 8);
     if (is_k2s2_exact(p, H, W, Ho, Wo) && W % 4 == 0) {

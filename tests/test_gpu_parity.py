@@ -76,7 +76,10 @@ def pool_case(shape, g, seed, cuda, ties=True):
 
 
 SHAPES = [(1, 1, 5, 7), (2, 3, 13, 13), (1, 64, 56, 56), (2, 5, 27, 27), (1, 7, 14, 14), (3, 2, 55, 55),
-          (1, 3, 9, 16), (2, 4, 12, 24), (1, 1, 1, 1), (2, 3, 8, 32), (1, 5, 6, 16), (1, 2, 10, 112)]
+          (1, 3, 9, 16), (2, 4, 12, 24), (1, 1, 1, 1), (2, 3, 8, 32), (1, 5, 6, 16), (1, 2, 10, 112),
+          # fused 2x2/s2 + mask: several word-aligned units with a partial last one (V = 2 and 4),
+          # tiny rows, and a row too wide for one unit (fallback)
+          (2, 9, 14, 14), (3, 7, 28, 28), (1, 3, 6, 6), (1, 1, 2, 2050)]
 
 
 @pytest.mark.parametrize("g", GEOMS, ids=gid)
