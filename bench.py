@@ -101,7 +101,7 @@ class Workload:
                 d["col"] = torch.empty(n, dtype=torch.uint8, device=dev)
                 d["val"] = torch.empty(n, dtype=torch.float32, device=dev)
                 d["nnz"] = self.nnz_all[k_ssdc:k_ssdc + 1]
-                d["ws"] = torch.empty(gist.gist_ssdc_workspace_bytes(n), dtype=torch.uint8, device=dev)
+                d["ws"] = gist.gist_ssdc_workspace(n, dev)
                 k_ssdc += 1
             else:
                 d["y"] = WL.dpr_map(shape, seed, dev)

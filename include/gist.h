@@ -79,9 +79,13 @@ int64_t gist_ssdc_rows(int64_t n);
 /* 5*nnz + 4*rows: SSDC encoded bytes (fp32 value + uint8 column per nonzero, int32 row end
  * per row; R10). */
 int64_t gist_ssdc_bytes(int64_t n, int64_t nnz);
-/* Device workspace gist_ssdc_encode needs for n elements: a tile ticket plus one flagged
- * 32-bit total per 32-row tile (128 + 4*ceil(rows/32) bytes, rounded up to 8). */
+/* Device workspace gist_ssdc_encode needs for n elements: a 128-byte counter line (tile
+ * ticket, finished-CTA count, call epoch) plus one epoch-tagged 64-bit total per 32-row tile
+ * (128 + 8*ceil(rows/32) bytes).  A workspace sized for n serves every n' <= n. */
 size_t gist_ssdc_workspace_bytes(int64_t n);
+/* Zero `bytes` of a workspace on `stream` (cudaMemsetAsync).  Required ONCE before the
+ * workspace's first gist_ssdc_encode; every encode leaves it ready for the next one. */
+gist_status gist_ssdc_workspace_init(void *workspace, size_t bytes, cudaStream_t stream);
 /* ceil(n / k), k = 2, 3, 4 values per 32-bit word for bits = 16, 10, 8; -1 for
  * unsupported bits. */
 int64_t gist_dpr_words(int64_t n, int32_t bits);
@@ -138,10 +142,13 @@ gist_status gist_pool_relu_bwd(const float *dout, const uint32_t *argmax, const 
  *           written; entries beyond are dropped.
  *   nnz     one DEVICE int64, written with the true number of nonzeros.  The encoding is
  *           complete iff *nnz <= capacity (capacity = n is always enough).
- *   workspace [>= gist_ssdc_workspace_bytes(n)] device bytes, scratch (clobbered).
+ *   workspace [>= gist_ssdc_workspace_bytes(n)] device bytes, zeroed once with
+ *           gist_ssdc_workspace_init before its first use; each call leaves it reusable (the
+ *           tile totals carry the call's epoch, so nothing is cleared per call).  One workspace
+ *           must not serve two calls that may run concurrently (different streams).
  * x is streamed from HBM once (tile counts), then re-read from L2 for the compaction; tile
- * offsets come from a running prefix over all tile totals kept by each CTA.  The workspace is
- * zeroed by the call itself (stream-ordered).  TOO_LARGE if n >= 2^31. */
+ * offsets come from a running prefix over all tile totals kept by each CTA.  One kernel launch.
+ * TOO_LARGE if n >= 2^31. */
 gist_status gist_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val,
                              int64_t capacity, int64_t *nnz, void *workspace,
                              size_t workspace_bytes, cudaStream_t stream);

@@ -20,7 +20,7 @@ import torch
 __all__ = [
     "GistError", "Pool2d", "lib", "library_path",
     "gist_binarize_words", "gist_argmax_words", "gist_pool2d_out_dims", "gist_ssdc_rows",
-    "gist_ssdc_bytes", "gist_ssdc_workspace_bytes", "gist_dpr_words", "gist_num_sms", "gist_launch_count",
+    "gist_ssdc_bytes", "gist_ssdc_workspace_bytes", "gist_ssdc_workspace", "gist_ssdc_workspace_init", "gist_dpr_words", "gist_num_sms", "gist_launch_count",
     "gist_binarize_encode", "gist_maxpool_fwd_argmax", "gist_pool_relu_bwd",
     "gist_ssdc_encode", "gist_ssdc_decode", "gist_dpr_encode", "gist_dpr_decode",
     "gist_ssdc_dpr_encode", "gist_ssdc_dpr_decode",
@@ -66,6 +66,7 @@ def _load() -> C.CDLL:
         "gist_ssdc_rows": (i64, [i64]),
         "gist_ssdc_bytes": (i64, [i64, i64]),
         "gist_ssdc_workspace_bytes": (sz, [i64]),
+        "gist_ssdc_workspace_init": (C.c_int, [p, sz, p]),
         "gist_dpr_words": (i64, [i64, i32]),
         "gist_num_sms": (i32, []),
         "gist_launch_count": (C.c_uint64, []),
@@ -142,6 +143,20 @@ def gist_ssdc_workspace_bytes(n: int) -> int:
     return lib.gist_ssdc_workspace_bytes(n)
 
 
+def gist_ssdc_workspace_init(workspace: torch.Tensor, stream=None) -> torch.Tensor:
+    """Zero a gist_ssdc_encode workspace (required once before its first use)."""
+    _check(lib.gist_ssdc_workspace_init(_ptr(workspace), workspace.numel() * workspace.element_size(),
+                                        _stream(workspace, stream)), "gist_ssdc_workspace_init")
+    return workspace
+
+
+def gist_ssdc_workspace(n: int, device, stream=None) -> torch.Tensor:
+    """A workspace for gist_ssdc_encode of up to n elements, initialised with
+    gist_ssdc_workspace_init (once; every encode leaves it reusable)."""
+    ws = torch.empty(max(gist_ssdc_workspace_bytes(n), 1), dtype=torch.uint8, device=device)
+    return gist_ssdc_workspace_init(ws, stream)
+
+
 def gist_dpr_words(n: int, bits: int) -> int:
     return lib.gist_dpr_words(n, bits)
 
@@ -210,7 +225,7 @@ def gist_ssdc_encode(x: torch.Tensor, capacity: int | None = None, row_end=None,
         nnz = torch.empty(1, dtype=torch.int64, device=dev)
     wsb = gist_ssdc_workspace_bytes(n)
     if workspace is None:
-        workspace = torch.empty(wsb, dtype=torch.uint8, device=dev)
+        workspace = gist_ssdc_workspace(n, dev, stream)
     _check(lib.gist_ssdc_encode(_ptr(x), n, _ptr(row_end), _ptr(col), _ptr(val), cap, _ptr(nnz),
                                 _ptr(workspace), workspace.numel() * workspace.element_size(), _stream(x, stream)),
            "gist_ssdc_encode")

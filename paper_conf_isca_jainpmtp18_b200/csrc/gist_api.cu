@@ -178,7 +178,14 @@ gist_status gist_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_
     if (n == 0) {  // still publish nnz = 0 (stream-ordered)
         return cudaMemsetAsync(nnz, 0, sizeof(int64_t), stream) == cudaSuccess ? GIST_OK : GIST_ERR_CUDA;
     }
-    return launched(gist::launch_ssdc_encode(x, n, row_end, col, val, capacity, nnz, workspace, stream), 2);
+    return launched(gist::launch_ssdc_encode(x, n, row_end, col, val, capacity, nnz, workspace, stream), 1);
+}
+
+gist_status gist_ssdc_workspace_init(void *workspace, size_t bytes, cudaStream_t stream) {
+    if (bytes == 0) return GIST_OK;
+    if (!workspace) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(workspace)) return GIST_ERR_MISALIGNED;
+    return cudaMemsetAsync(workspace, 0, bytes, stream) == cudaSuccess ? GIST_OK : GIST_ERR_CUDA;
 }
 
 gist_status gist_ssdc_decode(const int32_t *row_end, const uint8_t *col, const float *val, int64_t n, float *x,

@@ -20,8 +20,8 @@
 //   * gatherer warp: running prefix over tot[] -> the tile's global offset, and row_end;
 //   * 16 writer warps (2 rows each): re-read their rows with 128-bit loads (L2 hits; issued one
 //     tile ahead), rank nonzeros (lane l owns columns [8l, 8l+8); lane prefix from the ballots of
-//     the 4 bits of the lane counts), stage them in shared memory congruent to the output mod 4
-//     and store val/col with 128-/32-bit stores.
+//     the 4 bits of the lane counts), stage them in shared memory congruent to the output mod 16
+//     and store the whole 16-entry groups of val/col with two 1-D bulk copies (shared -> global).
 // A CTA holds at most kQ tiles between claim and write-out (bounded L2 footprint).  HBM sees
 // the algorithmic traffic: 4n read once, 5*nnz + 4*rows written (ncu: DRAM read = 4n).
 // The encode is issue-bound (~9k warp-instructions per 32 KB tile at ~80% issue utilisation);
@@ -41,12 +41,6 @@ namespace gist {
 namespace {
 
 constexpr int kRow = 256;
-
-__global__ void ssdc_ws_init(uint64_t *ws, int64_t words) {
-    pdl_enter();
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += (int64_t)gridDim.x * blockDim.x)
-        ws[i] = 0ull;
-}
 
 #ifndef GIST_SSDC_STAGES
 #define GIST_SSDC_STAGES 16
@@ -75,17 +69,21 @@ constexpr int kStages = GIST_SSDC_STAGES;
 constexpr int kQ = GIST_SSDC_Q;
 constexpr int kProd = 0, kCount = 1, kPub = kCount + kParts, kGather = kPub + 1, kWriter0 = kGather + 1;
 constexpr int kEncThreads = 32 * (kWriter0 + kWriters);  // 480
-constexpr uint32_t kTotFlag = 0x80000000u;
-constexpr int kStage = kWRows * kRow + 4;  // staged entries per writer warp (+ alignment pad)
+constexpr int kStage = kWRows * kRow + 16;  // staged entries per writer warp (+ 16-entry phase)
 constexpr int kGatherPer = 8;                     // totals per lane per gather round (256 per warp)
-constexpr int kTotOffset = 32;                    // tot[] after the ticket, one 128-B line apart
+// Workspace (zeroed once by the caller, left reusable by every call): u32 words ticket [0],
+// done [1] (CTAs finished), epoch [2] (calls completed); u64 tot[tiles] from word kTotOffset.
+// tot[t] = (epoch + 1) << 32 | count: the tag makes the previous call's totals read as
+// unpublished, so no per-call clearing is needed.  The last CTA to finish resets ticket and
+// done and advances the epoch.
+constexpr int kTotOffset = 32;                    // tot[] one 128-B line after the counters
 static_assert(kStages % kParts == 0, "each counter warp owns the stages of its part");
 static_assert(kPartRows % 2 == 0, "counters reduce two rows at a time");
 
 struct __align__(128) EncSmem {
     float raw[kStages][kPartElems];  // TMA ring (parts of tiles)
     uint32_t vst[kWriters][kStage];  // per-writer compacted value bits (congruent to the output mod 4)
-    uint32_t cst[kWriters][kStage];  // per-writer compacted columns (same index; packed at store)
+    uint8_t cst[kWriters][kStage];   // per-writer compacted columns (bytes, same index)
     uint32_t rcnt[kQ][kTileRows];   // per-row nonzero counts
     uint32_t rinc[kQ][kTileRows];   // tile-local inclusive row ends
     int64_t base[kQ];                // global offset of the tile
@@ -94,15 +92,15 @@ struct __align__(128) EncSmem {
     uint64_t counted[kQ], published[kQ], resolved[kQ], freed[kQ];
 };
 
-// The tile totals are self-contained words (flag | count) and nothing else is published with
+// The tile totals are self-contained words (tag | count) and nothing else is published with
 // them, so relaxed gpu-scope accesses suffice (no fences, no L1 invalidation).
-__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t *p) {
-    uint32_t v;
-    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+__device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p) {
+    uint64_t v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
-__device__ __forceinline__ void st_relaxed_u32(uint32_t *p, uint32_t v) {
-    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+__device__ __forceinline__ void st_relaxed_u64(uint64_t *p, uint64_t v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 __device__ __forceinline__ void mbar_arrive1(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
@@ -143,79 +141,78 @@ __device__ __forceinline__ uint32_t nz4(const uint4 &a) {  // nonzero bit patter
     return min1(a.x) + min1(a.y) + min1(a.z) + min1(a.w);
 }
 
-// Writer: compact the rows held in lo/hi (tile t, queue slot q) to val/col, and row_end.
-// Per row: lane count c (0..8), exclusive lane prefix from the ballots of c's 4 bits, then the
-// lane's nonzeros go to consecutive staging slots (value and column at the same index).
-__device__ __forceinline__ void write_rows(EncSmem &S, int q, int64_t t, int64_t rows, int w, int lane,
-                                           const uint4 (&lo)[kWRows], const uint4 (&hi)[kWRows],
-                                           int32_t *__restrict__ row_end, uint8_t *__restrict__ col,
+// Writer: compact the rows held in lo/hi (queue slot q) to val/col.  Per row: lane count c
+// (0..8), exclusive lane prefix from the ballots of c's 4 bits, then the lane's nonzeros go to
+// consecutive staging slots (value word and column byte at the same index).  The staging is
+// congruent to the output mod 16 entries, so the whole 16-entry groups of val (64 B) and col (16 B) leave as two 1-D bulk copies
+// (cp.async.bulk shared -> global) issued by lane 0; the ragged head and tail (< 16 entries
+// each) by lanes 0..15 and 16..31.
+__device__ __forceinline__ void write_rows(EncSmem &S, int q, int w, int lane, const uint4 (&lo)[kWRows],
+                                           const uint4 (&hi)[kWRows], uint8_t *__restrict__ col,
                                            float *__restrict__ val, int64_t capacity) {
     const uint32_t lt = (1u << lane) - 1u;
     const int rw = w * kWRows;
     const int64_t tile_base = S.base[q];
     const uint32_t w_excl = rw ? S.rinc[q][rw - 1] : 0u;
     const uint32_t w_cnt = S.rinc[q][rw + kWRows - 1] - w_excl;
-    const int64_t off = tile_base + w_excl;  // global index of the warp's first entry
-    if (w_cnt) {
-        const int a = (int)(off & 3);  // staging index = a + local index
-        uint32_t *vs = S.vst[w];
-        uint32_t *cs = S.cst[w];
-        uint32_t p = a;  // staging index of the row's first entry
+    const int64_t off = tile_base + w_excl;
+    if (w_cnt == 0 || off >= capacity) return;
+    uint32_t *vs = S.vst[w];
+    uint8_t *cs = S.cst[w];
+    if (lane == 0) bulk_wait_read();  // the previous tile's bulk copies have read the staging
+    __syncwarp();
+    uint32_t p = (uint32_t)(off & 15);
 #pragma unroll
-        for (int r = 0; r < kWRows; ++r) {
-            const uint32_t v[8] = {lo[r].x, lo[r].y, lo[r].z, lo[r].w, hi[r].x, hi[r].y, hi[r].z, hi[r].w};
-            const uint32_t c = nz4(lo[r]) + nz4(hi[r]);
-            const uint32_t b0 = __ballot_sync(kFull, c & 1u), b1 = __ballot_sync(kFull, c & 2u);
-            const uint32_t b2 = __ballot_sync(kFull, c & 4u), b3 = __ballot_sync(kFull, c & 8u);
-            uint32_t i = p + __popc(b0 & lt) + 2 * __popc(b1 & lt) + 4 * __popc(b2 & lt) + 8 * __popc(b3 & lt);
-            p += __popc(b0) + 2 * __popc(b1) + 4 * __popc(b2) + 8 * __popc(b3);
-            // predicated scatter with a running shared-memory address: per element one compare,
-            // two predicated stores (value, column at the same index) and one predicated add
-            uint32_t addr = smem_u32(vs + i);
-            const uint32_t c0 = 8u * lane;
+    for (int r = 0; r < kWRows; ++r) {
+        const uint32_t v[8] = {lo[r].x, lo[r].y, lo[r].z, lo[r].w, hi[r].x, hi[r].y, hi[r].z, hi[r].w};
+        const uint32_t c = nz4(lo[r]) + nz4(hi[r]);
+        const uint32_t b0 = __ballot_sync(kFull, c & 1u), b1 = __ballot_sync(kFull, c & 2u);
+        const uint32_t b2 = __ballot_sync(kFull, c & 4u), b3 = __ballot_sync(kFull, c & 8u);
+        const uint32_t i = p + __popc(b0 & lt) + 2 * __popc(b1 & lt) + 4 * __popc(b2 & lt) + 8 * __popc(b3 & lt);
+        p += __popc(b0) + 2 * __popc(b1) + 4 * __popc(b2) + 8 * __popc(b3);
+        uint32_t addr = smem_u32(vs + i), caddr = smem_u32(cs + i);
+        const uint32_t c0 = 8u * lane;
 #pragma unroll
-            for (int k = 0; k < 8; ++k) {
-                asm volatile(
-                    "{\n\t.reg .pred p;\n\t"
-                    "setp.ne.u32 p, %1, 0;\n\t"
-                    "@p st.shared.u32 [%0], %1;\n\t"
-                    "@p st.shared.u32 [%0+%3], %2;\n\t"
-                    "@p add.u32 %0, %0, 4;\n\t}"
-                    : "+r"(addr)
-                    : "r"(v[k]), "r"(c0 + k), "n"(kWriters * kStage * 4)
-                    : "memory");
-            }
+        for (int k = 0; k < 8; ++k) {
+            asm volatile(
+                "{\n\t.reg .pred p;\n\t"
+                "setp.ne.u32 p, %2, 0;\n\t"
+                "@p st.shared.u32 [%0], %2;\n\t"
+                "@p st.shared.u8 [%1], %3;\n\t"
+                "@p add.u32 %0, %0, 4;\n\t"
+                "@p add.u32 %1, %1, 1;\n\t}"
+                : "+r"(addr), "+r"(caddr)
+                : "r"(v[k]), "r"(c0 + k)
+                : "memory");
         }
-        __syncwarp();
-        // global entries [off, lim): whole 4-entry groups [4g, 4g+4) with 128-/32-bit stores
-        // (staging index 4g - (off & ~3)); the ragged head and tail (< 4 entries each) by lanes
-        // 0..3 and 4..7 with scalar stores.
-        const int64_t lim = (off + w_cnt < capacity) ? off + w_cnt : capacity;
-        const int64_t base4 = off & ~3ll;
-        const int64_t g_lo = (off + 3) >> 2, g_hi = lim >> 2;  // whole groups [g_lo, g_hi)
-        {
-            const int ng = (int)(g_hi - g_lo);           // whole groups (may be <= 0)
-            const int s0 = (int)(4 * g_lo - base4);      // staging index of the first one
-            uint4 *vo = reinterpret_cast<uint4 *>(val + 4 * g_lo);
-            uint32_t *co = reinterpret_cast<uint32_t *>(col + 4 * g_lo);
-            for (int k = lane; k < ng; k += 32) {
-                const uint4 cc = *reinterpret_cast<const uint4 *>(cs + s0 + 4 * k);
-                vo[k] = *reinterpret_cast<const uint4 *>(vs + s0 + 4 * k);
-                co[k] = __byte_perm(__byte_perm(cc.x, cc.y, 0x0040), __byte_perm(cc.z, cc.w, 0x0040), 0x5410);
-            }
-        }
-        if (lane < 8) {
-            // lanes 0..3: entries 4*g_lo - 4 + lane (head, below the first whole group);
-            // lanes 4..7: entries 4*g_hi + lane - 4 (tail)
-            const int64_t e = lane < 4 ? 4 * g_lo - 4 + lane : 4 * g_hi + lane - 4;
-            const bool in_range = e >= off && e < lim && (lane < 4 ? e < 4 * g_lo : true) && (g_hi >= g_lo || lane < 4);
-            if (in_range) {
-                val[e] = __uint_as_float(vs[e - base4]);
-                col[e] = (uint8_t)cs[e - base4];
-            }
-        }
-        __syncwarp();
     }
+    const int64_t lim = (off + w_cnt < capacity) ? off + w_cnt : capacity;
+    const int64_t base16 = off & ~15ll;                     // staging index of entry e: e - base16
+    const int64_t g_lo = (off + 15) >> 4, g_hi = lim >> 4;  // whole 16-entry groups [g_lo, g_hi)
+    fence_proxy_async_smem();  // generic staging writes -> async-proxy bulk reads
+    __syncwarp();
+    if (g_hi > g_lo) {
+        if (lane == 0) {
+            const int s0 = (int)(16 * g_lo - base16);
+            const uint32_t ng = (uint32_t)(g_hi - g_lo);
+            tma_store_1d(val + 16 * g_lo, vs + s0, 64u * ng);
+            tma_store_1d(col + 16 * g_lo, cs + s0, 16u * ng);
+            bulk_commit();
+        }
+        // head [off, 16 g_lo) by lanes 0..15, tail [16 g_hi, lim) by lanes 16..31
+        const int64_t e = lane < 16 ? 16 * g_lo - 16 + lane : 16 * g_hi + lane - 16;
+        if (e >= off && e < lim) {
+            val[e] = __uint_as_float(vs[e - base16]);
+            col[e] = cs[e - base16];
+        }
+    } else {
+        // no whole 16-entry group: fewer than 32 entries
+        for (int64_t e = off + lane; e < lim; e += 32) {
+            val[e] = __uint_as_float(vs[e - base16]);
+            col[e] = cs[e - base16];
+        }
+    }
+    __syncwarp();
 }
 
 #ifdef GIST_SSDC_TRACE
@@ -245,7 +242,9 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     uint32_t *ticket = ws;
-    uint32_t *tot = ws + kTotOffset;
+    uint64_t *tot = reinterpret_cast<uint64_t *>(ws + kTotOffset);
+    // every CTA reads the epoch before it counts itself done, so all see the same value
+    const uint64_t tag = (uint64_t)(*reinterpret_cast<volatile uint32_t *>(ws + 2) + 1u) << 32;
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < kStages; ++s) {
@@ -348,7 +347,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                     if (lane >= d) inc += u;
                 }
                 S.rinc[q][lane] = inc;
-                if (lane == 31) st_relaxed_u32(&tot[t], kTotFlag | inc);
+                if (lane == 31) st_relaxed_u64(&tot[t], tag | inc);
             }
             __syncwarp();
             if (lane == 0) {
@@ -368,23 +367,23 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
             const int64_t t = S.tile[q];
             const int64_t upto = t < tiles ? t : 0;
             while (pos < upto) {
-                uint32_t v[kGatherPer];
+                uint64_t v[kGatherPer];
 #pragma unroll
                 for (int i = 0; i < kGatherPer; ++i) {
                     const int64_t idx = pos + 32 * i + lane;
-                    v[i] = idx < upto ? ld_relaxed_u32(&tot[idx]) : kTotFlag;  // past upto: ready, 0
+                    v[i] = idx < upto ? ld_relaxed_u64(&tot[idx]) : tag;  // past upto: ready, 0
                 }
                 // the longest fully published prefix of the window
                 int64_t ready = 32 * kGatherPer;
 #pragma unroll
                 for (int i = kGatherPer - 1; i >= 0; --i) {
-                    const uint32_t miss = __ballot_sync(kFull, !(v[i] & kTotFlag));
+                    const uint32_t miss = __ballot_sync(kFull, (v[i] >> 32) != (tag >> 32));
                     if (miss) ready = 32 * i + __ffs(miss) - 1;
                 }
                 uint32_t add = 0;
 #pragma unroll
                 for (int i = 0; i < kGatherPer; ++i)
-                    if (32 * i + lane < ready) add += v[i] & ~kTotFlag;
+                    if (32 * i + lane < ready) add += (uint32_t)v[i];
                 sum += (int64_t)__reduce_add_sync(kFull, add);
                 pos += ready;
                 if (pos > upto) pos = upto;
@@ -421,7 +420,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
         auto retire = [&](int64_t jj, int64_t t, const uint4 (&l)[kWRows], const uint4 (&h)[kWRows]) {
             const int q = (int)(jj % kQ);
             mbar_wait_sleep(&S.resolved[q], (uint32_t)(jj / kQ) & 1u);
-            write_rows(S, q, t, rows, w, lane, l, h, row_end, col, val, capacity);
+            write_rows(S, q, w, lane, l, h, col, val, capacity);
             __syncwarp();
             if (lane == 0) {
                 if (w == 0) TRACE(jj, 3);
@@ -442,6 +441,14 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
             }
         }
     writers_done:;
+        if (lane == 0) bulk_wait_all();
+    }
+    // the last CTA to finish leaves the workspace ready for the next call
+    __syncthreads();
+    if (threadIdx.x == 0 && atomicAdd(ws + 1, 1u) == gridDim.x - 1) {
+        ws[0] = 0u;
+        ws[1] = 0u;
+        ws[2] += 1u;
     }
 }
 
@@ -505,16 +512,12 @@ extern "C" int gist_debug_ssdc_trace(void *buf) {
 size_t ssdc_workspace_bytes(int64_t n) {
     const int64_t rows = (n + kRow - 1) / kRow;
     const int64_t tiles = (rows + kTileRows - 1) / kTileRows;
-    return 4 * (size_t)kTotOffset + 8 * (size_t)((tiles + 1) / 2);  // ticket line + tot[tiles] uint32
+    return 4 * (size_t)kTotOffset + 8 * (size_t)tiles;  // counters line + tot[tiles] uint64
 }
 
 cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val,
                                int64_t capacity, int64_t *nnz, void *workspace, cudaStream_t s) {
     const int64_t rows = (n + kRow - 1) / kRow;
-    const int64_t ws_words = (int64_t)ssdc_workspace_bytes(n) / 8;
-    int64_t iblocks = ceil_div(ws_words, 256);
-    if (iblocks > 1024) iblocks = 1024;
-    launch_k(ssdc_ws_init, (unsigned)iblocks, 256, 0, s, reinterpret_cast<uint64_t *>(workspace), ws_words);
     // A tile's offset waits for the totals of all earlier tiles, claimed in ticket order by
     // running CTAs: one persistent CTA per SM (the shared-memory ring allows no more).
     static std::once_flag attr_once;

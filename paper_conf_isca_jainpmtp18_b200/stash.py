@@ -24,7 +24,7 @@ import torch
 import torch.nn.functional as F
 
 from . import (gist_dpr_decode, gist_dpr_encode, gist_maxpool_fwd_argmax, gist_pool_relu_bwd,
-               gist_ssdc_decode, gist_ssdc_encode, gist_ssdc_rows, gist_ssdc_workspace_bytes)
+               gist_ssdc_decode, gist_ssdc_encode, gist_ssdc_rows, gist_ssdc_workspace)
 
 
 def _pool_tuple(kernel_size, stride, padding, ceil_mode):
@@ -61,7 +61,7 @@ class CSRStash:
     def __init__(self, y: torch.Tensor):
         y = y.contiguous()
         self.shape, self.n = tuple(y.shape), y.numel()
-        ws = torch.empty(gist_ssdc_workspace_bytes(self.n), dtype=torch.uint8, device=y.device)
+        ws = gist_ssdc_workspace(self.n, y.device)
         nnz = torch.empty(1, dtype=torch.int64, device=y.device)
         row_end = torch.empty(gist_ssdc_rows(self.n), dtype=torch.int32, device=y.device)
         gist_ssdc_encode(y, capacity=0, row_end=row_end, nnz=nnz, workspace=ws)  # count only

@@ -1,0 +1,1 @@
+for shp in 64x512x14x14 64x256x28x28 64x64x224x224; do timeout 120 python scripts/ssdc_trace.py 0.8 $shp 2>&1 | tail -9; done

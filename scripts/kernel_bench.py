@@ -105,7 +105,7 @@ def main():
             del yy, m2, oo, aa, dd, dxx
 
     # SSDC on VGG16 relu1_1 b64 (822 MB) across the paper's sparsity range
-    ws = torch.empty(gist.gist_ssdc_workspace_bytes(n), dtype=torch.uint8, device=dev)
+    ws = gist.gist_ssdc_workspace(n, dev)
     row_end = torch.empty(words(n, 256), dtype=torch.int32, device=dev)
     col = torch.empty(n, dtype=torch.uint8, device=dev)
     val = torch.empty(n, dtype=torch.float32, device=dev)

@@ -17,8 +17,10 @@ fn = gist.lib.gist_debug_ssdc_trace
 fn.argtypes = [ctypes.c_void_p]
 fn.restype = ctypes.c_int
 s = float(sys.argv[1]) if len(sys.argv) > 1 else 0.8
-x = WL.relu_map((64, 64, 224, 224), s, 5, dev)
-ws = torch.empty(gist.gist_ssdc_workspace_bytes(x.numel()), dtype=torch.uint8, device=dev)
+shape = tuple(int(v) for v in sys.argv[2].split("x")) if len(sys.argv) > 2 else (64, 64, 224, 224)
+x = WL.relu_map(shape, s, 5, dev)
+print("shape", shape, "tiles", -(-x.numel() // 8192))
+ws = gist.gist_ssdc_workspace(x.numel(), dev)
 out = gist.gist_ssdc_encode(x, workspace=ws)
 torch.cuda.synchronize()
 print("set", fn(buf.data_ptr()))
@@ -47,5 +49,9 @@ for run in range(4):
     print(f"  per-CTA tile period (writer) median {np.median(per):.2f} us p90 {np.percentile(per, 90):.2f}")
     end = np.nanmax(T[:, :, 3], axis=1)
     print(f"  CTA end time: min {np.nanmin(end):.1f} median {np.nanmedian(end):.1f} max {np.nanmax(end):.1f} us")
+    first = T[:, 0, :]
+    print("  first tile: issue min %.2f max %.2f | publish med %.2f | resolved med %.2f max %.2f | written med %.2f max %.2f" % (
+        np.nanmin(first[:, 0]), np.nanmax(first[:, 0]), np.nanmedian(first[:, 1]), np.nanmedian(first[:, 2]),
+        np.nanmax(first[:, 2]), np.nanmedian(first[:, 3]), np.nanmax(first[:, 3])))
     lo = np.argsort(cnt)[:6]
     print("  fewest tiles (cta, smid, tiles):", [(int(c), int(smid[c]), int(cnt[c])) for c in lo])

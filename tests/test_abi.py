@@ -50,7 +50,7 @@ def test_size_helpers(gist):
     for bits, k in ((16, 2), (10, 3), (8, 4)):
         assert gist.gist_dpr_words(10, bits) == -(-10 // k)
     assert gist.gist_dpr_words(10, 12) == -1
-    assert gist.gist_ssdc_workspace_bytes(1 << 20) >= 4 * ((1 << 20) // 8192)  # one flagged total per 32-row slice
+    assert gist.gist_ssdc_workspace_bytes(1 << 20) == 128 + 8 * ((1 << 20) // 8192)  # counters + one tagged total per tile
     assert gist.gist_pool2d_out_dims(56, 56, (3, 3, 2, 2, 0, 0, 0)) == (27, 27)
     assert gist.gist_pool2d_out_dims(54, 54, (3, 3, 2, 2, 0, 0, 1)) == (27, 27)  # NiN ceil
     assert gist.gist_pool2d_out_dims(112, 112, (3, 3, 2, 2, 0, 0, 1)) == (56, 56)  # GoogLeNet
@@ -110,6 +110,9 @@ def test_validation_without_gpu(gist):
     assert L.gist_ssdc_encode(A, 1 << 20, B, B + (1 << 24), B + (1 << 26), 1 << 20, B + (1 << 28), B + (1 << 29),
                               8, None) == INVALID  # workspace too small
     assert L.gist_ssdc_encode(A, 1024, B, None, None, 0, B + 4100, B + 8192, 4096, None) == MISALIGNED  # nnz
+    assert L.gist_ssdc_workspace_init(None, 0, None) == OK  # nothing to zero: no CUDA call
+    assert L.gist_ssdc_workspace_init(None, 256, None) == INVALID
+    assert L.gist_ssdc_workspace_init(B + 4, 256, None) == MISALIGNED
     # f1: DPR over SSDC values (device count)
     assert L.gist_ssdc_dpr_encode(A, B, 0, 16, B + 64, None) == OK
     assert L.gist_ssdc_dpr_encode(A, B, 100, 12, B + 64, None) == UNSUPPORTED

@@ -177,13 +177,31 @@ def test_ssdc_capacity(gist, ref, cuda, cap_frac):
 
 def test_ssdc_repeated_calls_reuse_workspace(gist, ref, cuda):
     n = 256 * 1000 + 3
-    ws = torch.empty(gist.gist_ssdc_workspace_bytes(n), dtype=torch.uint8, device=cuda)
+    ws = gist.gist_ssdc_workspace(n, cuda)
     for seed in range(3):
         x = WL.relu_map((n,), 0.7, seed, cuda)
         row_end, col, val, nnz = gist.gist_ssdc_encode(x, workspace=ws, trim=True)
         r_row_end, r_col, _ = ref.ssdc_encode(host(x))
         assert_bits_equal(host(row_end), r_row_end, "row_end")
         assert_bits_equal(host(col), r_col, "col")
+
+
+def test_ssdc_workspace_reused_across_sizes(gist, ref, cuda):
+    """One workspace, initialised once, serves a sequence of calls of different sizes and
+    capacities (the epoch tag makes the previous call's tile totals read as unpublished)."""
+    big = 256 * 32 * 300 + 77
+    ws = gist.gist_ssdc_workspace(big, cuda)
+    for i, (n, cap) in enumerate([(big, None), (5000, None), (big, 0), (256 * 32 * 7, None), (big, None)] +
+                                 [(3000 + 97 * k, None) for k in range(40)] + [(big, None)]):
+        x = WL.relu_map((n,), 0.6 + 0.3 * (i % 2), 100 + i, cuda)
+        r_row_end, r_col, r_val = ref.ssdc_encode(host(x))
+        row_end, col, val, nnz = gist.gist_ssdc_encode(x, capacity=cap, workspace=ws)
+        assert int(nnz.item()) == r_col.size, (i, n)
+        assert_bits_equal(host(row_end), r_row_end, f"row_end call {i}")
+        if cap is None:
+            k = r_col.size
+            assert_bits_equal(host(col)[:k], r_col, f"col call {i}")
+            assert_bits_equal(host(val)[:k], r_val, f"val call {i}")
 
 
 # ------------------------------------------------------------------------ a6/a7 DPR
