@@ -20,6 +20,11 @@ cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, 
 cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uint32_t *mask, int32_t N, int32_t C,
                             int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo, float *dx,
                             cudaStream_t s);
+// 3x3 / stride 1 / pad <= 1 backward (pool_planes.cu): groups of whole planes staged by TMA
+bool pool_planes_ok(const gist_pool2d &p, int32_t H, int32_t W, int32_t Ho, int32_t Wo);
+cudaError_t launch_pool3s1_planes_bwd(const float *dout, const uint32_t *argmax, const uint32_t *mask, int32_t N,
+                                      int32_t C, int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo,
+                                      float *dx, cudaStream_t s);
 size_t ssdc_workspace_bytes(int64_t n);
 cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val,
                                int64_t capacity, int64_t *nnz, void *workspace, cudaStream_t s);

@@ -494,6 +494,9 @@ constexpr int kTileIn = 8192;   // staged floats per tile (32 KB)
 #ifndef GIST_POOL_K3S2_BLOCK
 #define GIST_POOL_K3S2_BLOCK 1
 #endif
+#ifndef GIST_POOL_PLANES
+#define GIST_POOL_PLANES 1
+#endif
 #ifndef GIST_POOL_FWD_TILED
 #define GIST_POOL_FWD_TILED 0
 #endif
@@ -951,6 +954,8 @@ cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uin
         const unsigned g2 = grid_for(ceil_div(a.n_out / 2, kPairU), kPoolThreads, 8);
         if (H == 2 * Ho) launch_k(pool_bwd_k2s2_pair_kernel<true>, g2, kPoolThreads, 0, s, dout, argmax, mask, a, dx);
         else launch_k(pool_bwd_k2s2_pair_kernel<false>, g2, kPoolThreads, 0, s, dout, argmax, mask, a, dx);
+    } else if (GIST_POOL_PLANES && pool_planes_ok(p, H, W, Ho, Wo)) {
+        return launch_pool3s1_planes_bwd(dout, argmax, mask, N, C, H, W, p, Ho, Wo, dx, s);
     } else if (is_k2s2_exact(p, H, W, Ho, Wo)) {
         launch_k(pool_bwd_k2s2_kernel, grid_for(ceil_div(a.n_out, kBwdU), kPoolThreads, 8), kPoolThreads, 0, s, dout, argmax, mask, a, dx);
     } else if (GIST_POOL_K3S2_BLOCK && p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2 && p.ph == 0 && p.pw == 0) {
