@@ -8,11 +8,13 @@ cap() {  # $1 name  $2 kernel regex  $3 rows  $4 skip
 }
 cap a1_binarize binarize_kernel a1 3
 cap a2_maxpool_fwd maxpool_fwd_k2s2_pair a2 3
+cap a2a1_maxpool_fwd_fused maxpool_fwd_k2s2_fused a2 3
 cap a3_pool_bwd pool_bwd_k2s2_pair a3 3
 cap a4_ssdc_encode ssdc_encode_kernel a4 7
 cap a5_ssdc_decode ssdc_decode_kernel a5 7
 cap a6_dpr_encode "dpr_encode_kernel" a6 3
 cap a7_dpr_decode "dpr_decode_kernel" a7 3
+timeout 300 ncu --set full --clock-control none --import-source on -k regex:pool3s1_planes_bwd -s 2 -c 1 -o $D/a3_pool3s1_planes_bwd python scripts/kernel_bench.py --small --only a3 --reps 2 > $D/a3_pool3s1.log 2>&1
 # the bench command: launch list (device time of every launch) and one full capture of the
 # dominant kernel on the step's largest SSDC site (relu1_1, the first ssdc launch of a step)
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $D/bench_launches.csv \
