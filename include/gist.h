@@ -83,8 +83,9 @@ int64_t gist_ssdc_bytes(int64_t n, int64_t nnz);
  * ticket, finished-CTA count, call epoch) plus one epoch-tagged 64-bit total per 32-row tile
  * (128 + 8*ceil(rows/32) bytes).  A workspace sized for n serves every n' <= n. */
 size_t gist_ssdc_workspace_bytes(int64_t n);
-/* Zero `bytes` of a workspace on `stream` (cudaMemsetAsync).  Required ONCE before the
- * workspace's first gist_ssdc_encode; every encode leaves it ready for the next one. */
+/* Initialise a workspace on `stream`: zero it and mark it initialised (one small kernel).
+ * Required ONCE before the workspace's first gist_ssdc_encode; every encode leaves it ready for
+ * the next one.  INVALID_ARGUMENT if bytes < gist_ssdc_workspace_bytes(1) (the counter line). */
 gist_status gist_ssdc_workspace_init(void *workspace, size_t bytes, cudaStream_t stream);
 /* ceil(n / k), k = 2, 3, 4 values per 32-bit word for bits = 16, 10, 8; -1 for
  * unsupported bits. */
@@ -145,7 +146,9 @@ gist_status gist_pool_relu_bwd(const float *dout, const uint32_t *argmax, const 
  *   workspace [>= gist_ssdc_workspace_bytes(n)] device bytes, zeroed once with
  *           gist_ssdc_workspace_init before its first use; each call leaves it reusable (the
  *           tile totals carry the call's epoch, so nothing is cleared per call).  One workspace
- *           must not serve two calls that may run concurrently (different streams).
+ *           must not serve two calls that may run concurrently (different streams).  A
+ *           workspace that was never initialised is detected on the device: the call then writes
+ *           *nnz = -1 and nothing else.
  * x is streamed from HBM once (tile counts), then re-read from L2 for the compaction; tile
  * offsets come from a running prefix over all tile totals kept by each CTA.  One kernel launch.
  * TOO_LARGE if n >= 2^31. */

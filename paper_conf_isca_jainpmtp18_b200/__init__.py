@@ -231,6 +231,8 @@ def gist_ssdc_encode(x: torch.Tensor, capacity: int | None = None, row_end=None,
            "gist_ssdc_encode")
     if trim:
         k = int(nnz.item())
+        if k < 0:
+            raise GistError(1, "gist_ssdc_encode: the workspace was not initialised (gist_ssdc_workspace_init)")
         if k > cap:
             raise GistError(4, f"gist_ssdc_encode: nnz {k} exceeds capacity {cap}")
         return row_end, col[:k], val[:k], nnz

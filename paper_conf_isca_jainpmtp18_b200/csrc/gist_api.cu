@@ -185,7 +185,8 @@ gist_status gist_ssdc_workspace_init(void *workspace, size_t bytes, cudaStream_t
     if (bytes == 0) return GIST_OK;
     if (!workspace) return GIST_ERR_INVALID_ARGUMENT;
     if (misaligned(workspace)) return GIST_ERR_MISALIGNED;
-    return cudaMemsetAsync(workspace, 0, bytes, stream) == cudaSuccess ? GIST_OK : GIST_ERR_CUDA;
+    if (bytes < gist_ssdc_workspace_bytes(1)) return GIST_ERR_INVALID_ARGUMENT;  // the counter line
+    return launched(gist::launch_ssdc_workspace_init(workspace, bytes, stream), 1);
 }
 
 gist_status gist_ssdc_decode(const int32_t *row_end, const uint8_t *col, const float *val, int64_t n, float *x,

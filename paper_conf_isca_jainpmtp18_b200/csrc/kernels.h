@@ -26,6 +26,7 @@ cudaError_t launch_pool3s1_planes_bwd(const float *dout, const uint32_t *argmax,
                                       int32_t C, int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo,
                                       float *dx, cudaStream_t s);
 size_t ssdc_workspace_bytes(int64_t n);
+cudaError_t launch_ssdc_workspace_init(void *workspace, size_t bytes, cudaStream_t s);
 cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val,
                                int64_t capacity, int64_t *nnz, void *workspace, cudaStream_t s);
 cudaError_t launch_ssdc_decode(const int32_t *row_end, const uint8_t *col, const float *val, int64_t n, float *x,

@@ -77,6 +77,13 @@ constexpr int kGatherPer = 8;                     // totals per lane per gather 
 // unpublished, so no per-call clearing is needed.  The last CTA to finish resets ticket and
 // done and advances the epoch.
 constexpr int kTotOffset = 32;                    // tot[] one 128-B line after the counters
+constexpr uint32_t kWsMagic = 0x47495354u;        // word 3 of an initialised workspace ("GIST")
+
+__global__ void ssdc_ws_init_kernel(uint32_t *ws, int64_t words) {
+    pdl_enter();
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += (int64_t)gridDim.x * blockDim.x)
+        ws[i] = i == 3 ? kWsMagic : 0u;
+}
 static_assert(kStages % kParts == 0, "each counter warp owns the stages of its part");
 static_assert(kPartRows % 2 == 0, "counters reduce two rows at a time");
 
@@ -241,6 +248,10 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
     EncSmem &S = *reinterpret_cast<EncSmem *>(smem_raw);
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
+    if (*reinterpret_cast<volatile uint32_t *>(ws + 3) != kWsMagic) {  // never initialised: report, no work
+        if (blockIdx.x == 0 && threadIdx.x == 0) *nnz_out = -1;
+        return;
+    }
     uint32_t *ticket = ws;
     uint64_t *tot = reinterpret_cast<uint64_t *>(ws + kTotOffset);
     // every CTA reads the epoch before it counts itself done, so all see the same value
@@ -513,6 +524,14 @@ size_t ssdc_workspace_bytes(int64_t n) {
     const int64_t rows = (n + kRow - 1) / kRow;
     const int64_t tiles = (rows + kTileRows - 1) / kTileRows;
     return 4 * (size_t)kTotOffset + 8 * (size_t)tiles;  // counters line + tot[tiles] uint64
+}
+
+cudaError_t launch_ssdc_workspace_init(void *workspace, size_t bytes, cudaStream_t s) {
+    const int64_t words = (int64_t)(bytes / 4);
+    int64_t blocks = ceil_div(words, 256);
+    if (blocks > 1024) blocks = 1024;
+    launch_k(ssdc_ws_init_kernel, (unsigned)blocks, 256, 0, s, reinterpret_cast<uint32_t *>(workspace), words);
+    return cudaPeekAtLastError();
 }
 
 cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val,

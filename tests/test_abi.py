@@ -113,6 +113,7 @@ def test_validation_without_gpu(gist):
     assert L.gist_ssdc_workspace_init(None, 0, None) == OK  # nothing to zero: no CUDA call
     assert L.gist_ssdc_workspace_init(None, 256, None) == INVALID
     assert L.gist_ssdc_workspace_init(B + 4, 256, None) == MISALIGNED
+    assert L.gist_ssdc_workspace_init(B, 64, None) == INVALID  # smaller than the counter line
     # f1: DPR over SSDC values (device count)
     assert L.gist_ssdc_dpr_encode(A, B, 0, 16, B + 64, None) == OK
     assert L.gist_ssdc_dpr_encode(A, B, 100, 12, B + 64, None) == UNSUPPORTED

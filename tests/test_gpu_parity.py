@@ -186,6 +186,19 @@ def test_ssdc_repeated_calls_reuse_workspace(gist, ref, cuda):
         assert_bits_equal(host(col), r_col, "col")
 
 
+def test_ssdc_uninitialised_workspace_is_reported(gist, cuda):
+    n = 256 * 32 * 20 + 5
+    x = WL.relu_map((n,), 0.7, 7, cuda)
+    ws = torch.full((gist.gist_ssdc_workspace_bytes(n),), 0xAB, dtype=torch.uint8, device=cuda)
+    row_end, col, val, nnz = gist.gist_ssdc_encode(x, workspace=ws)
+    assert int(nnz.item()) == -1
+    with pytest.raises(gist.GistError):
+        gist.gist_ssdc_encode(x, workspace=ws, trim=True)
+    gist.gist_ssdc_workspace_init(ws)
+    _, _, _, nnz = gist.gist_ssdc_encode(x, workspace=ws)
+    assert int(nnz.item()) == int((x.view(torch.int32) != 0).sum().item())
+
+
 def test_ssdc_workspace_reused_across_sizes(gist, ref, cuda):
     """One workspace, initialised once, serves a sequence of calls of different sizes and
     capacities (the epoch tag makes the previous call's tile totals read as unpublished)."""
