@@ -3,8 +3,8 @@
 // Encode: dense fp32 -> CSR with 256-column rows and uint8 column indices (Narrow Value
 // Optimization): row_end[rows] (inclusive ends, R10), col[nnz], val[nnz], nnz.
 //
-// Count, then compact from a second read served by L2; every CTA keeps its own running prefix
-// over ALL tile totals, so no tile waits on a serial look-back chain.
+// One read of x: count and compact from the same shared-memory ring; every CTA keeps its own
+// running prefix over ALL tile totals, so no tile waits on a serial look-back chain.
 //
 // Tiles are kTileRows = 32 rows (32 KB), claimed in ticket order by persistent CTAs (one per
 // SM).  The global offset of tile t is sum(tot[0..t)); a CTA's gatherer sums the published
@@ -13,20 +13,19 @@
 // predecessors' counts.  Warp roles per CTA, linked by mbarriers:
 //   * producer (1 lane): claims tiles (pre-claiming the next ticket) and streams each tile's
 //     four 8 KB parts into a kStages-deep shared-memory ring with 1-D TMA bulk copies
-//     (cp.async.bulk, HBM -> smem; the lines stay in L2 for the second read);
-//   * 4 counter warps (one per part): per-row nonzero bit-pattern counts (R8), stage released;
-//   * publisher warp: tile-local row scan -> rinc[], tile total published (flag | count in one
-//     word) to tot[tile];
+//     (cp.async.bulk, HBM -> smem);
+//   * 4 counter warps (one per part): per-row nonzero bit-pattern counts (R8);
+//   * publisher warp: tile-local row scan -> rinc[], tile total published (epoch tag | count
+//     in one word) to tot[tile];
 //   * gatherer warp: running prefix over tot[] -> the tile's global offset, and row_end;
-//   * 16 writer warps (2 rows each): re-read their rows with 128-bit loads (L2 hits; issued one
-//     tile ahead), rank nonzeros (lane l owns columns [8l, 8l+8); lane prefix from the ballots of
-//     the 4 bits of the lane counts), stage them in shared memory congruent to the output mod 16
-//     and store the whole 16-entry groups of val/col with two 1-D bulk copies (shared -> global).
-// A CTA holds at most kQ tiles between claim and write-out (bounded L2 footprint).  HBM sees
-// the algorithmic traffic: 4n read once, 5*nnz + 4*rows written (ncu: DRAM read = 4n).
-// The encode is issue-bound (~9k warp-instructions per 32 KB tile at ~80% issue utilisation);
+//   * 16 writer warps (2 rows each): once the tile is published, load their rows from the ring
+//     into registers (one tile ahead) and release the stage; rank nonzeros (lane l owns columns
+//     [8l, 8l+8); lane prefix: one shuffle scan of both rows' lane counts), stage them in
+//     shared memory congruent to the output mod 16, and store the whole 16-entry groups of
+//     val/col with two 1-D bulk copies (shared -> global) once the offset is resolved.
+// HBM sees the algorithmic traffic: 4n read once, 5*nnz + 4*rows written.
 // DESIGN.md §6 has the measured history of the alternatives (decoupled look-back, chunked
-// all-to-all prefix, single-pass compaction into a pending ring).
+// all-to-all prefix, single-pass compaction into a pending ring, L2 re-read writers).
 //
 // Decode: a warp expands 4 consecutive rows (whose entries are one contiguous range)
 //   through a 4 KB shared-memory row buffer and writes them back with float4 stores.
@@ -113,32 +112,6 @@ __device__ __forceinline__ void mbar_arrive1(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
-// Rows [rw, rw + kWRows) of tile t, rw = w * kWRows: lane l gets the 8
-// consecutive columns [8l, 8l+8) of each row (lo[r] = [8l, 8l+4), hi[r] = [8l+4, 8l+8)), so a
-// lane's nonzeros are contiguous in the output.  Last use of the data: L2 evict-first.
-// Elements past n read as zeros (never counted).
-__device__ __forceinline__ void load_rows(const float *__restrict__ x, int64_t n, int64_t t, int w, int lane,
-                                          uint4 (&lo)[kWRows], uint4 (&hi)[kWRows]) {
-#pragma unroll
-    for (int r = 0; r < kWRows; ++r) {
-        const int64_t e0 = (t * kTileRows + w * kWRows + r) * kRow;
-        const uint4 *p = reinterpret_cast<const uint4 *>(x + e0);
-        if (e0 + kRow <= n) {
-            lo[r] = __ldcs(p + 2 * lane);
-            hi[r] = __ldcs(p + 2 * lane + 1);
-        } else {
-            uint32_t v[8];
-#pragma unroll
-            for (int k = 0; k < 8; ++k) {
-                const int64_t e = e0 + 8 * lane + k;
-                v[k] = e < n ? __float_as_uint(x[e]) : 0u;
-            }
-            lo[r] = make_uint4(v[0], v[1], v[2], v[3]);
-            hi[r] = make_uint4(v[4], v[5], v[6], v[7]);
-        }
-    }
-}
-
 __device__ __forceinline__ uint32_t min1(uint32_t v) {  // 1 if the bit pattern is nonzero (one IMNMX)
     uint32_t r;
     asm("min.u32 %0, %1, 1;" : "=r"(r) : "r"(v));
@@ -148,16 +121,15 @@ __device__ __forceinline__ uint32_t nz4(const uint4 &a) {  // nonzero bit patter
     return min1(a.x) + min1(a.y) + min1(a.z) + min1(a.w);
 }
 
-// Writer: compact the rows held in lo/hi (queue slot q) to val/col.  Per row: lane count c
-// (0..8), exclusive lane prefix from the ballots of c's 4 bits, then the lane's nonzeros go to
-// consecutive staging slots (value word and column byte at the same index).  The staging is
-// congruent to the output mod 16 entries, so the whole 16-entry groups of val (64 B) and col (16 B) leave as two 1-D bulk copies
-// (cp.async.bulk shared -> global) issued by lane 0; the ragged head and tail (< 16 entries
-// each) by lanes 0..15 and 16..31.
+// Writer: compact the rows held in lo/hi (queue slot q) to val/col.  The lane counts (0..8) of
+// both rows are scanned together (two 16-bit fields, one 5-step shuffle scan); then each lane's
+// nonzeros go to consecutive staging slots (value word and column byte at the same index).
+// The staging is congruent to the output mod 16 entries, so the whole 16-entry groups of val
+// (64 B) and col (16 B) leave as two 1-D bulk copies (cp.async.bulk shared -> global) issued
+// by lane 0; the ragged head and tail (< 16 entries each) by lanes 0..15 and 16..31.
 __device__ __forceinline__ void write_rows(EncSmem &S, int q, int w, int lane, const uint4 (&lo)[kWRows],
                                            const uint4 (&hi)[kWRows], uint8_t *__restrict__ col,
                                            float *__restrict__ val, int64_t capacity) {
-    const uint32_t lt = (1u << lane) - 1u;
     const int rw = w * kWRows;
     const int64_t tile_base = S.base[q];
     const uint32_t w_excl = rw ? S.rinc[q][rw - 1] : 0u;
@@ -168,15 +140,22 @@ __device__ __forceinline__ void write_rows(EncSmem &S, int q, int w, int lane, c
     uint8_t *cs = S.cst[w];
     if (lane == 0) bulk_wait_read();  // the previous tile's bulk copies have read the staging
     __syncwarp();
-    uint32_t p = (uint32_t)(off & 15);
+    const uint32_t p = (uint32_t)(off & 15);
+    // lane prefix of both rows' lane counts in one warp scan (16-bit fields: row counts <= 256)
+    static_assert(kWRows == 2, "the packed scan carries two rows");
+    const uint32_t cnt0 = nz4(lo[0]) + nz4(hi[0]), cnt1 = nz4(lo[1]) + nz4(hi[1]);
+    uint32_t inc = cnt0 | (cnt1 << 16);
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t u = __shfl_up_sync(kFull, inc, d);
+        if (lane >= d) inc += u;
+    }
+    const uint32_t row0_tot = __shfl_sync(kFull, inc, 31) & 0xffffu;
+    const uint32_t excl[2] = {(inc & 0xffffu) - cnt0, row0_tot + (inc >> 16) - cnt1};
 #pragma unroll
     for (int r = 0; r < kWRows; ++r) {
         const uint32_t v[8] = {lo[r].x, lo[r].y, lo[r].z, lo[r].w, hi[r].x, hi[r].y, hi[r].z, hi[r].w};
-        const uint32_t c = nz4(lo[r]) + nz4(hi[r]);
-        const uint32_t b0 = __ballot_sync(kFull, c & 1u), b1 = __ballot_sync(kFull, c & 2u);
-        const uint32_t b2 = __ballot_sync(kFull, c & 4u), b3 = __ballot_sync(kFull, c & 8u);
-        const uint32_t i = p + __popc(b0 & lt) + 2 * __popc(b1 & lt) + 4 * __popc(b2 & lt) + 8 * __popc(b3 & lt);
-        p += __popc(b0) + 2 * __popc(b1) + 4 * __popc(b2) + 8 * __popc(b3);
+        const uint32_t i = p + excl[r];
         uint32_t addr = smem_u32(vs + i), caddr = smem_u32(cs + i);
         const uint32_t c0 = 8u * lane;
 #pragma unroll
@@ -260,7 +239,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
     if (threadIdx.x == 0) {
         for (int s = 0; s < kStages; ++s) {
             mbar_init(&S.full[s], 1);
-            mbar_init(&S.empty[s], 1);
+            mbar_init(&S.empty[s], kPartRows / kWRows);  // released by the part's writers
         }
         for (int q = 0; q < kQ; ++q) {
             mbar_init(&S.counted[q], kParts);
@@ -339,7 +318,6 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
             }
             __syncwarp();
             if (lane == 0) {
-                mbar_arrive1(&S.empty[s]);
                 mbar_arrive1(&S.counted[q]);
             }
             if (t >= tiles) break;
@@ -420,12 +398,29 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
         const int w = warp - kWriter0;
         uint4 lo[kDepth][kWRows], hi[kDepth][kWRows];
         int64_t tt[kDepth];
-        // the tile of local slot jj once published (its count is in rinc[]; its data in L2)
+        // the tile of local slot jj once published (its count is in rinc[]; its rows still in
+        // the ring); lane l gets the 8 consecutive columns [8l, 8l+8) of each of its rows, so a
+        // lane's nonzeros are contiguous in the output (elements past n were zero-filled)
         auto fetch = [&](int64_t jj, uint4 (&l)[kWRows], uint4 (&h)[kWRows]) -> int64_t {
             const int q = (int)(jj % kQ);
             mbar_wait_sleep(&S.published[q], (uint32_t)(jj / kQ) & 1u);
             const int64_t t = S.tile[q];
-            if (t < tiles) load_rows(x, n, t, w, lane, l, h);
+            // the tile is still in the TMA ring (the counters do not release it): read the rows
+            // from shared memory, then release the stage (the part's kPartRows / kWRows writers)
+            if (t < tiles) {
+                const int part = (w * kWRows) / kPartRows;
+                const int64_t js = kParts * jj + part;
+                const int st = (int)(js % kStages);
+                const float *rowp = S.raw[st] + (w * kWRows - part * kPartRows) * kRow;
+#pragma unroll
+                for (int r = 0; r < kWRows; ++r) {
+                    const uint4 *p4 = reinterpret_cast<const uint4 *>(rowp + r * kRow);
+                    l[r] = p4[2 * lane];
+                    h[r] = p4[2 * lane + 1];
+                }
+                __syncwarp();
+                if (lane == 0) mbar_arrive1(&S.empty[st]);
+            }
             return t;
         };
         auto retire = [&](int64_t jj, int64_t t, const uint4 (&l)[kWRows], const uint4 (&h)[kWRows]) {
