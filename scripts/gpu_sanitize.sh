@@ -1,3 +1,4 @@
+# Parity + compute-sanitizer (memcheck, racecheck, synccheck) over every kernel on small ragged shapes.
 mkdir -p gpurun_out
 timeout 900 python -m pytest tests -x -q -m "gpu and not slow" 2>&1 | tail -1
 for tool in memcheck racecheck synccheck; do
