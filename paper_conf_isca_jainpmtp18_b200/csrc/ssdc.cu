@@ -222,20 +222,18 @@ __global__ void __launch_bounds__(kEncThreads, 1)
 ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t tiles,
                     int32_t *__restrict__ row_end, uint8_t *__restrict__ col, float *__restrict__ val,
                     int64_t capacity, int64_t *__restrict__ nnz_out, uint32_t *__restrict__ ws) {
-    pdl_enter();
     extern __shared__ __align__(128) unsigned char smem_raw[];
     EncSmem &S = *reinterpret_cast<EncSmem *>(smem_raw);
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
-    if (*reinterpret_cast<volatile uint32_t *>(ws + 3) != kWsMagic) {  // never initialised: report, no work
-        if (blockIdx.x == 0 && threadIdx.x == 0) *nnz_out = -1;
-        return;
-    }
     uint32_t *ticket = ws;
     uint64_t *tot = reinterpret_cast<uint64_t *>(ws + kTotOffset);
-    // every CTA reads the epoch before it counts itself done, so all see the same value
-    const uint64_t tag = (uint64_t)(*reinterpret_cast<volatile uint32_t *>(ws + 2) + 1u) << 32;
-
+    // Prologue before the programmatic-dependency wait touches shared memory only (the barrier
+    // initialisation overlaps the previous kernel's tail); after it, the first ticket claim and
+    // the read of the counter line (epoch, magic) are issued together.
+#if GIST_PDL
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+#endif
     if (threadIdx.x == 0) {
         for (int s = 0; s < kStages; ++s) {
             mbar_init(&S.full[s], 1);
@@ -249,6 +247,20 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
         }
         fence_mbar_init();
     }
+#if GIST_PDL
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+#endif
+    // thread 0 is the producer lane: its first ticket is claimed now (on an uninitialised
+    // workspace the claim is harmless: the call reports and returns)
+    const uint32_t first_ticket = threadIdx.x == 0 ? atomicAdd(ticket, 1u) : 0u;
+    uint32_t epoch, magic;
+    asm volatile("ld.volatile.global.v2.u32 {%0, %1}, [%2];" : "=r"(epoch), "=r"(magic) : "l"(ws + 2) : "memory");
+    if (magic != kWsMagic) {  // never initialised: report, no work
+        if (blockIdx.x == 0 && threadIdx.x == 0) *nnz_out = -1;
+        return;
+    }
+    // every CTA reads the epoch before it counts itself done, so all see the same value
+    const uint64_t tag = (uint64_t)(epoch + 1u) << 32;
     __syncthreads();
 
     if (warp == kProd) {
@@ -262,7 +274,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                 g_trace[((int64_t)blockIdx.x * kTraceTiles + kTraceTiles - 1) * 4 + 3] = smid;
             }
 #endif
-            int64_t t = atomicAdd(ticket, 1u);
+            int64_t t = first_ticket;
             for (int64_t j = 0;; ++j) {
                 const int q = (int)(j % kQ);
                 if (j >= kQ) mbar_wait_sleep(&S.freed[q], (uint32_t)(j / kQ - 1) & 1u);
