@@ -102,6 +102,24 @@ def test_maxpool_fwd_and_fused_bwd(gist, ref, cuda, g, shape):
         assert_bits_equal(host(dx), r_dx, "dx" + (" (pool-only)" if m is None else ""))
 
 
+@pytest.mark.parametrize("shape", [(64, 192, 28, 28), (64, 480, 14, 14), (64, 832, 7, 7), (5, 37, 9, 11)],
+                         ids=lambda s: "x".join(map(str, s)))
+def test_pool3s1_full_googlenet_sizes(gist, ref, cuda, shape):
+    """GoogLeNet's in-module 3x3/s1/p1 pools at batch 64 (C4): the plane-group backward stages
+    many planes per group (odd plane sizes give every argmax-word and mask-word phase) and a
+    partial last group; pool-only and with a mask."""
+    g = (3, 3, 1, 1, 1, 1, 0)
+    y = pool_case(shape, g, 11, cuda)
+    out, arg, mask = gist.gist_maxpool_fwd_argmax(y, g, fuse_mask=True)
+    r_out, r_arg = ref.maxpool_fwd_argmax(host(y), g)
+    assert_bits_equal(host(arg), r_arg, "argmax")
+    dout = WL.grad_map(tuple(out.shape), 5, cuda)
+    for m, rm in ((None, None), (mask, ref.binarize_encode(host(y)))):
+        dx = gist.gist_pool_relu_bwd(dout, arg, m, shape, g)
+        r_dx = ref.pool_relu_bwd(host(dout), r_arg, rm, shape, g)
+        assert_bits_equal(host(dx), r_dx, "dx" + (" (pool-only)" if m is None else ""))
+
+
 def test_fused_bwd_equals_torch_autograd_on_gpu_inputs(gist, cuda):
     # Same chain as the CPU pin, but on the GPU kernels: relu -> max_pool2d (AlexNet 3x3/s2).
     g = (3, 3, 2, 2, 0, 0, 0)
