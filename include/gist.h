@@ -116,6 +116,19 @@ gist_status gist_maxpool_fwd_argmax(const float *y, int32_t N, int32_t C, int32_
                                     const gist_pool2d *p, float *out, uint32_t *argmax,
                                     uint32_t *mask, cudaStream_t stream);
 
+/* ---------------------------------------------------------------- f3: in-place ReLU + a1 + a2
+ * P:139 (inplace ReLU: the ReLU output is never a separate buffer) with P:152-P:156: x is the
+ * PRE-activation map (the producing conv's output).  Writes exactly what
+ * gist_maxpool_fwd_argmax(relu(x), ..., mask) writes, with relu(v) = (v < 0 ? +0.0f : v)
+ * (R21: torch's ReLU; -0.0 and NaN pass through), reading x once: out = the window max of
+ * relu(x), argmax = its 4-bit in-window index, mask bit i = (x[i] > 0) (= relu(x)[i] > 0).
+ * mask is required.  One kernel for 2x2/s2 with even H and W (VGG16, OverFeat); other
+ * geometries run the forward with relu on load plus a binarize pass over x.  Errors as
+ * gist_maxpool_fwd_argmax; mask == NULL -> INVALID_ARGUMENT. */
+gist_status gist_relu_maxpool_fwd_argmax(const float *x, int32_t N, int32_t C, int32_t H, int32_t W,
+                                         const gist_pool2d *p, float *out, uint32_t *argmax, uint32_t *mask,
+                                         cudaStream_t stream);
+
 /* ---------------------------------------------------------------- a3: fused pool+ReLU bwd
  * P:74 (ReLU bwd: dX = dY where Y > 0, else 0; MaxPool bwd routes dY to the argmax
  * location), P:156 ("Pool and ReLU backward pass ... perform computation on the encoded

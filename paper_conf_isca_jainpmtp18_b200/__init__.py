@@ -21,7 +21,7 @@ __all__ = [
     "GistError", "Pool2d", "lib", "library_path",
     "gist_binarize_words", "gist_argmax_words", "gist_pool2d_out_dims", "gist_ssdc_rows",
     "gist_ssdc_bytes", "gist_ssdc_workspace_bytes", "gist_ssdc_workspace", "gist_ssdc_workspace_init", "gist_dpr_words", "gist_num_sms", "gist_launch_count",
-    "gist_binarize_encode", "gist_maxpool_fwd_argmax", "gist_pool_relu_bwd",
+    "gist_binarize_encode", "gist_maxpool_fwd_argmax", "gist_relu_maxpool_fwd_argmax", "gist_pool_relu_bwd",
     "gist_ssdc_encode", "gist_ssdc_decode", "gist_dpr_encode", "gist_dpr_decode",
     "gist_ssdc_dpr_encode", "gist_ssdc_dpr_decode",
 ]
@@ -73,6 +73,7 @@ def _load() -> C.CDLL:
         "gist_binarize_encode": (C.c_int, [p, i64, p, p]),
         "gist_maxpool_fwd_argmax": (C.c_int, [p, i32, i32, i32, i32, P, p, p, p, p]),
         "gist_pool_relu_bwd": (C.c_int, [p, p, p, i32, i32, i32, i32, P, p, p]),
+        "gist_relu_maxpool_fwd_argmax": (C.c_int, [p, i32, i32, i32, i32, P, p, p, p, p]),
         "gist_ssdc_encode": (C.c_int, [p, i64, p, p, p, i64, p, p, sz, p]),
         "gist_ssdc_decode": (C.c_int, [p, p, p, i64, p, p]),
         "gist_dpr_encode": (C.c_int, [p, i64, i32, p, p]),
@@ -193,6 +194,22 @@ def gist_maxpool_fwd_argmax(y: torch.Tensor, pool, out=None, argmax=None, mask=N
         mask = _words(gist_binarize_words(y.numel()), y.device)
     _check(lib.gist_maxpool_fwd_argmax(_ptr(y), N, Cc, H, W, C.byref(g), _ptr(out), _ptr(argmax), _ptr(mask),
                                        _stream(y, stream)), "gist_maxpool_fwd_argmax")
+    return out, argmax, mask
+
+
+def gist_relu_maxpool_fwd_argmax(x: torch.Tensor, pool, out=None, argmax=None, mask=None, stream=None):
+    """f3 (P:139, P:152-P:156): ReLU applied on load to the pre-activation map x, then a2 + a1:
+    returns (out, argmax words, mask) equal to gist_maxpool_fwd_argmax(relu(x), pool, fuse_mask=True);
+    the ReLU output is never materialised."""
+    N, Cc, H, W = x.shape
+    g = Pool2d.of(pool)
+    Ho, Wo = gist_pool2d_out_dims(H, W, g)
+    if out is None:
+        out = torch.empty((N, Cc, Ho, Wo), dtype=torch.float32, device=x.device)
+    argmax = _words(gist_argmax_words(N * Cc * Ho * Wo), x.device, argmax)
+    mask = _words(gist_binarize_words(x.numel()), x.device, mask)
+    _check(lib.gist_relu_maxpool_fwd_argmax(_ptr(x), N, Cc, H, W, C.byref(g), _ptr(out), _ptr(argmax), _ptr(mask),
+                                            _stream(x, stream)), "gist_relu_maxpool_fwd_argmax")
     return out, argmax, mask
 
 

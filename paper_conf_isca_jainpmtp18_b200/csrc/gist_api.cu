@@ -144,6 +144,27 @@ gist_status gist_maxpool_fwd_argmax(const float *y, int32_t N, int32_t C, int32_
     return launched(e, separate ? 2 : 1);
 }
 
+gist_status gist_relu_maxpool_fwd_argmax(const float *x, int32_t N, int32_t C, int32_t H, int32_t W,
+                                         const gist_pool2d *p, float *out, uint32_t *argmax, uint32_t *mask,
+                                         cudaStream_t stream) {
+    int32_t Ho = 0, Wo = 0;
+    const gist_status st = check_pool(N, C, H, W, p, &Ho, &Wo);
+    if (st != GIST_OK) return st;
+    const int64_t n = (int64_t)N * C * H * W, n_out = (int64_t)N * C * Ho * Wo;
+    if (n == 0) return GIST_OK;
+    if (!x || !out || !argmax || !mask) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(x) || misaligned(out) || misaligned(argmax) || misaligned(mask)) return GIST_ERR_MISALIGNED;
+    if (n >= kI32Limit || n_out >= kI32Limit) return GIST_ERR_TOO_LARGE;
+    if (any_overlap({{x, 4 * n}},
+                    {{out, 4 * n_out}, {argmax, 4 * gist_argmax_words(n_out)}, {mask, 4 * gist_binarize_words(n)}}))
+        return GIST_ERR_INVALID_ARGUMENT;
+    bool fused = false;
+    cudaError_t e = gist::launch_relu_maxpool_fwd(x, N, C, H, W, *p, Ho, Wo, out, argmax, mask, &fused, stream);
+    // relu(x) > 0 iff x > 0: the mask of the pre-activation map is the mask of the ReLU output
+    if (e == cudaSuccess && !fused) e = gist::launch_binarize(x, n, mask, stream);
+    return launched(e, fused ? 1 : 2);
+}
+
 gist_status gist_pool_relu_bwd(const float *dout, const uint32_t *argmax, const uint32_t *mask, int32_t N, int32_t C,
                                int32_t H, int32_t W, const gist_pool2d *p, float *dx, cudaStream_t stream) {
     int32_t Ho = 0, Wo = 0;

@@ -17,6 +17,10 @@ cudaError_t launch_binarize(const float *y, int64_t n, uint32_t *mask, cudaStrea
 cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p,
                                int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, cudaStream_t s,
                                uint32_t *mask = nullptr, bool *mask_fused = nullptr);
+// f3: relu(x) on load (in-place ReLU); *mask_fused = false -> the caller adds binarize(x)
+cudaError_t launch_relu_maxpool_fwd(const float *x, int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p,
+                                    int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, uint32_t *mask, bool *mask_fused,
+                                    cudaStream_t s);
 cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uint32_t *mask, int32_t N, int32_t C,
                             int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo, float *dx,
                             cudaStream_t s);

@@ -40,8 +40,16 @@ __device__ __forceinline__ void take(float v, int idx, float &best, int &bi) {
     }
 }
 
-// KH/KW > 0: compile-time window; 0: runtime (a.kh, a.kw).
-template <int KH, int KW>
+// f3 in-place ReLU: the pre-activation map x is read and relu(v) = (v < 0 ? +0.0 : v)
+// (R21: torch's ReLU — -0.0 and NaN pass through) is applied on load, so the ReLU output never
+// exists in HBM.  relu(v) > 0 iff v > 0, so the a1 mask is the same either way.
+template <bool RELU>
+__device__ __forceinline__ float act(float v) {
+    return RELU ? (v < 0.0f ? 0.0f : v) : v;
+}
+
+// KH/KW > 0: compile-time window; 0: runtime (a.kh, a.kw).  RELU: relu(y) on load (f3).
+template <int KH, int KW, bool RELU = false>
 __global__ void __launch_bounds__(kPoolThreads)
 maxpool_fwd_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ out, uint32_t *__restrict__ arg) {
     pdl_enter();
@@ -72,7 +80,7 @@ maxpool_fwd_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ 
 #pragma unroll
                     for (int dy = 0; dy < (KH ? KH : 1); ++dy)
 #pragma unroll
-                        for (int dx = 0; dx < (KW ? KW : 1); ++dx) v[dy][dx] = ld_ro(plane + (h0 + dy) * a.W + w0 + dx);
+                        for (int dx = 0; dx < (KW ? KW : 1); ++dx) v[dy][dx] = act<RELU>(ld_ro(plane + (h0 + dy) * a.W + w0 + dx));
                     bi = 0;
                 } else {
 #pragma unroll
@@ -81,7 +89,7 @@ maxpool_fwd_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ 
                         for (int dx = 0; dx < (KW ? KW : 1); ++dx) {
                             const int ih = h0 + dy, iw = w0 + dx;
                             const bool in = ih >= 0 && ih < a.H && iw >= 0 && iw < a.W;
-                            v[dy][dx] = in ? ld_ro(plane + ih * a.W + iw) : -CUDART_INF_F;
+                            v[dy][dx] = in ? act<RELU>(ld_ro(plane + ih * a.W + iw)) : -CUDART_INF_F;
                         }
                     bi = max(0, -h0) * kw + max(0, -w0);
                 }
@@ -96,7 +104,7 @@ maxpool_fwd_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ 
                 for (int dx = 0; dx < kw; ++dx) {
                     const int iw = w0 + dx;
                     if (iw < 0 || iw >= a.W) continue;
-                    const float v = ld_ro(plane + ih * a.W + iw);
+                    const float v = act<RELU>(ld_ro(plane + ih * a.W + iw));
                     if (bi < 0) bi = dy * kw + dx;  // first in-bounds position (all -inf case)
                     take(v, dy * kw + dx, best, bi);
                 }
@@ -241,7 +249,7 @@ maxpool_fwd_k2s2_pair_kernel(const float *__restrict__ y, PoolArgs a, float *__r
 constexpr int kFusedUnitItems = 512;  // items per unit (upper bound; host picks BR)
 constexpr int kFusedU = 4;            // items per lane in flight
 
-template <int V>
+template <int V, bool RELU = false>
 __global__ void __launch_bounds__(kPoolThreads)
 maxpool_fwd_k2s2_fused_kernel(const float *__restrict__ y, PoolArgs a, int64_t blocks, int32_t BR, FastDiv div_ipr,
                               float *__restrict__ out, uint32_t *__restrict__ arg, uint32_t *__restrict__ mask) {
@@ -281,8 +289,9 @@ maxpool_fwd_k2s2_fused_kernel(const float *__restrict__ y, PoolArgs a, int64_t b
                     if constexpr (V == 4) {
                         float m0, m1;
                         uint32_t k0, k1;
-                        win4(t[k].x, t[k].y, bt[k].x, bt[k].y, m0, k0);
-                        win4(t[k].z, t[k].w, bt[k].z, bt[k].w, m1, k1);
+                        // mask bits below compare the raw values: relu(v) > 0 iff v > 0
+                        win4(act<RELU>(t[k].x), act<RELU>(t[k].y), act<RELU>(bt[k].x), act<RELU>(bt[k].y), m0, k0);
+                        win4(act<RELU>(t[k].z), act<RELU>(t[k].w), act<RELU>(bt[k].z), act<RELU>(bt[k].w), m1, k1);
                         reinterpret_cast<float2 *>(out + o0)[j] = make_float2(m0, m1);
                         part = (k0 | (k1 << 4)) << (8 * (lane & 3));
                         nt = (uint32_t)(t[k].x > 0.0f) | ((uint32_t)(t[k].y > 0.0f) << 1) |
@@ -292,7 +301,7 @@ maxpool_fwd_k2s2_fused_kernel(const float *__restrict__ y, PoolArgs a, int64_t b
                     } else {
                         float m;
                         uint32_t kk;
-                        win4(t[k].x, t[k].y, bt[k].x, bt[k].y, m, kk);
+                        win4(act<RELU>(t[k].x), act<RELU>(t[k].y), act<RELU>(bt[k].x), act<RELU>(bt[k].y), m, kk);
                         out[o0 + j] = m;
                         part = kk << (4 * (lane & 7));
                         nt = (uint32_t)(t[k].x > 0.0f) | ((uint32_t)(t[k].y > 0.0f) << 1);
@@ -898,6 +907,39 @@ unsigned grid_for(int64_t work_items, int64_t items_per_block, int per_sm) {
 }
 
 }  // namespace
+
+cudaError_t launch_relu_maxpool_fwd(const float *x, int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p,
+                                    int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, uint32_t *mask, bool *mask_fused,
+                                    cudaStream_t s) {
+    // f3: relu on load.  The fused 2x2/s2 kernel writes the mask in the same pass; other
+    // geometries use the L1 forward with relu on load and the caller adds binarize(x).
+    const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
+    *mask_fused = false;
+    if (is_k2s2_exact(p, H, W, Ho, Wo) && H == 2 * Ho) {
+        const int V = (W % 4 == 0) ? 4 : 2;
+        const int ipr = W / V;
+        int align = 16;
+        for (int g = W; g % 2 == 0 && align > 1; g /= 2) align /= 2;
+        const int64_t blocks = (int64_t)N * C * Ho;
+        const int64_t BR = align * std::max<int64_t>(1, 256 / ((int64_t)align * ipr));
+        if (BR * ipr <= kFusedUnitItems) {
+            const unsigned g = grid_for(ceil_div(blocks, BR), kPoolThreads / 32, 8);
+            const FastDiv d = FastDiv::make((uint32_t)ipr);
+            if (V == 4)
+                launch_k(maxpool_fwd_k2s2_fused_kernel<4, true>, g, kPoolThreads, 0, s, x, a, blocks, (int32_t)BR, d, out, argmax, mask);
+            else
+                launch_k(maxpool_fwd_k2s2_fused_kernel<2, true>, g, kPoolThreads, 0, s, x, a, blocks, (int32_t)BR, d, out, argmax, mask);
+            *mask_fused = true;
+            return cudaPeekAtLastError();
+        }
+    }
+    const unsigned grid = grid_for(a.n_out, kPoolThreads, 8);
+    if (p.kh == 3 && p.kw == 3)
+        launch_k(maxpool_fwd_kernel<3, 3, true>, grid, kPoolThreads, 0, s, x, a, out, argmax);
+    else
+        launch_k(maxpool_fwd_kernel<0, 0, true>, grid, kPoolThreads, 0, s, x, a, out, argmax);
+    return cudaPeekAtLastError();
+}
 
 cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p,
                                int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, cudaStream_t s, uint32_t *mask,

@@ -23,7 +23,7 @@ import contextlib
 import torch
 import torch.nn.functional as F
 
-from . import (gist_dpr_decode, gist_dpr_encode, gist_maxpool_fwd_argmax, gist_pool_relu_bwd,
+from . import (gist_dpr_decode, gist_dpr_encode, gist_relu_maxpool_fwd_argmax, gist_pool_relu_bwd,
                gist_ssdc_decode, gist_ssdc_encode, gist_ssdc_rows, gist_ssdc_workspace)
 
 
@@ -37,9 +37,9 @@ def _pool_tuple(kernel_size, stride, padding, ceil_mode):
 class _ReLUMaxPool(torch.autograd.Function):
     @staticmethod
     def forward(ctx, x, pool):
-        y = torch.relu(x)
-        out, arg, mask = gist_maxpool_fwd_argmax(y.contiguous(), pool, fuse_mask=True)
-        del y  # the fp32 ReLU output is not stashed
+        # in-place ReLU: relu is applied on load, the fp32 ReLU output never exists and
+        # is not stashed
+        out, arg, mask = gist_relu_maxpool_fwd_argmax(x.contiguous(), pool)
         ctx.save_for_backward(arg, mask)
         ctx.shape, ctx.pool = tuple(x.shape), pool
         return out

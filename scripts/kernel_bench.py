@@ -48,7 +48,7 @@ def timeit(fn, reps, warm=3):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--only", default=None, help="comma list of row ids: a1,a2,a3,a4,a5,a6,a7")
+    ap.add_argument("--only", default=None, help="comma list of row ids: a1,a2,a3,a4,a5,a6,a7,f3")
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--json", default=None)
     ap.add_argument("--small", action="store_true", help="secondary geometries too (3x3 pools)")
@@ -83,6 +83,12 @@ def main():
         lambda: gist.gist_maxpool_fwd_argmax(y, g, out=out, argmax=arg))
     rep("a2", "vgg16 relu1_2 b64 2x2/s2 +fused mask", 4 * n + 4 * n_o + 4 * words(n_o, 8) + 4 * words(n, 32),
         lambda: gist.gist_maxpool_fwd_argmax(y, g, out=out, argmax=arg, mask=mask))
+    xpre = WL.grad_map(shape, 4, dev)  # pre-activation map (the producing conv's output)
+    rep("f3", "vgg16 relu1_2 b64 2x2/s2 relu on load + mask (in-place ReLU)",
+        4 * n + 4 * n_o + 4 * words(n_o, 8) + 4 * words(n, 32),
+        lambda: gist.gist_relu_maxpool_fwd_argmax(xpre, g, out=out, argmax=arg, mask=mask))
+    del xpre
+    gist.gist_maxpool_fwd_argmax(y, g, out=out, argmax=arg)
     gist.gist_binarize_encode(y, mask=mask)
     dY = WL.grad_map(tuple(out.shape), 2, dev)
     dx = torch.empty_like(y)

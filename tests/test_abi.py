@@ -97,6 +97,9 @@ def test_validation_without_gpu(gist):
     assert L.gist_maxpool_fwd_argmax(A, 1, 1, 8, 8, C.byref(g), B, B + 4096, None, None) == UNSUPPORTED
     g = P(3, 3, 2, 2, 2, 2, 0)  # padding > k/2
     assert L.gist_maxpool_fwd_argmax(A, 1, 1, 8, 8, C.byref(g), B, B + 4096, None, None) == INVALID
+    g = P(2, 2, 2, 2, 0, 0, 0)
+    assert L.gist_relu_maxpool_fwd_argmax(A, 1, 1, 8, 8, C.byref(g), B, B + 4096, None, None) == INVALID  # f3 needs the mask
+    assert L.gist_relu_maxpool_fwd_argmax(A + 4, 1, 1, 8, 8, C.byref(g), B, B + 4096, B + 8192, None) == MISALIGNED
     g = P(3, 3, 0, 2, 0, 0, 0)  # zero stride
     assert L.gist_pool_relu_bwd(A, B, None, 1, 1, 8, 8, C.byref(g), B + 4096, None) == INVALID
     g = P(3, 3, 2, 2, 0, 0, 0)

@@ -120,6 +120,29 @@ def test_pool3s1_full_googlenet_sizes(gist, ref, cuda, shape):
         assert_bits_equal(host(dx), r_dx, "dx" + (" (pool-only)" if m is None else ""))
 
 
+@pytest.mark.parametrize("g", GEOMS, ids=gid)
+@pytest.mark.parametrize("shape", SHAPES + [(64, 64, 56, 56)], ids=lambda s: "x".join(map(str, s)))
+def test_relu_maxpool_fwd_in_place_relu(gist, ref, cuda, g, shape):
+    """f3: the pre-activation map goes in; out/argmax/mask equal the oracle's on
+    relu(x) (torch's ReLU, R21), and the fused-backward from them matches as well."""
+    N, Cc, H, W = shape
+    if H + 2 * g[4] < g[0] or W + 2 * g[5] < g[1]:
+        pytest.skip("window larger than padded input")
+    gen = torch.Generator(device=cuda).manual_seed(sum(shape) + 17)
+    x = torch.round(torch.randn(shape, device=cuda, generator=gen) * 2) / 2  # ties, negatives, zeros
+    r = torch.rand(shape, device=cuda, generator=gen)
+    x = torch.where(r < 0.01, torch.full_like(x, float("nan")), x)
+    x = torch.where((r >= 0.01) & (r < 0.02), torch.full_like(x, -float("inf")), x)
+    x = torch.where((r >= 0.02) & (r < 0.05), torch.full_like(x, -0.0), x)
+    x = torch.where((r >= 0.05) & (r < 0.06), torch.full_like(x, float("inf")), x)
+    y = torch.relu(x.cpu()).numpy()  # the definition of ReLU the path follows (R21)
+    out, arg, mask = gist.gist_relu_maxpool_fwd_argmax(x, g)
+    r_out, r_arg = ref.maxpool_fwd_argmax(y, g)
+    assert_bits_equal(host(out), r_out, "out")
+    assert_bits_equal(host(arg), r_arg, "argmax")
+    assert_bits_equal(host(mask), ref.binarize_encode(y), "mask")
+
+
 def test_fused_bwd_equals_torch_autograd_on_gpu_inputs(gist, cuda):
     # Same chain as the CPU pin, but on the GPU kernels: relu -> max_pool2d (AlexNet 3x3/s2).
     g = (3, 3, 2, 2, 0, 0, 0)

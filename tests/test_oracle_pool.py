@@ -175,3 +175,14 @@ def test_relu_pool_ratio_close_to_16x(ref):
     assert 4 * n / (4 * ref.binarize_words(n) + 4 * ref.argmax_words(n_o)) == pytest.approx(
         32 / (1 + 4 * n_o / n), rel=1e-4)
     assert (4 * n_o) / (4 * ref.argmax_words(n_o)) == pytest.approx(8.0, rel=1e-4)
+
+
+def test_relu_reading_r21_matches_torch():
+    """R21: the in-place ReLU of f3 is relu(v) = (v < 0 ? +0.0 : v) — torch's ReLU bit for bit
+    (-0.0 and NaN payloads pass through, -inf -> +0.0)."""
+    import numpy as np
+    v = np.array([-0.0, 0.0, -1.5, 2.5, np.inf, -np.inf, np.nan, 1e-45, -1e-45,
+                  np.frombuffer(np.uint32(0xFFC00001).tobytes(), np.float32)[0]], dtype=np.float32)
+    ours = np.where(v < 0, np.float32(0.0), v).astype(np.float32)
+    theirs = torch.relu(torch.from_numpy(v)).numpy()
+    assert np.array_equal(ours.view(np.uint32), theirs.view(np.uint32))
