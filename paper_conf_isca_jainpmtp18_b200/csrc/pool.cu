@@ -495,20 +495,11 @@ pool_bwd_k2s2_kernel(const float *__restrict__ dout, const uint32_t *__restrict_
     }
 }
 
-// ---- Generic geometry (any window <= 16 positions, stride, padding, ceil mode): shared-memory
-// tiles.  A tile is a band of output rows of one plane ("band") or several whole planes
-// ("multi"); its input rows are one contiguous range of the NCHW map, staged once with
-// coalesced float4 loads, so every window is read from shared memory.
+// ---- Generic-geometry backward (any window <= 16 positions, stride, padding, ceil mode):
+// shared-memory tiles.  A tile is a band of output rows of one plane ("band") or several whole
+// planes ("multi"); its dY rows are one contiguous range, staged once with coalesced float4
+// loads, so every covering window is read from shared memory.
 constexpr int kTileIn = 8192;   // staged floats per tile (32 KB)
-#ifndef GIST_POOL_K3S2_BLOCK
-#define GIST_POOL_K3S2_BLOCK 1
-#endif
-#ifndef GIST_POOL_PLANES
-#define GIST_POOL_PLANES 1
-#endif
-#ifndef GIST_POOL_FWD_TILED
-#define GIST_POOL_FWD_TILED 0
-#endif
 constexpr int kTileThreads = 256;
 
 struct TileSpec {
@@ -543,28 +534,6 @@ __device__ __forceinline__ TileRange tile_range(const TileSpec &T, const PoolArg
     return r;
 }
 
-// Argmax of output o straight from global memory (boundary words only).
-__device__ int window_argmax_global(const float *__restrict__ y, const PoolArgs &a, int64_t o) {
-    uint32_t q, ow, nc, oh;
-    a.div_wo.divmod((uint32_t)o, q, ow);
-    a.div_ho.divmod(q, nc, oh);
-    const int h0 = (int)oh * a.sh - a.ph, w0 = (int)ow * a.sw - a.pw;
-    const float *plane = y + (int64_t)nc * a.H * a.W;
-    float best = -CUDART_INF_F;
-    int bi = -1;
-    for (int dy = 0; dy < a.kh; ++dy) {
-        const int ih = h0 + dy;
-        if (ih < 0 || ih >= a.H) continue;
-        for (int dx = 0; dx < a.kw; ++dx) {
-            const int iw = w0 + dx;
-            if (iw < 0 || iw >= a.W) continue;
-            if (bi < 0) bi = dy * a.kw + dx;
-            take(ld_ro(plane + ih * a.W + iw), dy * a.kw + dx, best, bi);
-        }
-    }
-    return bi;
-}
-
 // Stage global floats [g_lo, g_hi) into smem: s[g - base], base = g_lo & ~3 (16-B phase kept).
 __device__ __forceinline__ int64_t stage_range(float *s, const float *__restrict__ g, int64_t g_lo, int64_t g_hi,
                                                int64_t n_total) {
@@ -579,75 +548,6 @@ __device__ __forceinline__ int64_t stage_range(float *s, const float *__restrict
         }
     }
     return base;
-}
-
-template <int KH, int KW>
-__global__ void __launch_bounds__(kTileThreads)
-maxpool_fwd_tiled_kernel(const float *__restrict__ y, PoolArgs a, TileSpec T, float *__restrict__ out,
-                         uint32_t *__restrict__ arg) {
-    pdl_enter();
-    __shared__ __align__(16) float s_in[kTileIn + 8];
-    __shared__ uint8_t s_nib[kTileIn];
-    const int kh = KH ? KH : a.kh, kw = KW ? KW : a.kw;
-    const int64_t HW = (int64_t)a.H * a.W, HoWo = (int64_t)a.Ho * a.Wo;
-    for (int64_t tile = blockIdx.x; tile < T.tiles; tile += gridDim.x) {
-        const TileRange r = tile_range(T, a, tile);
-        const int ih_lo = T.multi ? 0 : max(0, r.oh0 * a.sh - a.ph);
-        const int ih_hi = T.multi ? a.H : min(a.H, (r.oh1 - 1) * a.sh - a.ph + kh);
-        const int64_t g_lo = r.p0 * HW + (int64_t)ih_lo * a.W;
-        const int64_t g_hi = (r.p0 + r.np - 1) * HW + (int64_t)ih_hi * a.W;
-        const int64_t base = stage_range(s_in, y, g_lo, g_hi, a.n_in);
-        const int64_t o_lo = r.p0 * HoWo + (int64_t)r.oh0 * a.Wo;
-        const int64_t o_hi = (r.p0 + r.np - 1) * HoWo + (int64_t)r.oh1 * a.Wo;
-        __syncthreads();
-        for (int64_t o = o_lo + threadIdx.x; o < o_hi; o += blockDim.x) {
-            uint32_t q, ow, nc, oh;
-            a.div_wo.divmod((uint32_t)o, q, ow);
-            a.div_ho.divmod(q, nc, oh);
-            const int h0 = (int)oh * a.sh - a.ph, w0 = (int)ow * a.sw - a.pw;
-            const float *pl = s_in + ((int64_t)nc * HW - base);
-            float best = -CUDART_INF_F;
-            int bi = -1;
-            if (KH && KW && h0 >= 0 && w0 >= 0 && h0 + KH <= a.H && w0 + KW <= a.W) {  // interior window
-                const float *wp = pl + h0 * a.W + w0;
-                bi = 0;
-#pragma unroll
-                for (int dy = 0; dy < (KH ? KH : 1); ++dy)
-#pragma unroll
-                    for (int dx = 0; dx < (KW ? KW : 1); ++dx) take(wp[dy * a.W + dx], dy * kw + dx, best, bi);
-            } else
-#pragma unroll
-            for (int dy = 0; dy < (KH ? KH : 4); ++dy) {
-                if (!KH && dy >= kh) break;
-                const int ih = h0 + dy;
-                if (ih < 0 || ih >= a.H) continue;
-#pragma unroll
-                for (int dx = 0; dx < (KW ? KW : 4); ++dx) {
-                    if (!KW && dx >= kw) break;
-                    const int iw = w0 + dx;
-                    if (iw < 0 || iw >= a.W) continue;
-                    if (bi < 0) bi = dy * kw + dx;  // first in-bounds position
-                    take(pl[ih * a.W + iw], dy * kw + dx, best, bi);
-                }
-            }
-            out[o] = best;
-            s_nib[o - o_lo] = (uint8_t)bi;
-        }
-        __syncthreads();
-        // argmax words starting inside [o_lo, o_hi); nibbles past o_hi (next tile) from global
-        for (int64_t w = ((o_lo + 7) >> 3) + threadIdx.x; w < ((o_hi + 7) >> 3); w += blockDim.x) {
-            uint32_t word = 0;
-            for (int j = 0; j < 8; ++j) {
-                const int64_t o = 8 * w + j;
-                uint32_t nib = 0;
-                if (o < o_hi) nib = s_nib[o - o_lo];
-                else if (o < a.n_out) nib = (uint32_t)window_argmax_global(y, a, o);
-                word |= nib << (4 * j);
-            }
-            arg[w] = word;
-        }
-        __syncthreads();
-    }
 }
 
 template <int KH, int KW, int SH, int SW>
@@ -698,77 +598,6 @@ pool_bwd_tiled_kernel(const float *__restrict__ dout, const uint32_t *__restrict
                 }
             }
             dx[i] = acc;
-        }
-        __syncthreads();
-    }
-}
-
-// 3x3 stride 2, no padding (AlexNet, NiN, GoogLeNet stems; floor or ceil): one thread per 2x2
-// input block [2a, 2a+2) x [2b, 2b+2).  All four elements share the candidate windows
-// (oh, ow) in {a-1, a} x {b-1, b}; each window's nibble is decoded once and, visited in
-// ascending output order, routes +dY to the block element its argmax points at (R6).
-__global__ void __launch_bounds__(kTileThreads)
-pool_bwd_tiled_k3s2_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
-                           const uint32_t *__restrict__ mask, PoolArgs a, TileSpec T, FastDiv div_wb,
-                           FastDiv div_hb, float *__restrict__ dx) {
-    pdl_enter();
-    __shared__ __align__(16) float s_dy[kTileIn + 8];
-    __shared__ uint32_t s_arg[kTileIn / 8 + 2];
-    const int64_t HW = (int64_t)a.H * a.W, HoWo = (int64_t)a.Ho * a.Wo;
-    const int Wb = (a.W + 1) >> 1;
-    for (int64_t tile = blockIdx.x; tile < T.tiles; tile += gridDim.x) {
-        const TileRange r = tile_range(T, a, tile);
-        const int a_lo = T.multi ? 0 : r.oh0;                                      // block rows
-        const int a_hi = (T.multi || r.oh1 == a.Ho) ? (a.H + 1) >> 1 : r.oh1;
-        const int os_lo = T.multi ? 0 : max(0, r.oh0 - 1);
-        const int os_hi = T.multi ? a.Ho : min(a.Ho, a_hi);
-        const int64_t od_lo = r.p0 * HoWo + (int64_t)os_lo * a.Wo;
-        const int64_t od_hi = (r.p0 + r.np - 1) * HoWo + (int64_t)os_hi * a.Wo;
-        const int64_t dbase = stage_range(s_dy, dout, od_lo, od_hi, a.n_out);
-        const int64_t w_lo = od_lo >> 3;
-        for (int64_t w = w_lo + threadIdx.x; w < ((od_hi + 7) >> 3); w += blockDim.x) s_arg[w - w_lo] = ld_ro(arg + w);
-        __syncthreads();
-        const int64_t nblk = r.np * (int64_t)(a_hi - a_lo) * Wb;
-        for (int64_t t = threadIdx.x; t < nblk; t += blockDim.x) {
-            uint32_t q, b, pl, ar;
-            div_wb.divmod((uint32_t)t, q, b);
-            div_hb.divmod(q, pl, ar);  // div_hb divides by the tile's block-row count
-            const int A = a_lo + (int)ar;
-            const int64_t plane = r.p0 + pl;
-            const int64_t i00 = plane * HW + (int64_t)(2 * A) * a.W + 2 * (int)b;
-            float acc[2][2] = {{0.0f, 0.0f}, {0.0f, 0.0f}};
-#pragma unroll
-            for (int dwo = -1; dwo <= 0; ++dwo) {  // oh = A-1, A (ascending)
-                const int oh = A + dwo;
-                if (oh < 0 || oh >= a.Ho) continue;
-#pragma unroll
-                for (int dwc = -1; dwc <= 0; ++dwc) {  // ow = b-1, b (ascending)
-                    const int ow = (int)b + dwc;
-                    if (ow < 0 || ow >= a.Wo) continue;
-                    const int64_t o = plane * HoWo + (int64_t)oh * a.Wo + ow;
-                    const uint32_t nib = (s_arg[(o >> 3) - w_lo] >> (4 * (o & 7))) & 0xfu;
-                    const int ry = 2 * oh + (int)(nib / 3u) - 2 * A, rx = 2 * ow + (int)(nib % 3u) - 2 * (int)b;
-                    if (ry >= 0 && ry < 2 && rx >= 0 && rx < 2) {
-                        const float g = s_dy[o - dbase];
-                        if (ry == 0) {
-                            if (rx == 0) acc[0][0] = acc[0][0] + g; else acc[0][1] = acc[0][1] + g;
-                        } else {
-                            if (rx == 0) acc[1][0] = acc[1][0] + g; else acc[1][1] = acc[1][1] + g;
-                        }
-                    }
-                }
-            }
-#pragma unroll
-            for (int ry = 0; ry < 2; ++ry) {
-                if (2 * A + ry >= a.H) continue;
-#pragma unroll
-                for (int rx = 0; rx < 2; ++rx) {
-                    if (2 * (int)b + rx >= a.W) continue;
-                    const int64_t i = i00 + (int64_t)ry * a.W + rx;
-                    const bool on = mask == nullptr || ((ld_ro(mask + (i >> 5)) >> (i & 31)) & 1u);
-                    dx[i] = on ? acc[ry][rx] : 0.0f;
-                }
-            }
         }
         __syncthreads();
     }
@@ -972,16 +801,7 @@ cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, 
         else launch_k(maxpool_fwd_k2s2_pair_kernel<false>, g2, kPoolThreads, 0, s, y, a, out, argmax);
     } else if (is_k2s2_exact(p, H, W, Ho, Wo))
         launch_k(maxpool_fwd_k2s2_kernel, grid_for(ceil_div(a.n_out, kFwdU), kPoolThreads, 8), kPoolThreads, 0, s, y, a, out, argmax);
-    else if (GIST_POOL_FWD_TILED && tiled_ok(a)) {
-        const TileSpec T = make_tiles(a, N * C, false);
-        const unsigned gt = (unsigned)std::min<int64_t>(T.tiles, (int64_t)num_sms() * 6);
-        if (p.kh == 3 && p.kw == 3)
-            launch_k(maxpool_fwd_tiled_kernel<3, 3>, gt, kTileThreads, 0, s, y, a, T, out, argmax);
-        else if (p.kh == 2 && p.kw == 2)
-            launch_k(maxpool_fwd_tiled_kernel<2, 2>, gt, kTileThreads, 0, s, y, a, T, out, argmax);
-        else
-            launch_k(maxpool_fwd_tiled_kernel<0, 0>, gt, kTileThreads, 0, s, y, a, T, out, argmax);
-    } else if (p.kh == 3 && p.kw == 3)
+    else if (p.kh == 3 && p.kw == 3)
         launch_k(maxpool_fwd_kernel<3, 3>, grid, kPoolThreads, 0, s, y, a, out, argmax);
     else
         launch_k(maxpool_fwd_kernel<0, 0>, grid, kPoolThreads, 0, s, y, a, out, argmax);
@@ -996,11 +816,11 @@ cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uin
         const unsigned g2 = grid_for(ceil_div(a.n_out / 2, kPairU), kPoolThreads, 8);
         if (H == 2 * Ho) launch_k(pool_bwd_k2s2_pair_kernel<true>, g2, kPoolThreads, 0, s, dout, argmax, mask, a, dx);
         else launch_k(pool_bwd_k2s2_pair_kernel<false>, g2, kPoolThreads, 0, s, dout, argmax, mask, a, dx);
-    } else if (GIST_POOL_PLANES && pool_planes_ok(p, H, W, Ho, Wo)) {
+    } else if (pool_planes_ok(p, H, W, Ho, Wo)) {
         return launch_pool3s1_planes_bwd(dout, argmax, mask, N, C, H, W, p, Ho, Wo, dx, s);
     } else if (is_k2s2_exact(p, H, W, Ho, Wo)) {
         launch_k(pool_bwd_k2s2_kernel, grid_for(ceil_div(a.n_out, kBwdU), kPoolThreads, 8), kPoolThreads, 0, s, dout, argmax, mask, a, dx);
-    } else if (GIST_POOL_K3S2_BLOCK && p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2 && p.ph == 0 && p.pw == 0) {
+    } else if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2 && p.ph == 0 && p.pw == 0) {
         const int32_t hb = (H + 1) / 2, wb = (W + 1) / 2;
         const int64_t nblk = (int64_t)N * C * hb * wb;
         launch_k(pool_bwd_k3s2_block_kernel, grid_for(nblk, kPoolThreads, 8), kPoolThreads, 0, s, 
@@ -1008,13 +828,7 @@ cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uin
     } else if (tiled_ok(a)) {
         const TileSpec T = make_tiles(a, N * C, true);
         const unsigned gt = (unsigned)std::min<int64_t>(T.tiles, (int64_t)num_sms() * 6);
-        if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2 && p.ph == 0 && p.pw == 0) {
-            // block rows per tile: multi -> all (H+1)/2 of each plane; band -> TR (last band may be
-            // shorter: the kernel bounds t by its own count, the divisor only needs the stride)
-            const int32_t hb = T.multi ? (H + 1) / 2 : T.TR + 1;
-            launch_k(pool_bwd_tiled_k3s2_kernel, gt, kTileThreads, 0, s, dout, argmax, mask, a, T, FastDiv::make((W + 1) / 2),
-                                                                   FastDiv::make(hb), dx);
-        } else if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2)
+        if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2)
             launch_k(pool_bwd_tiled_kernel<3, 3, 2, 2>, gt, kTileThreads, 0, s, dout, argmax, mask, a, T, dx);
         else if (p.kh == 3 && p.kw == 3 && p.sh == 1 && p.sw == 1)
             launch_k(pool_bwd_tiled_kernel<3, 3, 1, 1>, gt, kTileThreads, 0, s, dout, argmax, mask, a, T, dx);
