@@ -240,6 +240,30 @@ def test_ssdc_uninitialised_workspace_is_reported(gist, cuda):
     assert int(nnz.item()) == int((x.view(torch.int32) != 0).sum().item())
 
 
+def test_ssdc_concurrent_streams_distinct_workspaces(gist, ref, cuda):
+    """Calls on different streams with distinct workspaces may overlap on the device (the
+    library is stateless apart from the workspace)."""
+    sizes = [256 * 32 * 900 + 13, 256 * 32 * 500 + 7, 256 * 32 * 60 + 1]
+    xs = [WL.relu_map((n,), 0.75, 300 + i, cuda) for i, n in enumerate(sizes)]
+    streams = [torch.cuda.Stream(cuda) for _ in sizes]
+    wss = [gist.gist_ssdc_workspace(n, cuda) for n in sizes]
+    torch.cuda.synchronize()
+    outs = []
+    for _ in range(3):
+        for x, st, ws in zip(xs, streams, wss):
+            with torch.cuda.stream(st):
+                outs.append(gist.gist_ssdc_encode(x, workspace=ws, stream=st))
+    torch.cuda.synchronize()
+    for i, (row_end, col, val, nnz) in enumerate(outs):
+        x = xs[i % len(xs)]
+        r_row_end, r_col, r_val = ref.ssdc_encode(host(x))
+        k = r_col.size
+        assert int(nnz.item()) == k
+        assert_bits_equal(host(row_end), r_row_end, f"row_end {i}")
+        assert_bits_equal(host(col)[:k], r_col, f"col {i}")
+        assert_bits_equal(host(val)[:k], r_val, f"val {i}")
+
+
 def test_ssdc_workspace_reused_across_sizes(gist, ref, cuda):
     """One workspace, initialised once, serves a sequence of calls of different sizes and
     capacities (the epoch tag makes the previous call's tile totals read as unpublished)."""
