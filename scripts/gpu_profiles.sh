@@ -10,6 +10,7 @@ cap a1_binarize binarize_kernel a1 3
 cap a2_maxpool_fwd maxpool_fwd_k2s2_pair a2 3
 cap a2a1_maxpool_fwd_fused maxpool_fwd_k2s2_fused a2 3
 cap a3_pool_bwd pool_bwd_k2s2_pair a3 3
+cap f3_relu_maxpool_fused fused_kernel f3 3  # --only f3: the only fused-kernel launches are <4, RELU>
 cap a4_ssdc_encode ssdc_encode_kernel a4 7
 cap a5_ssdc_decode ssdc_decode_kernel a5 7
 cap a6_dpr_encode "dpr_encode_kernel" a6 3
