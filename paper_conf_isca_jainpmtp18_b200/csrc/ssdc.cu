@@ -28,7 +28,9 @@
 // all-to-all prefix, single-pass compaction into a pending ring, L2 re-read writers).
 //
 // Decode: a warp expands 4 consecutive rows (whose entries are one contiguous range)
-//   through a 4 KB shared-memory row buffer and writes them back with float4 stores.
+//   through a 4 KB shared-memory row buffer and writes them back with float4 stores; the next
+//   group's row bounds are loaded one group ahead and up to 8 col/val entries per lane are in
+//   flight before the scatter.
 #include "common.cuh"
 #include "kernels.h"
 #include "tma.cuh"
@@ -49,6 +51,9 @@ constexpr int kRow = 256;
 #endif
 #ifndef GIST_SSDC_PARTS
 #define GIST_SSDC_PARTS 4
+#endif
+#ifndef GIST_SSDC_DEC_CTAS
+#define GIST_SSDC_DEC_CTAS 3  // decode CTAs per SM (grid cap); 4-6 measured slower in isolation
 #endif
 #ifndef GIST_SSDC_WROWS
 #define GIST_SSDC_WROWS 2
@@ -472,6 +477,10 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
 
 constexpr int kDecThreads = 256;
 constexpr int kDecRows = 4;  // rows per warp iteration
+#ifndef GIST_SSDC_DEC_BATCH
+#define GIST_SSDC_DEC_BATCH 8
+#endif
+constexpr int kDecBatch = GIST_SSDC_DEC_BATCH;  // col/val entries per lane in flight
 
 __global__ void __launch_bounds__(kDecThreads)
 ssdc_decode_kernel(const int32_t *__restrict__ row_end, const uint8_t *__restrict__ col,
@@ -485,25 +494,42 @@ ssdc_decode_kernel(const int32_t *__restrict__ row_end, const uint8_t *__restric
     const int64_t gwarp = ((int64_t)blockIdx.x * kDecThreads + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * kDecThreads) >> 5;
 
+    // lanes 0..4 hold the row boundaries of the warp's next group: bound[j] = end of row r0-1+j
+    // (loaded one group ahead, so only the col/val loads are on each group's critical path)
+    auto bounds = [&](int64_t g) -> int32_t {
+        const int64_t r = g * kDecRows - 1 + lane;
+        if (g >= groups || lane > kDecRows) return 0;
+        return (r < 0) ? 0 : (r < rows ? row_end[r] : row_end[rows - 1]);
+    };
+    int32_t bnd = bounds(gwarp);
     for (int64_t g = gwarp; g < groups; g += nwarps) {
         const int64_t r0 = g * kDecRows;
-        // lanes 0..4 fetch the row boundaries: bound[j] = end of row r0-1+j
-        int32_t bnd = 0;
-        if (lane <= kDecRows) {
-            const int64_t r = r0 - 1 + lane;
-            bnd = (r < 0) ? 0 : (r < rows ? row_end[r] : row_end[rows - 1]);
-        }
         const int32_t b0 = __shfl_sync(kFull, bnd, 0), b1 = __shfl_sync(kFull, bnd, 1);
         const int32_t b2 = __shfl_sync(kFull, bnd, 2), b3 = __shfl_sync(kFull, bnd, 3);
         const int32_t b4 = __shfl_sync(kFull, bnd, 4);
+        bnd = bounds(g + nwarps);
         // zero the 4-row buffer
         float4 *b4p = reinterpret_cast<float4 *>(buf);
 #pragma unroll
         for (int j = 0; j < kDecRows * kRow / 4 / 32; ++j) b4p[lane + 32 * j] = make_float4(0.f, 0.f, 0.f, 0.f);
         __syncwarp();
-        for (int32_t k = b0 + lane; k < b4; k += 32) {
-            const int rr = (k >= b1) + (k >= b2) + (k >= b3);
-            buf[rr * kRow + col[k]] = val[k];
+        // up to kDecBatch entries per lane in flight before any scatter
+        for (int32_t kb = b0; kb < b4; kb += 32 * kDecBatch) {
+            uint32_t c[kDecBatch];
+            float v[kDecBatch];
+#pragma unroll
+            for (int i = 0; i < kDecBatch; ++i) {
+                const int32_t k = kb + 32 * i + lane;
+                if (k < b4) {
+                    c[i] = col[k];
+                    v[i] = val[k];
+                }
+            }
+#pragma unroll
+            for (int i = 0; i < kDecBatch; ++i) {
+                const int32_t k = kb + 32 * i + lane;
+                if (k < b4) buf[((k >= b1) + (k >= b2) + (k >= b3)) * kRow + c[i]] = v[i];
+            }
         }
         __syncwarp();
         const int64_t base = r0 * kRow;
@@ -562,7 +588,7 @@ cudaError_t launch_ssdc_decode(const int32_t *row_end, const uint8_t *col, const
     const int64_t rows = (n + kRow - 1) / kRow;
     const int64_t groups = (rows + kDecRows - 1) / kDecRows;
     int64_t blocks = ceil_div(groups, kDecThreads / 32);
-    const int64_t cap = (int64_t)num_sms() * 6;
+    const int64_t cap = (int64_t)num_sms() * GIST_SSDC_DEC_CTAS;
     if (blocks > cap) blocks = cap;
     launch_k(ssdc_decode_kernel, (unsigned)blocks, kDecThreads, 0, s, row_end, col, val, n, rows, x);
     return cudaPeekAtLastError();

@@ -264,6 +264,21 @@ def test_ssdc_concurrent_streams_distinct_workspaces(gist, ref, cuda):
         assert_bits_equal(host(val)[:k], r_val, f"val {i}")
 
 
+def test_ssdc_back_to_back_chain_round_trips(gist, cuda):
+    """Encodes and decodes of many maps enqueued back to back with no host sync in between
+    (the programmatic-dependent-launch chain the bench runs): every map round-trips exactly."""
+    sizes = [64 * 512 * 14 * 14, 64 * 256 * 28 * 28, 256 * 33 + 5, 64 * 128 * 56 * 56 // 2, 64 * 512 * 7 * 7]
+    xs = [WL.relu_map((n,), 0.8, 900 + i, cuda) for i, n in enumerate(sizes)]
+    wss = [gist.gist_ssdc_workspace(n, cuda) for n in sizes]
+    torch.cuda.synchronize()
+    for _ in range(2):
+        encs = [gist.gist_ssdc_encode(x, workspace=ws) for x, ws in zip(xs, wss)]
+        outs = [gist.gist_ssdc_decode(e[0], e[1], e[2], x.numel()) for e, x in zip(reversed(encs), reversed(xs))]
+        torch.cuda.synchronize()
+        for x, y in zip(reversed(xs), outs):
+            assert torch.equal(x.view(torch.int32), y.view(torch.int32))
+
+
 def test_ssdc_workspace_reused_across_sizes(gist, ref, cuda):
     """One workspace, initialised once, serves a sequence of calls of different sizes and
     capacities (the epoch tag makes the previous call's tile totals read as unpublished)."""
