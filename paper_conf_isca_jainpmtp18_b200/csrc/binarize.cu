@@ -7,6 +7,10 @@
 #include "common.cuh"
 #include "kernels.h"
 
+#ifndef GIST_BIN_CTAS
+#define GIST_BIN_CTAS 8
+#endif
+
 namespace gist {
 
 namespace {
@@ -68,7 +72,7 @@ cudaError_t launch_binarize(const float *y, int64_t n, uint32_t *mask, cudaStrea
     const int64_t chunks = n / kChunk + 1;
     const int64_t per_block = kBinThreads / 32;
     int64_t blocks = ceil_div(chunks, per_block);
-    const int64_t cap = (int64_t)num_sms() * 8;  // 8 resident 256-thread CTAs per SM
+    const int64_t cap = (int64_t)num_sms() * GIST_BIN_CTAS;  // resident 256-thread CTAs per SM
     if (blocks > cap) blocks = cap;
     launch_k(binarize_kernel, (unsigned)blocks, kBinThreads, 0, stream, y, n, mask);
     return cudaPeekAtLastError();

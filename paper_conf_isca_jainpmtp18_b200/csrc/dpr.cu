@@ -239,13 +239,16 @@ dpr_decode_kernel(const uint32_t *__restrict__ packed, int64_t n, float *__restr
     }
 }
 
+#ifndef GIST_DPR_CTAS
+#define GIST_DPR_CTAS 8  // grid cap, CTAs per SM
+#endif
 template <int BITS>
 int64_t dpr_blocks(int64_t n) {
     constexpr int GF = (BITS == 10) ? 12 : 4;
     constexpr int U = (BITS == 10) ? kUnroll : kUnroll4;
     int64_t groups = n / GF + 1;
     int64_t blocks = ceil_div(ceil_div(groups, U), kDprThreads);
-    const int64_t cap = (int64_t)num_sms() * 8;
+    const int64_t cap = (int64_t)num_sms() * GIST_DPR_CTAS;
     return blocks > cap ? cap : blocks;
 }
 

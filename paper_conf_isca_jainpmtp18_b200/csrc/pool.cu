@@ -24,6 +24,12 @@ namespace gist {
 namespace {
 
 constexpr int kPoolThreads = 256;
+#ifndef GIST_POOL_FWD_CTAS
+#define GIST_POOL_FWD_CTAS 6  // grid cap, CTAs per SM (8, 7, 5, 4 measured slower on VGG16 maps)
+#endif
+#ifndef GIST_POOL_BWD_CTAS
+#define GIST_POOL_BWD_CTAS 6
+#endif
 
 struct PoolArgs {
     int32_t H, W, Ho, Wo;
@@ -752,7 +758,7 @@ cudaError_t launch_relu_maxpool_fwd(const float *x, int32_t N, int32_t C, int32_
         const int64_t blocks = (int64_t)N * C * Ho;
         const int64_t BR = align * std::max<int64_t>(1, 256 / ((int64_t)align * ipr));
         if (BR * ipr <= kFusedUnitItems) {
-            const unsigned g = grid_for(ceil_div(blocks, BR), kPoolThreads / 32, 8);
+            const unsigned g = grid_for(ceil_div(blocks, BR), kPoolThreads / 32, GIST_POOL_FWD_CTAS);
             const FastDiv d = FastDiv::make((uint32_t)ipr);
             if (V == 4)
                 launch_k(maxpool_fwd_k2s2_fused_kernel<4, true>, g, kPoolThreads, 0, s, x, a, blocks, (int32_t)BR, d, out, argmax, mask);
@@ -784,7 +790,7 @@ cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, 
         const int64_t blocks = (int64_t)N * C * Ho;
         int64_t BR = align * std::max<int64_t>(1, 256 / ((int64_t)align * ipr));
         if (BR * ipr <= kFusedUnitItems) {
-            const unsigned g = grid_for(ceil_div(blocks, BR), kPoolThreads / 32, 8);
+            const unsigned g = grid_for(ceil_div(blocks, BR), kPoolThreads / 32, GIST_POOL_FWD_CTAS);
             const FastDiv d = FastDiv::make((uint32_t)ipr);
             if (V == 4)
                 launch_k(maxpool_fwd_k2s2_fused_kernel<4>, g, kPoolThreads, 0, s, y, a, blocks, (int32_t)BR, d, out, argmax, mask);
@@ -813,13 +819,13 @@ cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uin
                             cudaStream_t s) {
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
     if (is_k2s2_exact(p, H, W, Ho, Wo) && W % 4 == 0) {
-        const unsigned g2 = grid_for(ceil_div(a.n_out / 2, kPairU), kPoolThreads, 8);
+        const unsigned g2 = grid_for(ceil_div(a.n_out / 2, kPairU), kPoolThreads, GIST_POOL_BWD_CTAS);
         if (H == 2 * Ho) launch_k(pool_bwd_k2s2_pair_kernel<true>, g2, kPoolThreads, 0, s, dout, argmax, mask, a, dx);
         else launch_k(pool_bwd_k2s2_pair_kernel<false>, g2, kPoolThreads, 0, s, dout, argmax, mask, a, dx);
     } else if (pool_planes_ok(p, H, W, Ho, Wo)) {
         return launch_pool3s1_planes_bwd(dout, argmax, mask, N, C, H, W, p, Ho, Wo, dx, s);
     } else if (is_k2s2_exact(p, H, W, Ho, Wo)) {
-        launch_k(pool_bwd_k2s2_kernel, grid_for(ceil_div(a.n_out, kBwdU), kPoolThreads, 8), kPoolThreads, 0, s, dout, argmax, mask, a, dx);
+        launch_k(pool_bwd_k2s2_kernel, grid_for(ceil_div(a.n_out, kBwdU), kPoolThreads, GIST_POOL_BWD_CTAS), kPoolThreads, 0, s, dout, argmax, mask, a, dx);
     } else if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2 && p.ph == 0 && p.pw == 0) {
         const int32_t hb = (H + 1) / 2, wb = (W + 1) / 2;
         const int64_t nblk = (int64_t)N * C * hb * wb;
