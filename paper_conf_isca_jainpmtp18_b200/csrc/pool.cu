@@ -27,6 +27,9 @@ constexpr int kPoolThreads = 256;
 #ifndef GIST_POOL_FWD_CTAS
 #define GIST_POOL_FWD_CTAS 6  // grid cap, CTAs per SM (8, 7, 5, 4 measured slower on VGG16 maps)
 #endif
+#ifndef GIST_POOL_GEN_CTAS
+#define GIST_POOL_GEN_CTAS 8  // generic-geometry kernels
+#endif
 #ifndef GIST_POOL_BWD_CTAS
 #define GIST_POOL_BWD_CTAS 6
 #endif
@@ -768,7 +771,7 @@ cudaError_t launch_relu_maxpool_fwd(const float *x, int32_t N, int32_t C, int32_
             return cudaPeekAtLastError();
         }
     }
-    const unsigned grid = grid_for(a.n_out, kPoolThreads, 8);
+    const unsigned grid = grid_for(a.n_out, kPoolThreads, GIST_POOL_GEN_CTAS);
     if (p.kh == 3 && p.kw == 3)
         launch_k(maxpool_fwd_kernel<3, 3, true>, grid, kPoolThreads, 0, s, x, a, out, argmax);
     else
@@ -800,7 +803,7 @@ cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, 
             return cudaPeekAtLastError();
         }
     }
-    const unsigned grid = grid_for(a.n_out, kPoolThreads, 8);
+    const unsigned grid = grid_for(a.n_out, kPoolThreads, GIST_POOL_GEN_CTAS);
     if (is_k2s2_exact(p, H, W, Ho, Wo) && W % 4 == 0) {
         const unsigned g2 = grid_for(ceil_div(a.n_out / 2, 32 * kPairU), kPoolThreads / 32, 8);
         if (H == 2 * Ho) launch_k(maxpool_fwd_k2s2_pair_kernel<true>, g2, kPoolThreads, 0, s, y, a, out, argmax);
@@ -829,7 +832,7 @@ cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uin
     } else if (p.kh == 3 && p.kw == 3 && p.sh == 2 && p.sw == 2 && p.ph == 0 && p.pw == 0) {
         const int32_t hb = (H + 1) / 2, wb = (W + 1) / 2;
         const int64_t nblk = (int64_t)N * C * hb * wb;
-        launch_k(pool_bwd_k3s2_block_kernel, grid_for(nblk, kPoolThreads, 8), kPoolThreads, 0, s, 
+        launch_k(pool_bwd_k3s2_block_kernel, grid_for(nblk, kPoolThreads, GIST_POOL_GEN_CTAS), kPoolThreads, 0, s, 
             dout, argmax, mask, a, FastDiv::make(wb), FastDiv::make(hb), nblk, dx);
     } else if (tiled_ok(a)) {
         const TileSpec T = make_tiles(a, N * C, true);
