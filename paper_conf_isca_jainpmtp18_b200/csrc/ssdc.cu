@@ -66,6 +66,7 @@ constexpr int kWriters = kTileRows / kWRows;
 #define GIST_SSDC_DEPTH 2
 #endif
 constexpr int kDepth = GIST_SSDC_DEPTH;                 // writer register sets (tiles in flight)
+static_assert(kDepth >= 2, "the writer loop prefetches at least one tile ahead");
 constexpr int kParts = GIST_SSDC_PARTS;               // counter warps = TMA stages per tile
 constexpr int kPartRows = kTileRows / kParts;
 constexpr int kPartElems = kPartRows * kRow;           // 8 KB per TMA stage (4 parts)
