@@ -162,7 +162,7 @@ gist_status gist_pool_relu_bwd(const float *dout, const uint32_t *argmax, const 
  *           must not serve two calls that may run concurrently (different streams).  A
  *           workspace that was never initialised is detected on the device: the call then writes
  *           *nnz = -1 and nothing else.
- * x is streamed from HBM once (tile counts), then re-read from L2 for the compaction; tile
+ * x is streamed from HBM once through a shared-memory ring (tile counts and compaction); tile
  * offsets come from a running prefix over all tile totals kept by each CTA.  One kernel launch.
  * TOO_LARGE if n >= 2^31. */
 gist_status gist_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val,
