@@ -234,8 +234,8 @@ dpr_decode_kernel(const uint32_t *__restrict__ packed, int64_t n, float *__restr
             for (int q = 0; q < 3; ++q) x4[c * 96 + 32 * q + lane] = b4[32 * q + lane];
             __syncwarp();
         }
-        if (tid == nthreads - 1)
-            for (int64_t i = chunks * 384; i < n; ++i) x[i] = value<10>((packed[i / 3] >> (10 * (i % 3))) & FIELD);
+        // the < 384 values past the last whole chunk: one per thread (not a serial loop)
+        for (int64_t i = chunks * 384 + tid; i < n; i += nthreads) x[i] = value<10>((packed[i / 3] >> (10 * (i % 3))) & FIELD);
     }
 }
 
@@ -244,10 +244,11 @@ dpr_decode_kernel(const uint32_t *__restrict__ packed, int64_t n, float *__restr
 #endif
 template <int BITS>
 int64_t dpr_blocks(int64_t n) {
+    // one group per thread until the grid cap is reached (the unrolled loops then take several
+    // per thread): small maps get every SM instead of 1/U of the threads
     constexpr int GF = (BITS == 10) ? 12 : 4;
-    constexpr int U = (BITS == 10) ? kUnroll : kUnroll4;
     int64_t groups = n / GF + 1;
-    int64_t blocks = ceil_div(ceil_div(groups, U), kDprThreads);
+    int64_t blocks = ceil_div(groups, kDprThreads);
     const int64_t cap = (int64_t)num_sms() * GIST_DPR_CTAS;
     return blocks > cap ? cap : blocks;
 }
