@@ -104,6 +104,8 @@ def main():
             oo, aa, _ = gist.gist_maxpool_fwd_argmax(yy, gg)
             nn, no = yy.numel(), oo.numel()
             rep("a2", name, 4 * nn + 4 * no + 4 * words(no, 8), lambda: gist.gist_maxpool_fwd_argmax(yy, gg, out=oo, argmax=aa))
+            rep("a2", name + " +mask", 4 * nn + 4 * no + 4 * words(no, 8) + 4 * words(nn, 32),
+                lambda: gist.gist_maxpool_fwd_argmax(yy, gg, out=oo, argmax=aa, mask=m2))
             dd = WL.grad_map(tuple(oo.shape), 4, dev)
             dxx = torch.empty_like(yy)
             rep("a3", name, 4 * no + 4 * words(no, 8) + 4 * words(nn, 32) + 4 * nn,

@@ -113,6 +113,7 @@ def test_pool3s1_full_googlenet_sizes(gist, ref, cuda, shape):
     out, arg, mask = gist.gist_maxpool_fwd_argmax(y, g, fuse_mask=True)
     r_out, r_arg = ref.maxpool_fwd_argmax(host(y), g)
     assert_bits_equal(host(arg), r_arg, "argmax")
+    assert_bits_equal(host(mask), ref.binarize_encode(host(y)), "fused mask")
     dout = WL.grad_map(tuple(out.shape), 5, cuda)
     for m, rm in ((None, None), (mask, ref.binarize_encode(host(y)))):
         dx = gist.gist_pool_relu_bwd(dout, arg, m, shape, g)
