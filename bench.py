@@ -71,9 +71,15 @@ def words(n, per):
 class Workload:
     """Device buffers of one rank's minibatch for every stash site, and the step."""
 
-    def __init__(self, gist, cfg: WL.Config, batch: int, sparsity: float, dpr_bits: int, rank: int, dev,
-                 fuse_mask: bool):
-        self.g, self.dev, self.bits, self.fuse = gist, dev, dpr_bits, fuse_mask
+    def __init__(self, gist, cfg: WL.Config, images, sparsity: float, dpr_bits: int, dev, fuse_mask: bool,
+                 many: bool = True):
+        """images: the GLOBAL image indices of this rank's minibatch shard (inputs are seeded per
+        image, so the shards of a strong-scaled batch add up to the single-GPU batch).
+        many: encode/decode all SSDC sites with one gist_ssdc_*_many launch and all DPR sites with
+        one gist_dpr_*_many launch per step; False: one C-ABI call per site."""
+        self.g, self.dev, self.bits, self.fuse, self.many = gist, dev, dpr_bits, fuse_mask, many
+        self.images = list(images)
+        batch = len(self.images)
         self.sites = []
         cidx = CONFIG_INDEX.get(cfg.key, 9)
         ssdc_sites = [s for s in WL.sites_for(cfg) if s.kind == "ssdc"]
@@ -84,18 +90,21 @@ class Workload:
             shape = (batch,) + s.chw
             n = s.numel(batch)
             max_n = max(max_n, n)
-            seed = WL.seed_for(cidx, si, rank)
+            seed0 = WL.image_seed(cidx, si, 0)
+            gseed0 = WL.image_seed(cidx, si, 0, grad=True)
             d = {"site": s, "shape": shape, "n": n}
             if s.kind in ("relu_pool", "pool_only"):
-                d["y"] = WL.relu_map(shape, 0.5, seed, dev)  # ReLU output feeding the pool
+                # ReLU output feeding the pool
+                d["y"] = WL.per_image(lambda sh, sd, dv: WL.relu_map(sh, 0.5, sd, dv), s.chw, self.images, seed0, dev)
                 oshape = (batch,) + pool_out(s.chw, s.pool)
                 d["n_out"] = oshape[0] * oshape[1] * oshape[2] * oshape[3]
                 d["out"] = torch.empty(oshape, device=dev)
                 d["arg"] = torch.empty(words(d["n_out"], 8), dtype=torch.int32, device=dev)
                 d["mask"] = torch.empty(words(n, 32), dtype=torch.int32, device=dev) if s.kind == "relu_pool" else None
-                d["dY"] = WL.grad_map(oshape, seed + 500, dev)
+                d["dY"] = WL.per_image(WL.grad_map, oshape[1:], self.images, gseed0, dev)
             elif s.kind == "ssdc":
-                d["y"] = WL.relu_map(shape, sparsity, seed, dev)
+                d["y"] = WL.per_image(lambda sh, sd, dv: WL.relu_map(sh, sparsity, sd, dv), s.chw, self.images, seed0,
+                                      dev)
                 rows = words(n, 256)
                 d["row_end"] = torch.empty(rows, dtype=torch.int32, device=dev)
                 d["col"] = torch.empty(n, dtype=torch.uint8, device=dev)
@@ -104,16 +113,37 @@ class Workload:
                 d["ws"] = gist.gist_ssdc_workspace(n, dev)
                 k_ssdc += 1
             else:
-                d["y"] = WL.dpr_map(shape, seed, dev)
+                d["y"] = WL.per_image(WL.dpr_map, s.chw, self.images, seed0, dev)
                 d["packed"] = torch.empty(gist.gist_dpr_words(n, dpr_bits), dtype=torch.int32, device=dev)
             self.sites.append(d)
         # decoded maps are short-lived (D lives only at its backward use): one scratch
         self.scratch = torch.empty(max_n, dtype=torch.float32, device=dev)
         self.stash_elems = sum(d["n"] for d in self.sites)
         self.bytes_per_step = 8 * self.stash_elems  # 4n encoded + 4n decoded per site
+        ss = [d for d in self.sites if d["site"].kind == "ssdc"]
+        ds = [d for d in self.sites if d["site"].kind == "dpr"]
+        self.ssdc_sites, self.dpr_sites = ss, ds
+        if many:
+            self.enc_many = gist.SsdcEncodeMany([{"x": d["y"], "row_end": d["row_end"], "col": d["col"], "val": d["val"],
+                                                  "nnz": d["nnz"], "capacity": d["n"]} for d in ss])
+            # decoded maps are short-lived: each site decodes into its own slice of one scratch
+            # buffer (the many-call needs distinct outputs)
+            tot = sum(d["n"] for d in ss) + sum(d["n"] for d in ds)
+            self.scratch_many = torch.empty(max(1, tot), dtype=torch.float32, device=dev)
+            o, views = 0, []
+            for d in ss + ds:
+                views.append(self.scratch_many[o:o + d["n"]])
+                o += d["n"]
+            self.dec_many = gist.SsdcDecodeMany([{"row_end": d["row_end"], "col": d["col"], "val": d["val"],
+                                                  "n": d["n"], "x": v} for d, v in zip(ss, views[:len(ss)])])
+            self.dpr_enc_many = gist.DprMany([{"x": d["y"], "packed": d["packed"]} for d in ds], dpr_bits, True)
+            self.dpr_dec_many = gist.DprMany([{"packed": d["packed"], "n": d["n"], "x": v}
+                                              for d, v in zip(ds, views[len(ss):])], dpr_bits, False)
 
     # ---- one pass: encode all sites (forward), decode all sites (backward)
     def step(self, timer=None):
+        if self.many:
+            return self.step_many(timer)
         g = self.g
         t = timer or (lambda kind, d: _Null())
         for d in self.sites:
@@ -151,11 +181,61 @@ class Workload:
                 with t("a7_dpr_decode", d):
                     g.gist_dpr_decode(d["packed"], n, self.bits, x=self.scratch[:n])
 
+    def step_many(self, timer=None):
+        """Forward: a2 (+a1) per ReLU->Pool site, then every SSDC site in one launch and every DPR
+        site in one launch; backward in reverse: DPR decodes, SSDC decodes, a3 per site."""
+        g = self.g
+        t = timer or (lambda kind, d: _Null())
+        for d in self.sites:
+            k = d["site"].kind
+            if k == "relu_pool":
+                with t("a2_maxpool_fwd_argmax+a1", d):
+                    g.gist_maxpool_fwd_argmax(d["y"], d["site"].pool, out=d["out"], argmax=d["arg"], mask=d["mask"])
+            elif k == "pool_only":
+                with t("a2_maxpool_fwd_argmax", d):
+                    g.gist_maxpool_fwd_argmax(d["y"], d["site"].pool, out=d["out"], argmax=d["arg"])
+        if self.ssdc_sites:
+            with t("a4_ssdc_encode", self.ssdc_sites):
+                self.enc_many()
+        if self.dpr_sites:
+            with t("a6_dpr_encode", self.dpr_sites):
+                self.dpr_enc_many()
+            with t("a7_dpr_decode", self.dpr_sites):
+                self.dpr_dec_many()
+        if self.ssdc_sites:
+            with t("a5_ssdc_decode", self.ssdc_sites):
+                self.dec_many()
+        for d in reversed(self.sites):
+            if d["site"].kind in ("relu_pool", "pool_only"):
+                dx = self.scratch[:d["n"]].view(d["shape"])
+                with t("a3_pool_relu_bwd", d):
+                    g.gist_pool_relu_bwd(d["dY"], d["arg"], d["mask"], d["shape"], d["site"].pool, dx=dx)
+
+    def encoded_views(self, nnz_list):
+        """Device views of every site's encoding (what Gist keeps through the forward->backward gap),
+        exact sizes: SSDC col/val trimmed to the site's nnz."""
+        out, k = [], 0
+        for d in self.sites:
+            kind = d["site"].kind
+            if kind in ("relu_pool", "pool_only"):
+                out.append(d["arg"])
+                if d["mask"] is not None:
+                    out.append(d["mask"])
+            elif kind == "ssdc":
+                m = int(nnz_list[k])
+                out += [d["row_end"], d["col"][:m], d["val"][:m]]
+                k += 1
+            else:
+                out.append(d["packed"])
+        return out
+
     def nnz_host(self):
         return self.nnz_all.cpu()
 
     # ---- algorithmic bytes of one launch (SURVEY.md §8(d)); nnz from the last step
     def algo_bytes(self, kind, d, nnz=None):
+        if isinstance(d, list):  # a many-map launch: the sum over its sites
+            return sum(self.algo_bytes(kind, e, nnz.get(id(e)) if isinstance(nnz, dict) else None) for e in d)
         n = d["n"]
         if kind == "a1_binarize_encode":
             return 4 * n + 4 * words(n, 32)
@@ -292,6 +372,20 @@ class ClockSampler:
 
 
 # --------------------------------------------------------------------------------- oracle legs
+def oracle_site(ref, d, bits):
+    """The oracle (as it stands) on one site of the sample: encode, then decode."""
+    s = d["site"]
+    if s.kind in ("relu_pool", "pool_only"):
+        mask = ref.binarize_encode(d["y"]) if s.kind == "relu_pool" else None
+        _, arg = ref.maxpool_fwd_argmax(d["y"], s.pool)
+        ref.pool_relu_bwd(d["dY"], arg, mask, d["y"].shape, s.pool)
+    elif s.kind == "ssdc":
+        enc = ref.ssdc_encode(d["y"])
+        ref.ssdc_decode(*enc, d["n"])
+    else:
+        ref.dpr_decode(ref.dpr_encode(d["y"], bits), d["n"], bits)
+
+
 def oracle_pass(ref, sites_host, bits):
     """The oracle (as it stands) over one sample: encode every site, then decode."""
     for d in sites_host:
@@ -331,55 +425,127 @@ def oracle_sample(cfg, images: int, sparsity: float, seed0: int):
     return sites
 
 
+def host_cpu():
+    """(usable cores, CPU model name) of this host."""
+    try:
+        cores = len(os.sched_getaffinity(0))
+    except AttributeError:
+        cores = os.cpu_count() or 1
+    model = "unknown"
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return cores, model
+
+
 def cpu_baseline(cfg, sparsity, bits, budget_s):
-    """Oracle timed on the host (1 thread) on a bounded sample: whole images of the same
-    workload, added until ~budget_s seconds of oracle work."""
+    """The oracle (as it stands, never tuned) timed on the host on a bounded sample of the same
+    workload: (i) single-threaded over whole images, (ii) on ALL host cores with
+    the independent units of the workload (one stash site of one image: encode + decode) spread
+    over a thread pool — the oracle's C functions run through ctypes, which releases the GIL, so
+    the threads run the unmodified oracle in parallel.  `value` is the all-cores figure."""
+    import concurrent.futures as cf
     import oracle as ref
     ref.lib()
+    cores, model = host_cpu()
+    # (i) one thread
     images, elapsed, nbytes = 0, 0.0, 0
-    while elapsed < budget_s and images < 64:
+    while elapsed < budget_s / 3 and images < 64:
         sample = oracle_sample(cfg, 1, sparsity, 777 + images)
         t0 = time.perf_counter()
         oracle_pass(ref, sample, bits)
         elapsed += time.perf_counter() - t0
         nbytes += 8 * sum(d["n"] for d in sample)
         images += 1
-    return {"value": round(nbytes / elapsed / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"{images} image(s) of the {cfg.key} workload (all stash sites, encode+decode), "
-                      f"{elapsed:.1f} s single-threaded"}
+    single = nbytes / elapsed / 1e9
+    # (ii) all cores: rounds of (cores x sites) units over 4 distinct images, until ~2/3 budget
+    pool_imgs = [oracle_sample(cfg, 1, sparsity, 4242 + k) for k in range(4)]
+    units = [d for img in pool_imgs for d in img]
+    unit_bytes = [8 * d["n"] for d in units]
+    per_round = max(1, -(-cores // len(units))) * len(units)  # every core busy, whole images
+    done_bytes, units_run, rounds = 0, 0, 0
+    with cf.ThreadPoolExecutor(max_workers=cores) as ex:
+        list(ex.map(lambda d: oracle_site(ref, d, bits), units[: min(len(units), cores)]))  # warm pages
+        t0 = time.perf_counter()
+        while True:
+            idx = [k % len(units) for k in range(per_round)]
+            list(ex.map(lambda k: oracle_site(ref, units[k], bits), idx))
+            done_bytes += sum(unit_bytes[k] for k in idx)
+            units_run += per_round
+            rounds += 1
+            if time.perf_counter() - t0 >= 2 * budget_s / 3 or rounds >= 50:
+                break
+        multi_s = time.perf_counter() - t0
+    multi = done_bytes / multi_s / 1e9
+    return {"value": round(multi, 4), "unit": "GB/s", "cores": cores, "kind": "oracle", "cpu_model": model,
+            "single_thread_GBps": round(single, 4),
+            "sample": f"{units_run} units (one stash site of one {cfg.key} image, encode+decode) on a {cores}-thread "
+                      f"pool over {multi_s:.1f} s; single-threaded: {images} whole image(s) in {elapsed:.1f} s"}
 
 
 def run_reference(args, cfg):
+    """The reference arm of this no-code tier: the CPU oracle, as it stands, on all host cores.
+    One step = one image's worth of units per usable core group: ceil(cores / sites) distinct
+    images, every (image, site) unit (encode + decode) run on a thread pool (ctypes releases the
+    GIL, so the unmodified oracle runs in parallel)."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return  # torchrun N>1: rank 0 alone runs the oracle arm
+    import concurrent.futures as cf
     import oracle as ref
     ref.lib()
-    images = 1
-    sample = oracle_sample(cfg, images, args.sparsity, 999)
-    for _ in range(args.warmup):
-        oracle_pass(ref, sample, args.dpr_bits)
-    t0 = time.perf_counter()
-    for _ in range(args.steps):
-        oracle_pass(ref, sample, args.dpr_bits)
-    dt = (time.perf_counter() - t0) / max(1, args.steps)
+    cores, model = host_cpu()
+    n_sites = len(WL.sites_for(cfg))
+    images = max(1, -(-cores // n_sites))
+    sample = oracle_sample(cfg, images, args.sparsity, 999)  # `images` images per site map
+    units = sample
     nbytes = 8 * sum(d["n"] for d in sample)
+    with cf.ThreadPoolExecutor(max_workers=cores) as ex:
+        def one_step():
+            # split each site's batch of `images` into per-image units
+            futs = []
+            for d in units:
+                per = d["n"] // images
+                for k in range(images):
+                    u = {"site": d["site"], "n": per, "y": d["y"][k:k + 1]}
+                    if "dY" in d:
+                        u["dY"] = d["dY"][k:k + 1]
+                    futs.append(ex.submit(oracle_site, ref, u, args.dpr_bits))
+            for f in futs:
+                f.result()
+        for _ in range(args.warmup):
+            one_step()
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            one_step()
+        dt = (time.perf_counter() - t0) / max(1, args.steps)
     value = nbytes / dt / 1e9
+    desc = (f"{images} image(s) of {cfg.key} per step, every (image, stash site) unit encoded+decoded by the "
+            f"oracle on a {cores}-thread pool")
     line = {
         "impl": "reference", "metric": baseline_metric(), "value": round(value, 4), "unit": "GB/s",
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": workload_config(args, cfg, images, note="bounded sample: 1 image per step"),
-        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-                         "sample": f"{images} image of {cfg.key} per step (all stash sites, encode+decode)"},
+        "config": workload_config(args, cfg, images, note="bounded sample: " + desc),
+        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": cores, "kind": "oracle",
+                         "cpu_model": model, "sample": desc},
         "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
 
 
-def workload_config(args, cfg, batch, note=None):
-    c = {"workload": f"{cfg.key}: {cfg.description}", "net": cfg.net, "batch_per_gpu": batch,
+def workload_config(args, cfg, batch, note=None, strong=False, world=1):
+    c = {"workload": f"{cfg.key}: {cfg.description}", "net": cfg.net,
+         **({"global_batch": batch, "batch_split": f"{batch} images over {world} rank(s) (shard_bounds)"} if strong
+            else {"batch_per_gpu": batch}),
          "ssdc_sparsity": args.sparsity, "dpr_bits": args.dpr_bits,
+         "calls": ("one gist_ssdc_*_many / gist_dpr_*_many launch per kind per step (P:171), a2/a3 per site"
+                   if getattr(args, "many", True) else "one C-ABI call per site"),
          "l2": "inputs larger than L2 (no flush needed)", "parallelism": f"dp{args.gpus} (minibatch shards, no "
          "collective on the hot path)"}
     if note:
@@ -398,10 +564,12 @@ def main():
     ap.add_argument("--batch", type=int, default=None, help="per-GPU batch (default: the config's)")
     ap.add_argument("--sparsity", type=float, default=None)
     ap.add_argument("--dpr-bits", type=int, default=None)
+    ap.add_argument("--per-site", dest="many", action="store_false",
+                    help="one C-ABI call per SSDC/DPR site instead of one gist_*_many launch per kind")
     ap.add_argument("--no-fuse-mask", dest="fuse_mask", action="store_false",
                     help="call a1 separately instead of passing the mask to the a2 call")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--cpu-seconds", type=float, default=8.0)
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--kernels-out", default=None, help="write the per-kernel breakdown JSON here")
     ap.add_argument("--same-device", action="store_true",
                     help="testing only: put every rank on cuda:0 and tally over gloo (exercises the N>1 "
@@ -418,6 +586,7 @@ def main():
         return
 
     import paper_conf_isca_jainpmtp18_b200 as gist
+    from paper_conf_isca_jainpmtp18_b200.shard import shard_bounds, tally
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -436,7 +605,14 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
 
-    wl = Workload(gist, cfg, batch, args.sparsity, args.dpr_bits, rank, dev, args.fuse_mask)
+    # C4 strong-scales one 64-image minibatch over the ranks; the other configs weak-scale (each rank
+    # its own per-GPU batch of distinct images).  SURVEY.md §8(e).
+    strong = cfg.key == "C4" and not args.batch
+    if strong:
+        lo, hi = shard_bounds(cfg.batch, world, rank)
+    else:
+        lo, hi = rank * batch, (rank + 1) * batch
+    wl = Workload(gist, cfg, range(lo, hi), args.sparsity, args.dpr_bits, dev, args.fuse_mask, args.many)
     stream = torch.cuda.current_stream(dev)
     for _ in range(args.warmup):
         wl.step()
@@ -479,7 +655,7 @@ def main():
         r = per.setdefault(kind, {"ms": 0.0, "launches": 0, "algo_bytes": 0})
         r["ms"] += s.elapsed_time(e)
         r["launches"] += 1
-        r["algo_bytes"] += wl.algo_bytes(kind, d, nnz_of.get(id(d)))
+        r["algo_bytes"] += wl.algo_bytes(kind, d, nnz_of if isinstance(d, list) else nnz_of.get(id(d)))
     peak, peak_src = hbm_peak()
     step_kernel_ms = sum(r["ms"] for r in per.values())
     kernels = {}
@@ -492,20 +668,22 @@ def main():
     dom_gbs = per[dom]["algo_bytes"] / (per[dom]["ms"] * 1e-3) / 1e9
 
     # ---- multi-rank: max time over ranks, sum of bytes (one collective, outside the timed region)
-    from paper_conf_isca_jainpmtp18_b200.shard import tally
     tdev = torch.device("cpu") if (dist is not None and args.same_device) else dev
     totals, elapsed_ms = tally(dist, {"fp32_bytes": wl.bytes_per_step * args.steps, "nnz": sum(nnz)}, elapsed_ms,
                                device=tdev)
     total_bytes = totals["fp32_bytes"]
     value = total_bytes / (elapsed_ms * 1e-3) / 1e9
 
-    # ---- e2e: host pinned inputs -> H2D -> the same C-ABI calls -> D2H of the nnz tally
+    # ---- e2e: host pinned inputs -> H2D -> the same C-ABI calls -> D2H of the step's results: the
+    # encoded stash of every site (exact bytes: the nnz of the deterministic inputs is known from the
+    # untimed steps) and the per-site nnz tally
     e2e = None
     if not args.no_e2e:
         hosts = [(d, d["y"].cpu().pin_memory(), d["dY"].cpu().pin_memory() if "dY" in d else None) for d in wl.sites]
         h2d = sum(h.numel() * 4 + (g.numel() * 4 if g is not None else 0) for _, h, g in hosts)
-        d2h = wl.nnz_all.numel() * 8
-        out_host = torch.empty_like(wl.nnz_all, device="cpu").pin_memory()
+        enc = wl.encoded_views(nnz) + [wl.nnz_all]
+        enc_host = [torch.empty(t.shape, dtype=t.dtype).pin_memory() for t in enc]
+        d2h = sum(t.numel() * t.element_size() for t in enc)
         e_steps = max(3, min(args.steps, 10))
 
         def e2e_step():
@@ -514,7 +692,8 @@ def main():
                 if g is not None:
                     d["dY"].copy_(g, non_blocking=True)
             wl.step()
-            out_host.copy_(wl.nnz_all, non_blocking=True)
+            for t, hbuf in zip(enc, enc_host):
+                hbuf.copy_(t, non_blocking=True)
 
         e2e_step()
         barrier()
@@ -529,8 +708,9 @@ def main():
         e_bytes = e_tot["fp32_bytes"]
         e2e = {"value": round(e_bytes / (e_ms * 1e-3) / 1e9, 3), "unit": "GB/s", "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "steps": e_steps,
-               "note": "pinned host maps copied H2D each step, then the step's C-ABI calls, then D2H of the "
-                       "per-site nnz tally"}
+               "note": "pinned host maps (and pool gradients) copied H2D each step, then the step's C-ABI calls, "
+                       "then D2H of every site's encoding (mask + argmax map, exact-size CSR, DPR words) and the "
+                       "per-site nnz tally; one stream, PCIe-bound"}
 
     if rank != 0:
         if dist is not None:
@@ -541,8 +721,9 @@ def main():
     line = {
         "metric": baseline_metric(), "value": round(value, 3), "unit": "GB/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(elapsed_ms / args.steps, 4),
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": workload_config(args, cfg, batch),
+        "higher_is_better": True, "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic",
+        "config": workload_config(args, cfg, batch if not strong else cfg.batch, strong=strong, world=world),
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": round(dom_gbs, 1), "peak": peak, "unit": "GB/s",
                      "frac": round(dom_gbs / peak, 4), "traffic": traffic_for(dom), "peak_source": peak_src},
         "cpu_baseline": cpu,

@@ -26,8 +26,10 @@
  *     next synchronization, as for any CUDA kernel.
  *   - Deterministic: all encodings are bit-identical run to run; padding bits, unused
  *     fields and tail fields are always written as 0, so whole buffers compare with
- *     memcmp.  The library is stateless apart from a cached SM count; concurrent calls
- *     on different streams are safe when they use distinct outputs and workspaces.
+ *     memcmp.  The library is stateless apart from per-device caches (SM count, the
+ *     dynamic shared-memory opt-in of two kernels) filled on first use on each device;
+ *     calls act on the CURRENT device (cudaSetDevice).  Concurrent calls on different
+ *     streams are safe when they use distinct outputs and workspaces.
  *   - Inputs and outputs must not overlap (GIST_ERR_INVALID_ARGUMENT).
  *
  * The readings of the paper taken wherever it is silent (bit orders, tie rules, rounding,
@@ -109,8 +111,10 @@ gist_status gist_binarize_encode(const float *y, int64_t n, uint32_t *mask, cuda
  *   out    [N,C,Ho,Wo] fp32, written (the pool output, still consumed in forward).
  *   argmax [gist_argmax_words(N*C*Ho*Wo)] uint32, written.
  *   mask   NULL, or [gist_binarize_words(N*C*H*W)] uint32: if non-NULL the a1 mask of y is
- *          written too — in the same pass (one read of y) for 2x2/s2 unpadded pools with
- *          W % 16 == 0 and H even, otherwise by a second kernel over y.
+ *          written too — in the same pass (one read of y) for 2x2/s2 unpadded pools with H and
+ *          W even whose warp unit of BR whole row pairs fits 512 items: BR*W/V <= 512 with
+ *          V = 4 if W % 4 == 0 else 2, a = 16/gcd(W,16), BR = a*max(1, floor(256/(a*W/V)))
+ *          (every VGG16 and OverFeat map); otherwise by a second kernel over y.
  * TOO_LARGE if N*C*H*W >= 2^31. */
 gist_status gist_maxpool_fwd_argmax(const float *y, int32_t N, int32_t C, int32_t H, int32_t W,
                                     const gist_pool2d *p, float *out, uint32_t *argmax,
@@ -203,6 +207,57 @@ gist_status gist_ssdc_dpr_encode(const float *val, const int64_t *nnz, int64_t c
                                  uint32_t *packed, cudaStream_t stream);
 gist_status gist_ssdc_dpr_decode(const uint32_t *packed, const int64_t *nnz, int64_t capacity, int32_t bits,
                                  float *val, cudaStream_t stream);
+
+/* ---------------------------------------------------------------- many maps per call
+ * P:171 ("these conversions can happen in parallel"): a network stashes many maps per minibatch;
+ * these calls encode/decode several maps in ONE persistent launch (per up to 48 SSDC / 64 SSDC-
+ * decode / 96 DPR maps), so the per-launch fill and drain is paid once instead of once per map.
+ * Each job's results are exactly those of the single-map call on the same arguments; every job is
+ * validated as the single-map call validates it (status of the first failing job, nothing
+ * launched).  Jobs must not overlap each other's outputs.  count == 0 returns GIST_OK.
+ *
+ * offset (append mode, f2): NULL, or a DEVICE int64 holding the position where this map's CSR
+ * entries start inside col/val (a stash arena shared by several maps).  Then entry k of the map is
+ * written at col[*offset + k] / val[*offset + k] (only where *offset + k < capacity), row_end holds
+ * ABSOLUTE inclusive ends (< 2^31), and *nnz receives the END offset *offset + count.  Decode jobs
+ * take the same offset so that row 0 starts at *offset.  With offset == NULL a job is the plain
+ * single-map encoding (*nnz = count).  Within one encode_many call a job's offset may be the nnz
+ * of the PREVIOUS job (both n > 0): its entries then follow that job's in the same arena, computed
+ * in the same launch (a chained stash arena: exact-size, no host synchronization).  Any other
+ * aliasing of an offset with a job's nnz is INVALID_ARGUMENT. */
+typedef struct {
+    const float *x;
+    int64_t n;
+    int32_t *row_end;
+    uint8_t *col;
+    float *val;
+    int64_t capacity;
+    int64_t *nnz;
+    const int64_t *offset;
+} gist_ssdc_job;
+
+typedef struct {
+    const int32_t *row_end;
+    const uint8_t *col;
+    const float *val;
+    const int64_t *offset;
+    int64_t n;
+    float *x;
+} gist_ssdc_decode_job;
+
+typedef struct {
+    const float *x;    /* encode: read; decode: written */
+    int64_t n;
+    uint32_t *packed;  /* encode: written; decode: read */
+} gist_dpr_job;
+
+/* Workspace bytes for gist_ssdc_encode_many over these jobs: 128 + 8 * sum of their 32-row tiles. */
+size_t gist_ssdc_workspace_bytes_many(const gist_ssdc_job *jobs, int32_t count);
+gist_status gist_ssdc_encode_many(const gist_ssdc_job *jobs, int32_t count, void *workspace,
+                                  size_t workspace_bytes, cudaStream_t stream);
+gist_status gist_ssdc_decode_many(const gist_ssdc_decode_job *jobs, int32_t count, cudaStream_t stream);
+gist_status gist_dpr_encode_many(const gist_dpr_job *jobs, int32_t count, int32_t bits, cudaStream_t stream);
+gist_status gist_dpr_decode_many(const gist_dpr_job *jobs, int32_t count, int32_t bits, cudaStream_t stream);
 
 /* Number of SMs the launch heuristics use (cached on first call; for diagnostics). */
 int32_t gist_num_sms(void);

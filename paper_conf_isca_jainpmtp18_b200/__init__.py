@@ -1,9 +1,9 @@
 """Python binding of libgist — Gist's stash-time encode/decode hot path on B200 (sm_100a).
 
-Argument marshalling only: every function below validates nothing itself, allocates
-outputs with torch on the input's device when the caller passes none, and forwards raw
-device pointers plus torch's current CUDA stream to the same-named C-ABI call in
-``include/gist.h`` (ctypes).  All arithmetic runs in the CUDA kernels of ``csrc/``.
+Argument marshalling only: every function below checks what the C ABI cannot see (a torch
+tensor's device, dtype, contiguity and element count), allocates outputs with torch on the
+input's device when the caller passes none, and forwards raw device pointers plus torch's
+current CUDA stream to the same-named C-ABI call in ``include/gist.h`` (ctypes).  All arithmetic runs in the CUDA kernels of ``csrc/``.
 There is no CPU fallback: importing this package without ``libgist.so`` raises, and a
 non-CUDA tensor is rejected.
 
@@ -24,6 +24,8 @@ __all__ = [
     "gist_binarize_encode", "gist_maxpool_fwd_argmax", "gist_relu_maxpool_fwd_argmax", "gist_pool_relu_bwd",
     "gist_ssdc_encode", "gist_ssdc_decode", "gist_dpr_encode", "gist_dpr_decode",
     "gist_ssdc_dpr_encode", "gist_ssdc_dpr_decode",
+    "gist_ssdc_workspace_bytes_many", "gist_ssdc_encode_many", "gist_ssdc_decode_many", "gist_dpr_encode_many",
+    "gist_dpr_decode_many", "SsdcEncodeMany", "SsdcDecodeMany", "DprMany",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -48,6 +50,23 @@ class Pool2d(C.Structure):
         if isinstance(g, Pool2d):
             return g
         return cls(*[int(v) for v in g])
+
+
+class SsdcJob(C.Structure):
+    """gist_ssdc_job (include/gist.h)."""
+    _fields_ = [("x", C.c_void_p), ("n", C.c_int64), ("row_end", C.c_void_p), ("col", C.c_void_p),
+                ("val", C.c_void_p), ("capacity", C.c_int64), ("nnz", C.c_void_p), ("offset", C.c_void_p)]
+
+
+class SsdcDecodeJob(C.Structure):
+    """gist_ssdc_decode_job (include/gist.h)."""
+    _fields_ = [("row_end", C.c_void_p), ("col", C.c_void_p), ("val", C.c_void_p), ("offset", C.c_void_p),
+                ("n", C.c_int64), ("x", C.c_void_p)]
+
+
+class DprJob(C.Structure):
+    """gist_dpr_job (include/gist.h)."""
+    _fields_ = [("x", C.c_void_p), ("n", C.c_int64), ("packed", C.c_void_p)]
 
 
 def _load() -> C.CDLL:
@@ -80,6 +99,11 @@ def _load() -> C.CDLL:
         "gist_dpr_decode": (C.c_int, [p, i64, i32, p, p]),
         "gist_ssdc_dpr_encode": (C.c_int, [p, p, i64, i32, p, p]),
         "gist_ssdc_dpr_decode": (C.c_int, [p, p, i64, i32, p, p]),
+        "gist_ssdc_workspace_bytes_many": (sz, [p, i32]),
+        "gist_ssdc_encode_many": (C.c_int, [p, i32, p, sz, p]),
+        "gist_ssdc_decode_many": (C.c_int, [p, i32, p]),
+        "gist_dpr_encode_many": (C.c_int, [p, i32, i32, p]),
+        "gist_dpr_decode_many": (C.c_int, [p, i32, i32, p]),
     }
     for name, (res, args) in sigs.items():
         fn = getattr(L, name)
@@ -92,13 +116,28 @@ lib = _load()
 
 
 # ------------------------------------------------------------------ marshalling helpers
-def _ptr(t: torch.Tensor | None):
+_F32 = (torch.float32,)
+_W32 = (torch.int32, torch.uint32)  # uint32 words (the binding allocates int32 views)
+_U8 = (torch.uint8,)
+_I32 = (torch.int32,)
+_I64 = (torch.int64,)
+
+
+def _ptr(t: torch.Tensor | None, dtypes=None, device=None, numel: int | None = None, name: str = "tensor"):
+    """Raw device pointer of `t` after the checks the C ABI cannot make: a CUDA tensor,
+    contiguous, of one of `dtypes`, on `device` (when given), with at least `numel` elements."""
     if t is None:
         return None
     if not t.is_cuda:
-        raise ValueError("libgist takes CUDA tensors only (no CPU fallback)")
+        raise ValueError(f"libgist takes CUDA tensors only (no CPU fallback): {name} is on {t.device}")
     if not t.is_contiguous():
-        raise ValueError("libgist takes contiguous tensors")
+        raise ValueError(f"libgist takes contiguous tensors: {name}")
+    if dtypes is not None and t.dtype not in dtypes:
+        raise ValueError(f"{name} must be {' or '.join(str(d) for d in dtypes)}, got {t.dtype}")
+    if device is not None and t.device != device:
+        raise ValueError(f"{name} is on {t.device}, the call's tensors are on {device}")
+    if numel is not None and t.numel() < numel:
+        raise ValueError(f"{name} holds {t.numel()} elements, the call needs {numel}")
     return t.data_ptr()
 
 
@@ -172,28 +211,44 @@ def gist_launch_count() -> int:
 
 
 # ------------------------------------------------------------------ a1..a7
+# Every call runs under torch.cuda.device(<the call's device>), so the library's per-device
+# launch state (SM count, shared-memory opt-ins) is the one of the device the tensors live on.
 def gist_binarize_encode(y: torch.Tensor, mask: torch.Tensor | None = None, stream=None) -> torch.Tensor:
     """a1: 1-bit ReLU mask, int32 tensor of uint32 words (bit i = y[i] > 0)."""
     n = y.numel()
-    mask = _words(gist_binarize_words(n), y.device, mask)
-    _check(lib.gist_binarize_encode(_ptr(y), n, _ptr(mask), _stream(y, stream)), "gist_binarize_encode")
+    dev = y.device
+    mask = _words(gist_binarize_words(n), dev, mask)
+    with torch.cuda.device(dev):
+        _check(lib.gist_binarize_encode(_ptr(y, _F32, name="y"), n,
+                                        _ptr(mask, _W32, dev, gist_binarize_words(n), "mask"), _stream(y, stream)),
+               "gist_binarize_encode")
     return mask
+
+
+def _pool_outputs(x, g, out, argmax):
+    N, Cc, H, W = x.shape
+    Ho, Wo = gist_pool2d_out_dims(H, W, g)
+    if out is None:
+        out = torch.empty((N, Cc, Ho, Wo), dtype=torch.float32, device=x.device)
+    argmax = _words(gist_argmax_words(N * Cc * Ho * Wo), x.device, argmax)
+    return (N, Cc, H, W), N * Cc * Ho * Wo, out, argmax
 
 
 def gist_maxpool_fwd_argmax(y: torch.Tensor, pool, out=None, argmax=None, mask=None, fuse_mask=False,
                             stream=None):
     """a2: returns (out [N,C,Ho,Wo] fp32, argmax int32 words, mask or None).
     fuse_mask=True (or a mask tensor) also writes the a1 mask of y."""
-    N, Cc, H, W = y.shape
     g = Pool2d.of(pool)
-    Ho, Wo = gist_pool2d_out_dims(H, W, g)
-    if out is None:
-        out = torch.empty((N, Cc, Ho, Wo), dtype=torch.float32, device=y.device)
-    argmax = _words(gist_argmax_words(N * Cc * Ho * Wo), y.device, argmax)
+    (N, Cc, H, W), n_out, out, argmax = _pool_outputs(y, g, out, argmax)
+    dev = y.device
     if mask is None and fuse_mask:
-        mask = _words(gist_binarize_words(y.numel()), y.device)
-    _check(lib.gist_maxpool_fwd_argmax(_ptr(y), N, Cc, H, W, C.byref(g), _ptr(out), _ptr(argmax), _ptr(mask),
-                                       _stream(y, stream)), "gist_maxpool_fwd_argmax")
+        mask = _words(gist_binarize_words(y.numel()), dev)
+    with torch.cuda.device(dev):
+        _check(lib.gist_maxpool_fwd_argmax(
+            _ptr(y, _F32, name="y"), N, Cc, H, W, C.byref(g), _ptr(out, _F32, dev, n_out, "out"),
+            _ptr(argmax, _W32, dev, gist_argmax_words(n_out), "argmax"),
+            _ptr(mask, _W32, dev, gist_binarize_words(y.numel()), "mask"), _stream(y, stream)),
+            "gist_maxpool_fwd_argmax")
     return out, argmax, mask
 
 
@@ -201,15 +256,16 @@ def gist_relu_maxpool_fwd_argmax(x: torch.Tensor, pool, out=None, argmax=None, m
     """f3 (P:139, P:152-P:156): ReLU applied on load to the pre-activation map x, then a2 + a1:
     returns (out, argmax words, mask) equal to gist_maxpool_fwd_argmax(relu(x), pool, fuse_mask=True);
     the ReLU output is never materialised."""
-    N, Cc, H, W = x.shape
     g = Pool2d.of(pool)
-    Ho, Wo = gist_pool2d_out_dims(H, W, g)
-    if out is None:
-        out = torch.empty((N, Cc, Ho, Wo), dtype=torch.float32, device=x.device)
-    argmax = _words(gist_argmax_words(N * Cc * Ho * Wo), x.device, argmax)
-    mask = _words(gist_binarize_words(x.numel()), x.device, mask)
-    _check(lib.gist_relu_maxpool_fwd_argmax(_ptr(x), N, Cc, H, W, C.byref(g), _ptr(out), _ptr(argmax), _ptr(mask),
-                                            _stream(x, stream)), "gist_relu_maxpool_fwd_argmax")
+    (N, Cc, H, W), n_out, out, argmax = _pool_outputs(x, g, out, argmax)
+    dev = x.device
+    mask = _words(gist_binarize_words(x.numel()), dev, mask)
+    with torch.cuda.device(dev):
+        _check(lib.gist_relu_maxpool_fwd_argmax(
+            _ptr(x, _F32, name="x"), N, Cc, H, W, C.byref(g), _ptr(out, _F32, dev, n_out, "out"),
+            _ptr(argmax, _W32, dev, gist_argmax_words(n_out), "argmax"),
+            _ptr(mask, _W32, dev, gist_binarize_words(x.numel()), "mask"), _stream(x, stream)),
+            "gist_relu_maxpool_fwd_argmax")
     return out, argmax, mask
 
 
@@ -217,10 +273,17 @@ def gist_pool_relu_bwd(dout: torch.Tensor, argmax: torch.Tensor, mask: torch.Ten
                        dx: torch.Tensor | None = None, stream=None) -> torch.Tensor:
     """a3: dx [N,C,H,W] from dY, the 4-bit argmax map and the 1-bit mask."""
     N, Cc, H, W = shape
+    g = Pool2d.of(pool)
+    Ho, Wo = gist_pool2d_out_dims(H, W, g)
+    n, n_out = N * Cc * H * W, N * Cc * Ho * Wo
+    dev = dout.device
     if dx is None:
-        dx = torch.empty((N, Cc, H, W), dtype=torch.float32, device=dout.device)
-    _check(lib.gist_pool_relu_bwd(_ptr(dout), _ptr(argmax), _ptr(mask), N, Cc, H, W, C.byref(Pool2d.of(pool)),
-                                  _ptr(dx), _stream(dout, stream)), "gist_pool_relu_bwd")
+        dx = torch.empty((N, Cc, H, W), dtype=torch.float32, device=dev)
+    with torch.cuda.device(dev):
+        _check(lib.gist_pool_relu_bwd(
+            _ptr(dout, _F32, dev, n_out, "dout"), _ptr(argmax, _W32, dev, gist_argmax_words(n_out), "argmax"),
+            _ptr(mask, _W32, dev, gist_binarize_words(n), "mask"), N, Cc, H, W, C.byref(g),
+            _ptr(dx, _F32, dev, n, "dx"), _stream(dout, stream)), "gist_pool_relu_bwd")
     return dx
 
 
@@ -240,12 +303,14 @@ def gist_ssdc_encode(x: torch.Tensor, capacity: int | None = None, row_end=None,
         val = torch.empty(max(cap, 1), dtype=torch.float32, device=dev)
     if nnz is None:
         nnz = torch.empty(1, dtype=torch.int64, device=dev)
-    wsb = gist_ssdc_workspace_bytes(n)
     if workspace is None:
         workspace = gist_ssdc_workspace(n, dev, stream)
-    _check(lib.gist_ssdc_encode(_ptr(x), n, _ptr(row_end), _ptr(col), _ptr(val), cap, _ptr(nnz),
-                                _ptr(workspace), workspace.numel() * workspace.element_size(), _stream(x, stream)),
-           "gist_ssdc_encode")
+    with torch.cuda.device(dev):
+        _check(lib.gist_ssdc_encode(
+            _ptr(x, _F32, name="x"), n, _ptr(row_end, _I32, dev, gist_ssdc_rows(n), "row_end"),
+            _ptr(col, _U8, dev, cap, "col"), _ptr(val, _F32, dev, cap, "val"), cap, _ptr(nnz, _I64, dev, 1, "nnz"),
+            _ptr(workspace, None, dev, name="workspace"), workspace.numel() * workspace.element_size(),
+            _stream(x, stream)), "gist_ssdc_encode")
     if trim:
         k = int(nnz.item())
         if k < 0:
@@ -259,10 +324,13 @@ def gist_ssdc_encode(x: torch.Tensor, capacity: int | None = None, row_end=None,
 def gist_ssdc_decode(row_end: torch.Tensor, col: torch.Tensor, val: torch.Tensor, n: int,
                      x: torch.Tensor | None = None, stream=None) -> torch.Tensor:
     """a5: dense fp32 [n] from the CSR encoding."""
+    dev = row_end.device
     if x is None:
-        x = torch.empty(n, dtype=torch.float32, device=row_end.device)
-    _check(lib.gist_ssdc_decode(_ptr(row_end), _ptr(col), _ptr(val), n, _ptr(x), _stream(row_end, stream)),
-           "gist_ssdc_decode")
+        x = torch.empty(n, dtype=torch.float32, device=dev)
+    with torch.cuda.device(dev):
+        _check(lib.gist_ssdc_decode(_ptr(row_end, _I32, dev, gist_ssdc_rows(n), "row_end"),
+                                    _ptr(col, _U8, dev, name="col"), _ptr(val, _F32, dev, name="val"), n,
+                                    _ptr(x, _F32, dev, n, "x"), _stream(row_end, stream)), "gist_ssdc_decode")
     return x
 
 
@@ -272,17 +340,26 @@ def gist_dpr_encode(x: torch.Tensor, bits: int, packed: torch.Tensor | None = No
     words = gist_dpr_words(n, bits)
     if words < 0:
         raise GistError(3, "gist_dpr_encode")
-    packed = _words(words, x.device, packed)
-    _check(lib.gist_dpr_encode(_ptr(x), n, bits, _ptr(packed), _stream(x, stream)), "gist_dpr_encode")
+    dev = x.device
+    packed = _words(words, dev, packed)
+    with torch.cuda.device(dev):
+        _check(lib.gist_dpr_encode(_ptr(x, _F32, name="x"), n, bits, _ptr(packed, _W32, dev, words, "packed"),
+                                   _stream(x, stream)), "gist_dpr_encode")
     return packed
 
 
 def gist_dpr_decode(packed: torch.Tensor, n: int, bits: int, x: torch.Tensor | None = None,
                     stream=None) -> torch.Tensor:
     """a7: packed codes -> fp32 [n]."""
+    dev = packed.device
+    words = gist_dpr_words(n, bits)
+    if words < 0:
+        raise GistError(3, "gist_dpr_decode")
     if x is None:
-        x = torch.empty(n, dtype=torch.float32, device=packed.device)
-    _check(lib.gist_dpr_decode(_ptr(packed), n, bits, _ptr(x), _stream(packed, stream)), "gist_dpr_decode")
+        x = torch.empty(n, dtype=torch.float32, device=dev)
+    with torch.cuda.device(dev):
+        _check(lib.gist_dpr_decode(_ptr(packed, _W32, dev, words, "packed"), n, bits, _ptr(x, _F32, dev, n, "x"),
+                                   _stream(packed, stream)), "gist_dpr_decode")
     return x
 
 
@@ -293,17 +370,173 @@ def gist_ssdc_dpr_encode(val: torch.Tensor, nnz: torch.Tensor, bits: int, capaci
     words = gist_dpr_words(cap, bits)
     if words < 0:
         raise GistError(3, "gist_ssdc_dpr_encode")
-    packed = _words(words, val.device, packed)
-    _check(lib.gist_ssdc_dpr_encode(_ptr(val), _ptr(nnz), cap, bits, _ptr(packed), _stream(val, stream)),
-           "gist_ssdc_dpr_encode")
+    dev = val.device
+    packed = _words(words, dev, packed)
+    with torch.cuda.device(dev):
+        _check(lib.gist_ssdc_dpr_encode(_ptr(val, _F32, dev, cap, "val"), _ptr(nnz, _I64, dev, 1, "nnz"), cap, bits,
+                                        _ptr(packed, _W32, dev, words, "packed"), _stream(val, stream)),
+               "gist_ssdc_dpr_encode")
     return packed
 
 
 def gist_ssdc_dpr_decode(packed: torch.Tensor, nnz: torch.Tensor, bits: int, capacity: int,
                          val: torch.Tensor | None = None, stream=None) -> torch.Tensor:
     """f1: restore the first min(nnz, capacity) CSR values to fp32."""
+    dev = packed.device
+    words = gist_dpr_words(int(capacity), bits)
+    if words < 0:
+        raise GistError(3, "gist_ssdc_dpr_decode")
     if val is None:
-        val = torch.empty(max(capacity, 1), dtype=torch.float32, device=packed.device)
-    _check(lib.gist_ssdc_dpr_decode(_ptr(packed), _ptr(nnz), int(capacity), bits, _ptr(val), _stream(packed, stream)),
-           "gist_ssdc_dpr_decode")
+        val = torch.empty(max(capacity, 1), dtype=torch.float32, device=dev)
+    with torch.cuda.device(dev):
+        _check(lib.gist_ssdc_dpr_decode(_ptr(packed, _W32, dev, words, "packed"), _ptr(nnz, _I64, dev, 1, "nnz"),
+                                        int(capacity), bits, _ptr(val, _F32, dev, int(capacity), "val"),
+                                        _stream(packed, stream)), "gist_ssdc_dpr_decode")
     return val
+
+
+# ------------------------------------------------------------------ many maps per launch (P:171)
+class SsdcEncodeMany:
+    """A prepared gist_ssdc_encode_many call: the job table is marshalled once, and every call
+    re-runs it (one persistent launch per up to 48 maps).  jobs: dicts with x and optional
+    row_end / col / val / nnz / capacity / offset (append mode: a device int64 start offset);
+    missing outputs are allocated like gist_ssdc_encode's.  .outputs[k] = (row_end, col, val, nnz)."""
+
+    def __init__(self, jobs, workspace=None, stream=None):
+        self.outputs, self._keep = [], []
+        arr = (SsdcJob * max(1, len(jobs)))()
+        dev = jobs[0]["x"].device if jobs else None
+        for k, jb in enumerate(jobs):
+            x = jb["x"]
+            n = x.numel()
+            cap = n if jb.get("capacity") is None else int(jb["capacity"])
+            row_end = jb.get("row_end")
+            if row_end is None:
+                row_end = torch.empty(gist_ssdc_rows(n), dtype=torch.int32, device=dev)
+            col = jb.get("col")
+            if col is None:
+                col = torch.empty(max(cap, 1), dtype=torch.uint8, device=dev)
+            val = jb.get("val")
+            if val is None:
+                val = torch.empty(max(cap, 1), dtype=torch.float32, device=dev)
+            nnz = jb.get("nnz")
+            if nnz is None:
+                nnz = torch.empty(1, dtype=torch.int64, device=dev)
+            off = jb.get("offset")
+            arr[k] = SsdcJob(_ptr(x, _F32, dev, name="x"), n, _ptr(row_end, _I32, dev, gist_ssdc_rows(n), "row_end"),
+                             _ptr(col, _U8, dev, cap, "col"), _ptr(val, _F32, dev, cap, "val"), cap,
+                             _ptr(nnz, _I64, dev, 1, "nnz"), _ptr(off, _I64, dev, 1, "offset"))
+            self.outputs.append((row_end, col, val, nnz))
+            self._keep += [x, off]
+        self.jobs, self.count, self.device = arr, len(jobs), dev
+        self.ws_bytes = lib.gist_ssdc_workspace_bytes_many(arr, len(jobs))
+        if workspace is None and jobs:
+            workspace = torch.empty(self.ws_bytes, dtype=torch.uint8, device=dev)
+            gist_ssdc_workspace_init(workspace, stream)
+        self.workspace = workspace
+
+    def __call__(self, stream=None):
+        if not self.count:
+            return self.outputs
+        with torch.cuda.device(self.device):
+            _check(lib.gist_ssdc_encode_many(self.jobs, self.count, _ptr(self.workspace, None, self.device),
+                                             self.workspace.numel() * self.workspace.element_size(),
+                                             _stream(self.workspace, stream)), "gist_ssdc_encode_many")
+        return self.outputs
+
+
+class SsdcDecodeMany:
+    """A prepared gist_ssdc_decode_many call.  jobs: dicts with row_end, col, val, n and optional
+    x / offset.  .outputs[k] = x."""
+
+    def __init__(self, jobs):
+        arr = (SsdcDecodeJob * max(1, len(jobs)))()
+        dev = jobs[0]["row_end"].device if jobs else None
+        self.outputs, self._keep = [], []
+        for k, jb in enumerate(jobs):
+            n = int(jb["n"])
+            x = jb.get("x")
+            if x is None:
+                x = torch.empty(n, dtype=torch.float32, device=dev)
+            off = jb.get("offset")
+            arr[k] = SsdcDecodeJob(_ptr(jb["row_end"], _I32, dev, gist_ssdc_rows(n), "row_end"),
+                                   _ptr(jb["col"], _U8, dev, name="col"), _ptr(jb["val"], _F32, dev, name="val"),
+                                   _ptr(off, _I64, dev, 1, "offset"), n, _ptr(x, _F32, dev, n, "x"))
+            self.outputs.append(x)
+            self._keep += [jb["row_end"], jb["col"], jb["val"], off]
+        self.jobs, self.count, self.device = arr, len(jobs), dev
+
+    def __call__(self, stream=None):
+        if self.count:
+            with torch.cuda.device(self.device):
+                _check(lib.gist_ssdc_decode_many(self.jobs, self.count, _stream(self.outputs[0], stream)),
+                       "gist_ssdc_decode_many")
+        return self.outputs
+
+
+class DprMany:
+    """A prepared gist_dpr_encode_many (encode=True: jobs of x, optional packed) or
+    gist_dpr_decode_many (encode=False: jobs of packed, n, optional x) call."""
+
+    def __init__(self, jobs, bits: int, encode: bool):
+        arr = (DprJob * max(1, len(jobs)))()
+        key = "x" if encode else "packed"
+        dev = jobs[0][key].device if jobs else None
+        self.outputs, self._keep = [], []
+        for k, jb in enumerate(jobs):
+            if encode:
+                x = jb["x"]
+                n = x.numel()
+                words = gist_dpr_words(n, bits)
+                if words < 0:
+                    raise GistError(3, "gist_dpr_encode_many")
+                packed = _words(words, dev, jb.get("packed"))
+                self.outputs.append(packed)
+            else:
+                packed, n = jb["packed"], int(jb["n"])
+                words = gist_dpr_words(n, bits)
+                if words < 0:
+                    raise GistError(3, "gist_dpr_decode_many")
+                x = jb.get("x")
+                if x is None:
+                    x = torch.empty(n, dtype=torch.float32, device=dev)
+                self.outputs.append(x)
+            arr[k] = DprJob(_ptr(x, _F32, dev, n, "x"), n, _ptr(packed, _W32, dev, words, "packed"))
+            self._keep += [x, packed]
+        self.jobs, self.count, self.bits, self.encode, self.device = arr, len(jobs), bits, encode, dev
+
+    def __call__(self, stream=None):
+        if self.count:
+            fn = lib.gist_dpr_encode_many if self.encode else lib.gist_dpr_decode_many
+            with torch.cuda.device(self.device):
+                _check(fn(self.jobs, self.count, self.bits, _stream(self.outputs[0], stream)),
+                       "gist_dpr_encode_many" if self.encode else "gist_dpr_decode_many")
+        return self.outputs
+
+
+def gist_ssdc_workspace_bytes_many(ns) -> int:
+    """Workspace bytes of gist_ssdc_encode_many over maps of these sizes."""
+    arr = (SsdcJob * max(1, len(ns)))()
+    for k, n in enumerate(ns):
+        arr[k].n = int(n)
+    return lib.gist_ssdc_workspace_bytes_many(arr, len(ns))
+
+
+def gist_ssdc_encode_many(jobs, workspace=None, stream=None):
+    """a4 over several maps in one launch; see SsdcEncodeMany.  Returns [(row_end, col, val, nnz)]."""
+    return SsdcEncodeMany(jobs, workspace, stream)(stream)
+
+
+def gist_ssdc_decode_many(jobs, stream=None):
+    """a5 over several maps in one launch; see SsdcDecodeMany.  Returns [x]."""
+    return SsdcDecodeMany(jobs)(stream)
+
+
+def gist_dpr_encode_many(xs, bits: int, stream=None):
+    """a6 over several maps in one launch.  Returns [packed]."""
+    return DprMany([{"x": x} for x in xs], bits, True)(stream)
+
+
+def gist_dpr_decode_many(packed, ns, bits: int, stream=None):
+    """a7 over several maps in one launch.  Returns [x]."""
+    return DprMany([{"packed": p, "n": n} for p, n in zip(packed, ns)], bits, False)(stream)

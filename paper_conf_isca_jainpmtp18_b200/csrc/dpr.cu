@@ -113,16 +113,14 @@ __device__ uint32_t encode_word_scalar(const float *x, int64_t n, int64_t w) {
 }
 
 // Group = 16 input bytes per step for FP16/FP8 (1 float4), 48 for FP10 (3 float4).
+// One map, by thread `tid` of `nthreads` (the many-map kernels rotate tid per map so that small
+// maps land on different threads).
 template <int BITS>
-__global__ void __launch_bounds__(kDprThreads)
-dpr_encode_kernel(const float *__restrict__ x, int64_t n, uint32_t *__restrict__ packed, const int64_t *__restrict__ n_dev) {
-    pdl_enter();
-    if (n_dev) n = min(n, *n_dev);  // count known only on the device (DPR over SSDC values)
+__device__ __forceinline__ void dpr_encode_body(const float *__restrict__ x, int64_t n, uint32_t *__restrict__ packed,
+                                                int64_t tid, int64_t nthreads) {
     constexpr int K = Fmt<BITS>::K;
     constexpr int GF = (BITS == 10) ? 12 : 4;  // floats per group
     const int64_t groups = n / GF;
-    const int64_t tid = (int64_t)blockIdx.x * kDprThreads + threadIdx.x;
-    const int64_t nthreads = (int64_t)gridDim.x * kDprThreads;
     const float4 *x4 = reinterpret_cast<const float4 *>(x);
     constexpr int U = (BITS == 10) ? kUnroll : kUnroll4;
 
@@ -170,13 +168,18 @@ dpr_encode_kernel(const float *__restrict__ x, int64_t n, uint32_t *__restrict__
 
 template <int BITS>
 __global__ void __launch_bounds__(kDprThreads)
-dpr_decode_kernel(const uint32_t *__restrict__ packed, int64_t n, float *__restrict__ x, const int64_t *__restrict__ n_dev) {
+dpr_encode_kernel(const float *__restrict__ x, int64_t n, uint32_t *__restrict__ packed, const int64_t *__restrict__ n_dev) {
     pdl_enter();
     if (n_dev) n = min(n, *n_dev);  // count known only on the device (DPR over SSDC values)
+    dpr_encode_body<BITS>(x, n, packed, (int64_t)blockIdx.x * kDprThreads + threadIdx.x,
+                          (int64_t)gridDim.x * kDprThreads);
+}
+
+template <int BITS>
+__device__ __forceinline__ void dpr_decode_body(const uint32_t *__restrict__ packed, int64_t n, float *__restrict__ x,
+                                                int64_t tid, int64_t nthreads) {
     constexpr int K = Fmt<BITS>::K;
     constexpr uint32_t FIELD = (1u << BITS) - 1u;
-    const int64_t tid = (int64_t)blockIdx.x * kDprThreads + threadIdx.x;
-    const int64_t nthreads = (int64_t)gridDim.x * kDprThreads;
     float4 *x4 = reinterpret_cast<float4 *>(x);
     if constexpr (BITS != 10) {
         // FP16: one uint2 (2 words) -> one float4; FP8: one word -> one float4.  Both sides of
@@ -239,6 +242,53 @@ dpr_decode_kernel(const uint32_t *__restrict__ packed, int64_t n, float *__restr
     }
 }
 
+template <int BITS>
+__global__ void __launch_bounds__(kDprThreads)
+dpr_decode_kernel(const uint32_t *__restrict__ packed, int64_t n, float *__restrict__ x, const int64_t *__restrict__ n_dev) {
+    pdl_enter();
+    if (n_dev) n = min(n, *n_dev);  // count known only on the device (DPR over SSDC values)
+    dpr_decode_body<BITS>(packed, n, x, (int64_t)blockIdx.x * kDprThreads + threadIdx.x,
+                          (int64_t)gridDim.x * kDprThreads);
+}
+
+// Many maps in one launch ("these conversions can happen in parallel"): the grid walks the
+// maps in order, each with the single-map loop; map k's thread index is rotated by the groups of
+// the maps before it, so consecutive small maps run on different threads (and SMs) at once.
+constexpr int kMaxDprJobs = 96;
+struct DprJob {
+    const void *in;
+    void *out;
+    int64_t n;
+};
+struct DprJobs {
+    DprJob j[kMaxDprJobs];
+    int32_t count;
+};
+static_assert(sizeof(DprJobs) + 16 <= 4096, "kernel parameters must fit 4 KB");
+
+template <int BITS, bool ENCODE>
+__global__ void __launch_bounds__(kDprThreads)
+dpr_many_kernel(const __grid_constant__ DprJobs J) {
+    pdl_enter();
+    const int64_t nthreads = (int64_t)gridDim.x * kDprThreads;
+    const int64_t me = (int64_t)blockIdx.x * kDprThreads + threadIdx.x;
+    // FP10 decode is warp-based (384-value chunks): rotate by whole warps
+    constexpr bool WARPS = !ENCODE && BITS == 10;
+    constexpr int GF = ENCODE ? ((BITS == 10) ? 12 : 4) : (BITS == 10 ? 384 : 4);
+    int64_t rot = 0;
+    for (int k = 0; k < J.count; ++k) {
+        const DprJob &jb = J.j[k];
+        int64_t tid = WARPS ? (me + 32 * rot) % nthreads : (me + rot) % nthreads;
+        if (ENCODE)
+            dpr_encode_body<BITS>(reinterpret_cast<const float *>(jb.in), jb.n, reinterpret_cast<uint32_t *>(jb.out),
+                                  tid, nthreads);
+        else
+            dpr_decode_body<BITS>(reinterpret_cast<const uint32_t *>(jb.in), jb.n, reinterpret_cast<float *>(jb.out),
+                                  tid, nthreads);
+        rot += jb.n / GF + 1;
+    }
+}
+
 #ifndef GIST_DPR_CTAS
 #define GIST_DPR_CTAS 8  // grid cap, CTAs per SM
 #endif
@@ -275,6 +325,45 @@ cudaError_t launch_dpr_decode(const uint32_t *packed, int64_t n, int bits, float
         default: return cudaErrorInvalidValue;
     }
     return cudaPeekAtLastError();
+}
+
+cudaError_t launch_dpr_many(const gist_dpr_job *jobs, int32_t count, int bits, bool encode, cudaStream_t s,
+                            int *launches) {
+    *launches = 0;
+    for (int32_t k0 = 0; k0 < count; k0 += kMaxDprJobs) {
+        DprJobs J{};
+        int64_t n_max = 0;
+        for (int32_t k = k0; k < count && k < k0 + kMaxDprJobs; ++k) {
+            DprJob &e = J.j[J.count++];
+            e.in = encode ? (const void *)jobs[k].x : (const void *)jobs[k].packed;
+            e.out = encode ? (void *)jobs[k].packed : (void *)jobs[k].x;
+            e.n = jobs[k].n;
+            n_max = n_max > jobs[k].n ? n_max : jobs[k].n;
+        }
+        int64_t n_sum = 0;
+        for (int k = 0; k < J.count; ++k) n_sum += J.j[k].n;
+        unsigned grid = 1;
+        switch (bits) {
+            case 16: grid = (unsigned)dpr_blocks<16>(n_sum); break;
+            case 10: grid = (unsigned)dpr_blocks<10>(n_sum); break;
+            case 8: grid = (unsigned)dpr_blocks<8>(n_sum); break;
+            default: return cudaErrorInvalidValue;
+        }
+        (void)n_max;
+#define GIST_DPR_MANY(B) \
+    (encode ? launch_k(dpr_many_kernel<B, true>, grid, kDprThreads, 0, s, J) \
+            : launch_k(dpr_many_kernel<B, false>, grid, kDprThreads, 0, s, J))
+        switch (bits) {
+            case 16: GIST_DPR_MANY(16); break;
+            case 10: GIST_DPR_MANY(10); break;
+            case 8: GIST_DPR_MANY(8); break;
+        }
+#undef GIST_DPR_MANY
+        const cudaError_t e = cudaPeekAtLastError();
+        if (e != cudaSuccess) return e;
+        ++*launches;
+    }
+    return cudaSuccess;
 }
 
 }  // namespace gist

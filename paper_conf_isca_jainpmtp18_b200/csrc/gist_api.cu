@@ -1,9 +1,10 @@
 // gist_api.cu — the C ABI (include/gist.h): host-side validation, size helpers, dispatch
-// to the sm_100a kernels.  Stateless apart from the cached SM count.
+// to the sm_100a kernels.  Stateless apart from per-device caches (SM count, shared-memory opt-ins).
 #include <cuda_runtime.h>
 
 #include <atomic>
-#include <mutex>
+#include <climits>
+#include <vector>
 
 #include "../../include/gist.h"
 #include "kernels.h"
@@ -13,16 +14,36 @@ namespace gist {
 static std::atomic<uint64_t> g_launches{0};
 void count_launches(int k) { g_launches.fetch_add((uint64_t)k, std::memory_order_relaxed); }
 
+int current_device() {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0) dev = 0;
+    return dev;
+}
+
+// SM count of the CURRENT device, cached per device (a process may drive several GPUs).
 int num_sms() {
-    static std::once_flag once;
-    static int sms = 148;
-    std::call_once(once, [] {
-        int dev = 0, v = 0;
-        if (cudaGetDevice(&dev) == cudaSuccess &&
-            cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && v > 0)
-            sms = v;
-    });
-    return sms;
+    constexpr int kMaxDev = 64;
+    static std::atomic<int> cache[kMaxDev];
+    const int dev = current_device();
+    if (dev >= kMaxDev) {
+        int v = 0;
+        return cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && v > 0 ? v : 148;
+    }
+    int v = cache[dev].load(std::memory_order_relaxed);
+    if (v <= 0) {
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v <= 0) v = 148;
+        cache[dev].store(v, std::memory_order_relaxed);
+    }
+    return v;
+}
+
+cudaError_t PerDeviceAttr::ensure(const void *func, int smem_bytes) {
+    const int dev = current_device();
+    const uint64_t bit = dev < 64 ? (1ull << dev) : 0ull;
+    if (bit && (done.load(std::memory_order_acquire) & bit)) return cudaSuccess;
+    const cudaError_t e = cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+    if (e == cudaSuccess && bit) done.fetch_or(bit, std::memory_order_acq_rel);
+    return e;
 }
 
 }  // namespace gist
@@ -62,11 +83,11 @@ gist_status launched(cudaError_t e, int kernels) {
 }
 
 int32_t pool_dim(int32_t in, int32_t k, int32_t s, int32_t p, int32_t ceil_mode) {
-    const int32_t span = in + 2 * p - k;
+    const int64_t span = (int64_t)in + 2 * (int64_t)p - k;  // int64: no wrap for any int32 inputs
     if (span < 0) return 0;
-    int32_t out = ceil_mode ? (span + s - 1) / s + 1 : span / s + 1;
-    if (ceil_mode && (int64_t)(out - 1) * s >= (int64_t)in + p) out -= 1;
-    return out;
+    int64_t out = ceil_mode ? (span + s - 1) / s + 1 : span / s + 1;
+    if (ceil_mode && (out - 1) * s >= (int64_t)in + p) out -= 1;
+    return out > INT32_MAX ? -1 : (int32_t)out;
 }
 
 gist_status check_pool(int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d *p, int32_t *Ho, int32_t *Wo) {
@@ -74,7 +95,8 @@ gist_status check_pool(int32_t N, int32_t C, int32_t H, int32_t W, const gist_po
     if (p->kh < 1 || p->kw < 1 || p->sh < 1 || p->sw < 1 || p->ph < 0 || p->pw < 0 || p->ph > p->kh / 2 ||
         p->pw > p->kw / 2)
         return GIST_ERR_INVALID_ARGUMENT;
-    if (p->kh * p->kw > 16) return GIST_ERR_UNSUPPORTED;  // argmax must fit 4 bits
+    // argmax must fit 4 bits; each side is bounded first so the product cannot wrap
+    if (p->kh > 16 || p->kw > 16 || (int64_t)p->kh * p->kw > 16) return GIST_ERR_UNSUPPORTED;
     *Ho = pool_dim(H, p->kh, p->sh, p->ph, p->ceil_mode);
     *Wo = pool_dim(W, p->kw, p->sw, p->pw, p->ceil_mode);
     if ((H > 0 && *Ho < 1) || (W > 0 && *Wo < 1)) return GIST_ERR_INVALID_ARGUMENT;
@@ -181,25 +203,79 @@ gist_status gist_pool_relu_bwd(const float *dout, const uint32_t *argmax, const 
     return launched(gist::launch_pool_bwd(dout, argmax, mask, N, C, H, W, *p, Ho, Wo, dx, stream), 1);
 }
 
-gist_status gist_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val, int64_t capacity,
-                             int64_t *nnz, void *workspace, size_t workspace_bytes, cudaStream_t stream) {
+// Host-side checks of one SSDC encode job (shared by the single- and many-map calls).
+static gist_status check_ssdc_job(const gist_ssdc_job &j, const void *workspace, size_t workspace_bytes) {
+    const int64_t n = j.n, capacity = j.capacity;
     if (n < 0 || capacity < 0) return GIST_ERR_INVALID_ARGUMENT;
     if (n >= kI32Limit) return GIST_ERR_TOO_LARGE;
-    if (!nnz) return GIST_ERR_INVALID_ARGUMENT;
-    if (n > 0 && (!x || !row_end || !workspace)) return GIST_ERR_INVALID_ARGUMENT;
-    if (capacity > 0 && (!col || !val)) return GIST_ERR_INVALID_ARGUMENT;
-    if (misaligned(x) || misaligned(row_end) || misaligned(col) || misaligned(val) || misaligned(workspace) ||
-        (reinterpret_cast<uintptr_t>(nnz) & 7u))
+    if (!j.nnz) return GIST_ERR_INVALID_ARGUMENT;
+    if (n > 0 && (!j.x || !j.row_end || !workspace)) return GIST_ERR_INVALID_ARGUMENT;
+    if (capacity > 0 && (!j.col || !j.val)) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(j.x) || misaligned(j.row_end) || misaligned(j.col) || misaligned(j.val) || misaligned(workspace) ||
+        (reinterpret_cast<uintptr_t>(j.nnz) & 7u) || (reinterpret_cast<uintptr_t>(j.offset) & 7u))
         return GIST_ERR_MISALIGNED;
-    if (n > 0 && workspace_bytes < gist_ssdc_workspace_bytes(n)) return GIST_ERR_INVALID_ARGUMENT;
-    const int64_t cap = capacity < n ? capacity : n;
-    if (any_overlap({{x, 4 * n}}, {{row_end, 4 * gist_ssdc_rows(n)}, {col, cap}, {val, 4 * cap}, {nnz, 8},
-                                   {workspace, (int64_t)workspace_bytes}}))
+    // plain mode writes at most n entries; append mode anywhere in the capacity-sized arena
+    const int64_t cap = j.offset ? capacity : (capacity < n ? capacity : n);
+    if (any_overlap({{j.x, 4 * n}, {j.offset, j.offset ? 8 : 0}},
+                    {{j.row_end, 4 * gist_ssdc_rows(n)}, {j.col, cap}, {j.val, 4 * cap}, {j.nnz, 8},
+                     {workspace, (int64_t)workspace_bytes}}))
         return GIST_ERR_INVALID_ARGUMENT;
-    if (n == 0) {  // still publish nnz = 0 (stream-ordered)
-        return cudaMemsetAsync(nnz, 0, sizeof(int64_t), stream) == cudaSuccess ? GIST_OK : GIST_ERR_CUDA;
-    }
+    return GIST_OK;
+}
+
+// n == 0: publish *nnz (= 0, or the start offset in append mode) in stream order, no kernel
+static gist_status publish_empty(const gist_ssdc_job &j, cudaStream_t stream) {
+    const cudaError_t e = j.offset ? cudaMemcpyAsync(j.nnz, j.offset, sizeof(int64_t), cudaMemcpyDeviceToDevice, stream)
+                                   : cudaMemsetAsync(j.nnz, 0, sizeof(int64_t), stream);
+    return e == cudaSuccess ? GIST_OK : GIST_ERR_CUDA;
+}
+
+gist_status gist_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val, int64_t capacity,
+                             int64_t *nnz, void *workspace, size_t workspace_bytes, cudaStream_t stream) {
+    const gist_ssdc_job j{x, n, row_end, col, val, capacity, nnz, nullptr};
+    gist_status st = check_ssdc_job(j, workspace, workspace_bytes);
+    if (st != GIST_OK) return st;
+    if (n > 0 && workspace_bytes < gist_ssdc_workspace_bytes(n)) return GIST_ERR_INVALID_ARGUMENT;
+    if (n == 0) return publish_empty(j, stream);
     return launched(gist::launch_ssdc_encode(x, n, row_end, col, val, capacity, nnz, workspace, stream), 1);
+}
+
+size_t gist_ssdc_workspace_bytes_many(const gist_ssdc_job *jobs, int32_t count) {
+    if (!jobs || count <= 0) return gist_ssdc_workspace_bytes(0);
+    return gist::ssdc_workspace_bytes_many(jobs, count);
+}
+
+gist_status gist_ssdc_encode_many(const gist_ssdc_job *jobs, int32_t count, void *workspace, size_t workspace_bytes,
+                                  cudaStream_t stream) {
+    if (count < 0 || (count > 0 && !jobs)) return GIST_ERR_INVALID_ARGUMENT;
+    if (count == 0) return GIST_OK;
+    std::vector<gist_ssdc_job> live;
+    live.reserve(count);
+    for (int32_t k = 0; k < count; ++k) {
+        const gist_status st = check_ssdc_job(jobs[k], workspace, workspace_bytes);
+        if (st != GIST_OK) return st;
+        if (jobs[k].n > 0) live.push_back(jobs[k]);
+    }
+    if (!live.empty() && workspace_bytes < gist::ssdc_workspace_bytes_many(live.data(), (int32_t)live.size()))
+        return GIST_ERR_INVALID_ARGUMENT;
+    // an offset may be the nnz (end offset) of the PREVIOUS job only (a chained arena); any other job's
+    // nnz, or its own, is written during the launch
+    for (int32_t k = 0; k < count; ++k) {
+        if (!jobs[k].offset) continue;
+        for (int32_t i = 0; i < count; ++i)
+            if (jobs[i].nnz == jobs[k].offset && i != k - 1) return GIST_ERR_INVALID_ARGUMENT;
+        if (k > 0 && jobs[k].offset == jobs[k - 1].nnz && (jobs[k].n == 0 || jobs[k - 1].n == 0))
+            return GIST_ERR_INVALID_ARGUMENT;  // chaining links launched maps (n > 0) only
+    }
+    for (int32_t k = 0; k < count; ++k)
+        if (jobs[k].n == 0) {
+            const gist_status st = publish_empty(jobs[k], stream);
+            if (st != GIST_OK) return st;
+        }
+    if (live.empty()) return GIST_OK;
+    int launches = 0;
+    const cudaError_t e = gist::launch_ssdc_encode_many(live.data(), (int32_t)live.size(), workspace, stream, &launches);
+    return launched(e, launches);
 }
 
 gist_status gist_ssdc_workspace_init(void *workspace, size_t bytes, cudaStream_t stream) {
@@ -210,17 +286,42 @@ gist_status gist_ssdc_workspace_init(void *workspace, size_t bytes, cudaStream_t
     return launched(gist::launch_ssdc_workspace_init(workspace, bytes, stream), 1);
 }
 
-gist_status gist_ssdc_decode(const int32_t *row_end, const uint8_t *col, const float *val, int64_t n, float *x,
-                             cudaStream_t stream) {
+static gist_status check_ssdc_decode_job(const gist_ssdc_decode_job &j) {
+    const int64_t n = j.n;
     if (n < 0) return GIST_ERR_INVALID_ARGUMENT;
     if (n >= kI32Limit) return GIST_ERR_TOO_LARGE;
     if (n == 0) return GIST_OK;
-    if (!row_end || !x) return GIST_ERR_INVALID_ARGUMENT;
-    if (misaligned(row_end) || misaligned(col) || misaligned(val) || misaligned(x)) return GIST_ERR_MISALIGNED;
-    if (any_overlap({{row_end, 4 * gist_ssdc_rows(n)}}, {{x, 4 * n}})) return GIST_ERR_INVALID_ARGUMENT;
+    if (!j.row_end || !j.x) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(j.row_end) || misaligned(j.col) || misaligned(j.val) || misaligned(j.x) ||
+        (reinterpret_cast<uintptr_t>(j.offset) & 7u))
+        return GIST_ERR_MISALIGNED;
+    if (any_overlap({{j.row_end, 4 * gist_ssdc_rows(n)}, {j.offset, j.offset ? 8 : 0}}, {{j.x, 4 * n}}))
+        return GIST_ERR_INVALID_ARGUMENT;
+    return GIST_OK;
+}
+
+gist_status gist_ssdc_decode(const int32_t *row_end, const uint8_t *col, const float *val, int64_t n, float *x,
+                             cudaStream_t stream) {
+    const gist_ssdc_decode_job j{row_end, col, val, nullptr, n, x};
+    const gist_status st = check_ssdc_decode_job(j);
+    if (st != GIST_OK || n == 0) return st;
     // col/val extents are only known on the device (row_end[rows-1]); they may be NULL only
     // for an all-zero map, which the kernel then never dereferences.
     return launched(gist::launch_ssdc_decode(row_end, col, val, n, x, stream), 1);
+}
+
+gist_status gist_ssdc_decode_many(const gist_ssdc_decode_job *jobs, int32_t count, cudaStream_t stream) {
+    if (count < 0 || (count > 0 && !jobs)) return GIST_ERR_INVALID_ARGUMENT;
+    std::vector<gist_ssdc_decode_job> live;
+    for (int32_t k = 0; k < count; ++k) {
+        const gist_status st = check_ssdc_decode_job(jobs[k]);
+        if (st != GIST_OK) return st;
+        if (jobs[k].n > 0) live.push_back(jobs[k]);
+    }
+    if (live.empty()) return GIST_OK;
+    int launches = 0;
+    const cudaError_t e = gist::launch_ssdc_decode_many(live.data(), (int32_t)live.size(), stream, &launches);
+    return launched(e, launches);
 }
 
 gist_status gist_dpr_encode(const float *x, int64_t n, int32_t bits, uint32_t *packed, cudaStream_t stream) {
@@ -241,6 +342,25 @@ gist_status gist_dpr_decode(const uint32_t *packed, int64_t n, int32_t bits, flo
     if (misaligned(x) || misaligned(packed)) return GIST_ERR_MISALIGNED;
     if (any_overlap({{packed, 4 * gist_dpr_words(n, bits)}}, {{x, 4 * n}})) return GIST_ERR_INVALID_ARGUMENT;
     return launched(gist::launch_dpr_decode(packed, n, bits, x, stream), 1);
+}
+
+static gist_status dpr_many(const gist_dpr_job *jobs, int32_t count, int32_t bits, bool encode, cudaStream_t stream) {
+    if (bits != 8 && bits != 10 && bits != 16) return GIST_ERR_UNSUPPORTED;
+    if (count < 0 || (count > 0 && !jobs)) return GIST_ERR_INVALID_ARGUMENT;
+    std::vector<gist_dpr_job> live;
+    for (int32_t k = 0; k < count; ++k) {
+        const gist_dpr_job &j = jobs[k];
+        if (j.n < 0) return GIST_ERR_INVALID_ARGUMENT;
+        if (j.n == 0) continue;
+        if (!j.x || !j.packed) return GIST_ERR_INVALID_ARGUMENT;
+        if (misaligned(j.x) || misaligned(j.packed)) return GIST_ERR_MISALIGNED;
+        if (overlap({j.x, 4 * j.n}, {j.packed, 4 * gist_dpr_words(j.n, bits)})) return GIST_ERR_INVALID_ARGUMENT;
+        live.push_back(j);
+    }
+    if (live.empty()) return GIST_OK;
+    int launches = 0;
+    const cudaError_t e = gist::launch_dpr_many(live.data(), (int32_t)live.size(), bits, encode, stream, &launches);
+    return launched(e, launches);
 }
 
 gist_status gist_ssdc_dpr_encode(const float *val, const int64_t *nnz, int64_t capacity, int32_t bits,
@@ -265,6 +385,14 @@ gist_status gist_ssdc_dpr_decode(const uint32_t *packed, const int64_t *nnz, int
     if (any_overlap({{packed, 4 * gist_dpr_words(capacity, bits)}, {nnz, 8}}, {{val, 4 * capacity}}))
         return GIST_ERR_INVALID_ARGUMENT;
     return launched(gist::launch_dpr_decode(packed, capacity, bits, val, stream, nnz), 1);
+}
+
+gist_status gist_dpr_encode_many(const gist_dpr_job *jobs, int32_t count, int32_t bits, cudaStream_t stream) {
+    return dpr_many(jobs, count, bits, true, stream);
+}
+
+gist_status gist_dpr_decode_many(const gist_dpr_job *jobs, int32_t count, int32_t bits, cudaStream_t stream) {
+    return dpr_many(jobs, count, bits, false, stream);
 }
 
 }  // extern "C"

@@ -4,11 +4,21 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
+
 #include "../../include/gist.h"
 
 namespace gist {
 
-int num_sms();
+int current_device();
+int num_sms();  // of the current device (cached per device)
+// Dynamic shared-memory opt-in (cudaFuncAttributeMaxDynamicSharedMemorySize) of one kernel, applied
+// once per DEVICE: the attribute is per device, so a process that launches on a second GPU sets it
+// there too.
+struct PerDeviceAttr {
+    std::atomic<uint64_t> done{0};  // bit d: set on device d (devices >= 64: set on every launch)
+    cudaError_t ensure(const void *func, int smem_bytes);
+};
 void count_launches(int k);  // bookkeeping for gist_launch_count()
 
 cudaError_t launch_binarize(const float *y, int64_t n, uint32_t *mask, cudaStream_t s);
@@ -33,11 +43,20 @@ size_t ssdc_workspace_bytes(int64_t n);
 cudaError_t launch_ssdc_workspace_init(void *workspace, size_t bytes, cudaStream_t s);
 cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val,
                                int64_t capacity, int64_t *nnz, void *workspace, cudaStream_t s);
+int64_t ssdc_tiles(int64_t n);
+size_t ssdc_workspace_bytes_many(const gist_ssdc_job *jobs, int32_t count);
+// every job has n > 0; *launches = kernels enqueued
+cudaError_t launch_ssdc_encode_many(const gist_ssdc_job *jobs, int32_t count, void *workspace, cudaStream_t s,
+                                    int *launches);
+cudaError_t launch_ssdc_decode_many(const gist_ssdc_decode_job *jobs, int32_t count, cudaStream_t s, int *launches);
 cudaError_t launch_ssdc_decode(const int32_t *row_end, const uint8_t *col, const float *val, int64_t n, float *x,
                                cudaStream_t s);
 // n_dev != nullptr: the element count is min(n, *n_dev), read on the device.
 cudaError_t launch_dpr_encode(const float *x, int64_t n, int bits, uint32_t *packed, cudaStream_t s,
                               const int64_t *n_dev = nullptr);
+// every job has n > 0
+cudaError_t launch_dpr_many(const gist_dpr_job *jobs, int32_t count, int bits, bool encode, cudaStream_t s,
+                            int *launches);
 cudaError_t launch_dpr_decode(const uint32_t *packed, int64_t n, int bits, float *x, cudaStream_t s,
                               const int64_t *n_dev = nullptr);
 

@@ -647,11 +647,13 @@ pool_bwd_k3s2_block_kernel(const float *__restrict__ dout, const uint32_t *__res
         const bool r1 = 2 * (int)A + 1 < a.H, c1 = 2 * (int)b + 1 < a.W;
         uint32_t m0 = 3u, m1 = 3u;
         if (mask) {
-            const uint32_t w0 = ld_ro(mask + (i00 >> 5)), w0b = ld_ro(mask + ((i00 + 1) >> 5));
+            // the right-hand bit is read only when that column exists (c1): in the last column of
+            // an odd-W map, element i00 + 1 may be element n, one word past the mask buffer
+            const uint32_t w0 = ld_ro(mask + (i00 >> 5)), w0b = c1 ? ld_ro(mask + ((i00 + 1) >> 5)) : 0u;
             m0 = ((w0 >> (i00 & 31)) & 1u) | (((w0b >> ((i00 + 1) & 31)) & 1u) << 1);
             if (r1) {
                 const int64_t i10 = i00 + a.W;
-                const uint32_t w1 = ld_ro(mask + (i10 >> 5)), w1b = ld_ro(mask + ((i10 + 1) >> 5));
+                const uint32_t w1 = ld_ro(mask + (i10 >> 5)), w1b = c1 ? ld_ro(mask + ((i10 + 1) >> 5)) : 0u;
                 m1 = ((w1 >> (i10 & 31)) & 1u) | (((w1b >> ((i10 + 1) & 31)) & 1u) << 1);
             }
         }

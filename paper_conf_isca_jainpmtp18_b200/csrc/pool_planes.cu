@@ -13,7 +13,6 @@
 #include <math_constants.h>
 
 #include <algorithm>
-#include <mutex>
 
 #include "common.cuh"
 #include "kernels.h"
@@ -208,10 +207,9 @@ cudaError_t launch_pool3s1_planes_bwd(const float *dout, const uint32_t *argmax,
     const int64_t G = a.G;
     a.a_off = (int32_t)((G * a.HoWo + 8 + 3) & ~3ll);
     a.m_off = (int32_t)((a.a_off + (G * a.HoWo + 7) / 8 + 8 + 3) & ~3ll);
-    static std::once_flag once;
-    std::call_once(once, [] {
-        cudaFuncSetAttribute(pool3s1_planes_bwd_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)planes_smem());
-    });
+    static PerDeviceAttr attr;
+    const cudaError_t ea = attr.ensure(reinterpret_cast<const void *>(pool3s1_planes_bwd_kernel), (int)planes_smem());
+    if (ea != cudaSuccess) return ea;
     const unsigned grid = (unsigned)std::min<int64_t>(a.groups, num_sms());
     launch_k(pool3s1_planes_bwd_kernel, grid, kPT, planes_smem(), s, dout, argmax, mask, a, dx);
     return cudaPeekAtLastError();

@@ -35,7 +35,6 @@
 #include "kernels.h"
 #include "tma.cuh"
 
-#include <mutex>
 
 namespace gist {
 
@@ -73,9 +72,10 @@ constexpr int kPartElems = kPartRows * kRow;           // 8 KB per TMA stage (4 
 constexpr int kStages = GIST_SSDC_STAGES;
 constexpr int kQ = GIST_SSDC_Q;
 constexpr int kProd = 0, kCount = 1, kPub = kCount + kParts, kGather = kPub + 1, kWriter0 = kGather + 1;
-constexpr int kEncThreads = 32 * (kWriter0 + kWriters);  // 480
+constexpr int kEncThreads = 32 * (kWriter0 + kWriters);  // 23 warps = 736 threads
 constexpr int kStage = kWRows * kRow + 16;  // staged entries per writer warp (+ 16-entry phase)
 constexpr int kGatherPer = 8;                     // totals per lane per gather round (256 per warp)
+constexpr int kMaxEncJobs = 48;                   // maps per encode launch (job table in kernel params)
 // Workspace (zeroed once by the caller, left reusable by every call): u32 words ticket [0],
 // done [1] (CTAs finished), epoch [2] (calls completed); u64 tot[tiles] from word kTotOffset.
 // tot[t] = (epoch + 1) << 32 | count: the tag makes the previous call's totals read as
@@ -92,6 +92,28 @@ __global__ void ssdc_ws_init_kernel(uint32_t *ws, int64_t words) {
 static_assert(kStages % kParts == 0, "each counter warp owns the stages of its part");
 static_assert(kPartRows % 2 == 0, "counters reduce two rows at a time");
 
+// Job table (a kernel parameter, < 4 KB): one launch encodes up to kMaxEncJobs maps.  The tiles of
+// all jobs form one ticket space (job j owns global tiles [tile0_j, tile0_{j+1})), so a single
+// persistent grid streams every map with one fill and one drain, and each job's running prefix
+// restarts at its first tile (no wait on the totals of earlier jobs).
+struct EncJob {
+    const float *x;
+    int32_t *row_end;
+    uint8_t *col;
+    float *val;
+    int64_t *nnz;
+    const int64_t *base;  // NULL, or the device offset where this job's entries start (append mode)
+    int64_t n, capacity, tile0;
+    int32_t head;  // first job of this job's chain (a job whose offset is the previous job's nnz
+                   // continues that job's entries; the prefix then runs across both)
+};
+struct EncJobs {
+    EncJob j[kMaxEncJobs];
+    int64_t tiles;  // total tiles of all jobs
+    int32_t count;
+};
+static_assert(sizeof(EncJobs) + 16 <= 4096, "kernel parameters must fit 4 KB");
+
 struct __align__(128) EncSmem {
     float raw[kStages][kPartElems];  // TMA ring (parts of tiles)
     uint32_t vst[kWriters][kStage];  // per-writer compacted value bits (congruent to the output mod 4)
@@ -100,6 +122,7 @@ struct __align__(128) EncSmem {
     uint32_t rinc[kQ][kTileRows];   // tile-local inclusive row ends
     int64_t base[kQ];                // global offset of the tile
     int64_t tile[kQ];                // tile claimed in this slot (>= tiles: no more work)
+    int32_t job[kQ];                 // job of that tile
     uint64_t full[kStages], empty[kStages];
     uint64_t counted[kQ], published[kQ], resolved[kQ], freed[kQ];
 };
@@ -134,8 +157,11 @@ __device__ __forceinline__ uint32_t nz4(const uint4 &a) {  // nonzero bit patter
 // (64 B) and col (16 B) leave as two 1-D bulk copies (cp.async.bulk shared -> global) issued
 // by lane 0; the ragged head and tail (< 16 entries each) by lanes 0..15 and 16..31.
 __device__ __forceinline__ void write_rows(EncSmem &S, int q, int w, int lane, const uint4 (&lo)[kWRows],
-                                           const uint4 (&hi)[kWRows], uint8_t *__restrict__ col,
-                                           float *__restrict__ val, int64_t capacity) {
+                                           const uint4 (&hi)[kWRows], const EncJobs &J) {
+    const EncJob &jb = J.j[S.job[q]];
+    uint8_t *__restrict__ col = jb.col;
+    float *__restrict__ val = jb.val;
+    const int64_t capacity = jb.capacity;
     const int rw = w * kWRows;
     const int64_t tile_base = S.base[q];
     const uint32_t w_excl = rw ? S.rinc[q][rw - 1] : 0u;
@@ -225,9 +251,8 @@ __device__ __forceinline__ void trace(int64_t j, int ev) {
 #endif
 
 __global__ void __launch_bounds__(kEncThreads, 1)
-ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t tiles,
-                    int32_t *__restrict__ row_end, uint8_t *__restrict__ col, float *__restrict__ val,
-                    int64_t capacity, int64_t *__restrict__ nnz_out, uint32_t *__restrict__ ws) {
+ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws) {
+    const int64_t tiles = J.tiles;
     extern __shared__ __align__(128) unsigned char smem_raw[];
     EncSmem &S = *reinterpret_cast<EncSmem *>(smem_raw);
     const int lane = threadIdx.x & 31;
@@ -262,7 +287,8 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
     uint32_t epoch, magic;
     asm volatile("ld.volatile.global.v2.u32 {%0, %1}, [%2];" : "=r"(epoch), "=r"(magic) : "l"(ws + 2) : "memory");
     if (magic != kWsMagic) {  // never initialised: report, no work
-        if (blockIdx.x == 0 && threadIdx.x == 0) *nnz_out = -1;
+        if (blockIdx.x == 0 && threadIdx.x == 0)
+            for (int k = 0; k < J.count; ++k) *J.j[k].nnz = -1;
         return;
     }
     // every CTA reads the epoch before it counts itself done, so all see the same value
@@ -281,23 +307,28 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
             }
 #endif
             int64_t t = first_ticket;
+            int jc = 0;  // job cursor: tickets rise, so jobs only move forward
             for (int64_t j = 0;; ++j) {
                 const int q = (int)(j % kQ);
                 if (j >= kQ) mbar_wait_sleep(&S.freed[q], (uint32_t)(j / kQ - 1) & 1u);
+                if (t < tiles)
+                    while (jc + 1 < J.count && t >= J.j[jc + 1].tile0) ++jc;
                 S.tile[q] = t;
+                S.job[q] = jc;
                 TRACE(j, 0);
-                const int64_t e_tile = t * (int64_t)(kTileRows * kRow);
+                const EncJob &jb = J.j[jc];
+                const int64_t e_tile = (t - jb.tile0) * (int64_t)(kTileRows * kRow);
                 for (int h = 0; h < kParts; ++h) {
                     const int64_t js = kParts * j + h;
                     const int s = (int)(js % kStages);
                     if (js >= kStages) mbar_wait_sleep(&S.empty[s], (uint32_t)(js / kStages - 1) & 1u);
                     const int64_t e0 = e_tile + h * kPartElems;
-                    const int64_t avail = t < tiles ? n - e0 : 0;
+                    const int64_t avail = t < tiles ? jb.n - e0 : 0;
                     const uint32_t bytes =
                         avail >= kPartElems ? kPartElems * 4u : (avail > 0 ? (uint32_t)((avail * 4) & ~15ll) : 0u);
-                    mbar_arrive_expect_tx(&S.full[s], bytes);  // also publishes S.tile[q] to the counter
+                    mbar_arrive_expect_tx(&S.full[s], bytes);  // also publishes S.tile/job[q] to the counter
                     if (bytes) {
-                        tma_load_1d_normal(S.raw[s], x + e0, bytes, &S.full[s]);
+                        tma_load_1d_normal(S.raw[s], jb.x + e0, bytes, &S.full[s]);
                     }
                 }
                 if (t >= tiles) break;
@@ -315,11 +346,12 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
             const int64_t t = S.tile[q];
             if (t < tiles) {
                 float *T = S.raw[s];
-                const int64_t e0 = t * (int64_t)(kTileRows * kRow) + h * kPartElems;
-                const int64_t avail = n - e0;
+                const EncJob &jb = J.j[S.job[q]];
+                const int64_t e0 = (t - jb.tile0) * (int64_t)(kTileRows * kRow) + h * kPartElems;
+                const int64_t avail = jb.n - e0;
                 if (avail < kPartElems) {  // ragged end of the map: the part the TMA could not copy, zeros
                     const int from = avail > 0 ? (int)(((avail * 4) & ~15ll) / 4) : 0;
-                    for (int i = from + lane; i < kPartElems; i += 32) T[i] = (i < avail) ? x[e0 + i] : 0.0f;
+                    for (int i = from + lane; i < kPartElems; i += 32) T[i] = (i < avail) ? jb.x[e0 + i] : 0.0f;
                     fence_proxy_async_smem();  // generic writes into a TMA stage (once per call)
                     __syncwarp();
                 }
@@ -368,11 +400,18 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
         // CTA's tiles t: sum tot[pos .. t) (up to 256 totals per coalesced round trip; re-poll
         // until all are published), base(t) = sum.
         int64_t pos = 0, sum = 0;
+        int cur = -1;  // chain head of the running prefix
         for (int64_t j = 0;; ++j) {
             const int q = (int)(j % kQ);
             mbar_wait_sleep(&S.published[q], (uint32_t)(j / kQ) & 1u);
             const int64_t t = S.tile[q];
-            const int64_t upto = t < tiles ? t : 0;
+            const int jj = S.job[q];
+            if (t < tiles && J.j[jj].head != cur) {  // first tile of a new chain for this CTA: restart
+                cur = J.j[jj].head;
+                pos = J.j[cur].tile0;
+                sum = J.j[cur].base ? *J.j[cur].base : 0;
+            }
+            const int64_t upto = t < tiles ? t : pos;
             while (pos < upto) {
                 uint64_t v[kGatherPer];
 #pragma unroll
@@ -397,10 +436,12 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
                 if (ready < 32 * kGatherPer && pos < upto) __nanosleep(32);
             }
             if (t < tiles) {
+                const EncJob &jb = J.j[jj];
                 if (lane == 0) S.base[q] = sum;
-                const int64_t r = t * kTileRows + lane;  // kTileRows == 32: lane r owns row r
-                if (r < rows) row_end[r] = (int32_t)(sum + S.rinc[q][lane]);
-                if (t == tiles - 1 && lane == 0) *nnz_out = sum + S.rinc[q][kTileRows - 1];
+                const int64_t r = (t - jb.tile0) * kTileRows + lane;  // kTileRows == 32: lane r owns row r
+                if (r < (jb.n + kRow - 1) / kRow) jb.row_end[r] = (int32_t)(sum + S.rinc[q][lane]);
+                const int64_t last = (jj + 1 < J.count ? J.j[jj + 1].tile0 : tiles) - 1;
+                if (t == last && lane == 0) *jb.nnz = sum + S.rinc[q][kTileRows - 1];
             }
             __syncwarp();
             if (lane == 0) {
@@ -444,7 +485,7 @@ ssdc_encode_kernel(const float *__restrict__ x, int64_t n, int64_t rows, int64_t
         auto retire = [&](int64_t jj, int64_t t, const uint4 (&l)[kWRows], const uint4 (&h)[kWRows]) {
             const int q = (int)(jj % kQ);
             mbar_wait_sleep(&S.resolved[q], (uint32_t)(jj / kQ) & 1u);
-            write_rows(S, q, w, lane, l, h, col, val, capacity);
+            write_rows(S, q, w, lane, l, h, J);
             __syncwarp();
             if (lane == 0) {
                 if (w == 0) TRACE(jj, 3);
@@ -482,33 +523,66 @@ constexpr int kDecRows = 4;  // rows per warp iteration
 #define GIST_SSDC_DEC_BATCH 8
 #endif
 constexpr int kDecBatch = GIST_SSDC_DEC_BATCH;  // col/val entries per lane in flight
+constexpr int kMaxDecJobs = 64;                 // maps per decode launch (job table in kernel params)
 
+struct DecJob {
+    const int32_t *row_end;
+    const uint8_t *col;
+    const float *val;
+    const int64_t *base;  // NULL, or the device offset where the map's entries start (append mode)
+    float *x;
+    int64_t n;
+    int64_t g0;  // first global 4-row group of the map
+};
+struct DecJobs {
+    DecJob j[kMaxDecJobs];
+    int64_t groups;
+    int32_t count;
+};
+static_assert(sizeof(DecJobs) + 16 <= 4096, "kernel parameters must fit 4 KB");
+
+// The 4-row groups of all maps form one index space; a warp takes groups g, g + nwarps, ... and
+// advances its job cursor monotonically.
 __global__ void __launch_bounds__(kDecThreads)
-ssdc_decode_kernel(const int32_t *__restrict__ row_end, const uint8_t *__restrict__ col,
-                   const float *__restrict__ val, int64_t n, int64_t rows, float *__restrict__ x) {
+ssdc_decode_kernel(const __grid_constant__ DecJobs J) {
     pdl_enter();
     __shared__ __align__(16) float s_buf[kDecThreads / 32][kDecRows * kRow];
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     float *buf = s_buf[warp];
-    const int64_t groups = (rows + kDecRows - 1) / kDecRows;
+    const int64_t groups = J.groups;
     const int64_t gwarp = ((int64_t)blockIdx.x * kDecThreads + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * kDecThreads) >> 5;
+    auto job_of = [&](int64_t g, int jc) {
+        while (jc + 1 < J.count && g >= J.j[jc + 1].g0) ++jc;
+        return jc;
+    };
 
     // lanes 0..4 hold the row boundaries of the warp's next group: bound[j] = end of row r0-1+j
     // (loaded one group ahead, so only the col/val loads are on each group's critical path)
-    auto bounds = [&](int64_t g) -> int32_t {
-        const int64_t r = g * kDecRows - 1 + lane;
+    auto bounds = [&](int64_t g, int jc) -> int32_t {
         if (g >= groups || lane > kDecRows) return 0;
-        return (r < 0) ? 0 : (r < rows ? row_end[r] : row_end[rows - 1]);
+        const DecJob &jb = J.j[jc];
+        const int64_t rows = (jb.n + kRow - 1) / kRow;
+        const int64_t r = (g - jb.g0) * kDecRows - 1 + lane;
+        if (r < 0) return jb.base ? (int32_t)*jb.base : 0;
+        return r < rows ? jb.row_end[r] : jb.row_end[rows - 1];
     };
-    int32_t bnd = bounds(gwarp);
+    int jc = job_of(gwarp < groups ? gwarp : 0, 0);
+    int32_t bnd = bounds(gwarp, jc);
     for (int64_t g = gwarp; g < groups; g += nwarps) {
-        const int64_t r0 = g * kDecRows;
+        const DecJob &jb = J.j[jc];
+        const int64_t r0 = (g - jb.g0) * kDecRows;
         const int32_t b0 = __shfl_sync(kFull, bnd, 0), b1 = __shfl_sync(kFull, bnd, 1);
         const int32_t b2 = __shfl_sync(kFull, bnd, 2), b3 = __shfl_sync(kFull, bnd, 3);
         const int32_t b4 = __shfl_sync(kFull, bnd, 4);
-        bnd = bounds(g + nwarps);
+        const uint8_t *__restrict__ col = jb.col;
+        const float *__restrict__ val = jb.val;
+        float *__restrict__ x = jb.x;
+        const int64_t n = jb.n;
+        const int64_t gn = g + nwarps;
+        const int jn = gn < groups ? job_of(gn, jc) : jc;
+        bnd = bounds(gn, jn);
         // zero the 4-row buffer
         float4 *b4p = reinterpret_cast<float4 *>(buf);
 #pragma unroll
@@ -543,6 +617,7 @@ ssdc_decode_kernel(const int32_t *__restrict__ row_end, const uint8_t *__restric
                 if (base + j < n) x[base + j] = buf[j];
         }
         __syncwarp();
+        jc = jn;
     }
 }
 
@@ -568,31 +643,97 @@ cudaError_t launch_ssdc_workspace_init(void *workspace, size_t bytes, cudaStream
     return cudaPeekAtLastError();
 }
 
+int64_t ssdc_tiles(int64_t n) { return (((n + kRow - 1) / kRow) + kTileRows - 1) / kTileRows; }
+
+size_t ssdc_workspace_bytes_many(const gist_ssdc_job *jobs, int32_t count) {
+    int64_t tiles = 0;
+    for (int32_t k = 0; k < count; ++k) tiles += ssdc_tiles(jobs[k].n);
+    return 4 * (size_t)kTotOffset + 8 * (size_t)tiles;
+}
+
+// Every map of the call in one persistent launch per kMaxEncJobs maps (launches share the
+// workspace in stream order; each leaves it ready for the next).  Maps with n == 0 only publish
+// *nnz (= *offset or 0) through a one-job launch of zero tiles... they are filtered by the caller.
+cudaError_t launch_ssdc_encode_many(const gist_ssdc_job *jobs, int32_t count, void *workspace, cudaStream_t s,
+                                    int *launches) {
+    static PerDeviceAttr attr;
+    const cudaError_t ea = attr.ensure(reinterpret_cast<const void *>(ssdc_encode_kernel), (int)sizeof(EncSmem));
+    if (ea != cudaSuccess) return ea;
+    *launches = 0;
+    for (int32_t k0 = 0; k0 < count; k0 += kMaxEncJobs) {
+        EncJobs J{};
+        J.count = 0;
+        int64_t tiles = 0;
+        for (int32_t k = k0; k < count && k < k0 + kMaxEncJobs; ++k) {
+            EncJob &e = J.j[J.count++];
+            e.x = jobs[k].x;
+            e.row_end = jobs[k].row_end;
+            e.col = jobs[k].col;
+            e.val = jobs[k].val;
+            e.nnz = jobs[k].nnz;
+            e.base = jobs[k].offset;
+            e.n = jobs[k].n;
+            e.capacity = jobs[k].capacity;
+            e.tile0 = tiles;
+            // chained: this map's entries follow the previous map's in the same arena
+            const bool chained = k > k0 && jobs[k].offset && jobs[k].offset == jobs[k - 1].nnz;
+            e.head = chained ? J.j[J.count - 2].head : J.count - 1;
+            tiles += ssdc_tiles(jobs[k].n);
+        }
+        J.tiles = tiles;
+        // A tile's offset waits for the totals of all earlier tiles of its map, claimed in ticket
+        // order by running CTAs: one persistent CTA per SM (the shared-memory ring allows no more).
+        const int64_t grid = tiles < num_sms() ? tiles : num_sms();
+        launch_k(ssdc_encode_kernel, (unsigned)grid, kEncThreads, sizeof(EncSmem), s, J,
+                 reinterpret_cast<uint32_t *>(workspace));
+        const cudaError_t e = cudaPeekAtLastError();
+        if (e != cudaSuccess) return e;
+        ++*launches;
+    }
+    return cudaSuccess;
+}
+
 cudaError_t launch_ssdc_encode(const float *x, int64_t n, int32_t *row_end, uint8_t *col, float *val,
                                int64_t capacity, int64_t *nnz, void *workspace, cudaStream_t s) {
-    const int64_t rows = (n + kRow - 1) / kRow;
-    // A tile's offset waits for the totals of all earlier tiles, claimed in ticket order by
-    // running CTAs: one persistent CTA per SM (the shared-memory ring allows no more).
-    static std::once_flag attr_once;
-    std::call_once(attr_once, [] {
-        cudaFuncSetAttribute(ssdc_encode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(EncSmem));
-    });
-    const int64_t tiles = (rows + kTileRows - 1) / kTileRows;
-    const int64_t grid = tiles < num_sms() ? tiles : num_sms();
-    launch_k(ssdc_encode_kernel, (unsigned)grid, kEncThreads, sizeof(EncSmem), s, 
-        x, n, rows, tiles, row_end, col, val, capacity, nnz, reinterpret_cast<uint32_t *>(workspace));
-    return cudaPeekAtLastError();
+    gist_ssdc_job job{x, n, row_end, col, val, capacity, nnz, nullptr};
+    int launches = 0;
+    return launch_ssdc_encode_many(&job, 1, workspace, s, &launches);
+}
+
+cudaError_t launch_ssdc_decode_many(const gist_ssdc_decode_job *jobs, int32_t count, cudaStream_t s, int *launches) {
+    *launches = 0;
+    for (int32_t k0 = 0; k0 < count; k0 += kMaxDecJobs) {
+        DecJobs J{};
+        int64_t groups = 0;
+        for (int32_t k = k0; k < count && k < k0 + kMaxDecJobs; ++k) {
+            DecJob &e = J.j[J.count++];
+            e.row_end = jobs[k].row_end;
+            e.col = jobs[k].col;
+            e.val = jobs[k].val;
+            e.base = jobs[k].offset;
+            e.x = jobs[k].x;
+            e.n = jobs[k].n;
+            e.g0 = groups;
+            groups += ((jobs[k].n + kRow - 1) / kRow + kDecRows - 1) / kDecRows;
+        }
+        J.groups = groups;
+        int64_t blocks = ceil_div(groups, kDecThreads / 32);
+        const int64_t cap = (int64_t)num_sms() * GIST_SSDC_DEC_CTAS;
+        if (blocks > cap) blocks = cap;
+        if (blocks < 1) blocks = 1;
+        launch_k(ssdc_decode_kernel, (unsigned)blocks, kDecThreads, 0, s, J);
+        const cudaError_t e = cudaPeekAtLastError();
+        if (e != cudaSuccess) return e;
+        ++*launches;
+    }
+    return cudaSuccess;
 }
 
 cudaError_t launch_ssdc_decode(const int32_t *row_end, const uint8_t *col, const float *val, int64_t n, float *x,
                                cudaStream_t s) {
-    const int64_t rows = (n + kRow - 1) / kRow;
-    const int64_t groups = (rows + kDecRows - 1) / kDecRows;
-    int64_t blocks = ceil_div(groups, kDecThreads / 32);
-    const int64_t cap = (int64_t)num_sms() * GIST_SSDC_DEC_CTAS;
-    if (blocks > cap) blocks = cap;
-    launch_k(ssdc_decode_kernel, (unsigned)blocks, kDecThreads, 0, s, row_end, col, val, n, rows, x);
-    return cudaPeekAtLastError();
+    gist_ssdc_decode_job job{row_end, col, val, nullptr, n, x};
+    int launches = 0;
+    return launch_ssdc_decode_many(&job, 1, s, &launches);
 }
 
 }  // namespace gist

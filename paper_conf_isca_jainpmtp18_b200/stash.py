@@ -101,8 +101,8 @@ class _StashedConv(torch.autograd.Function):
         gx, gw, gb = torch.ops.aten.convolution_backward(
             dout.contiguous(), y, weight, [weight.shape[0]] if has_bias else None, stride, padding, dilation, False,
             [0, 0], groups, [True, True, has_bias])
-        if relu:
-            gx.masked_fill_(y == 0, 0.0)  # ReLU backward: y = relu(x) is 0 exactly where x <= 0
+        if relu:  # ReLU backward with torch's own rule (threshold_backward on the ReLU output)
+            gx = torch.ops.aten.threshold_backward(gx, y, 0)
         del y
         return gx, gw, gb, None, None, None, None, None
 

@@ -10,7 +10,9 @@ import workloads as WL  # noqa: E402
 
 dev = torch.device("cuda:0")
 for g, shape in [(WL.P2S2, (2, 8, 16, 16)), (WL.P2S2, (1, 3, 14, 14)), (WL.P3S2, (2, 4, 13, 13)),
-                 (WL.P3S2C, (1, 4, 12, 12)), (WL.P3S1P1, (1, 4, 9, 9))]:
+                 (WL.P3S2C, (1, 4, 12, 12)), (WL.P3S1P1, (1, 4, 9, 9)),
+                 # odd W with n % 32 == 0: the last 2x2 block of the 3x3/s2 backward sits on element n - 1
+                 (WL.P3S2, (1, 32, 13, 13)), (WL.P3S2C, (1, 32, 13, 13))]:
     y = WL.relu_map(shape, 0.5, 1, dev)
     out, arg, mask = gist.gist_maxpool_fwd_argmax(y, g, fuse_mask=True)
     gist.gist_pool_relu_bwd(torch.randn_like(out), arg, mask, shape, g)

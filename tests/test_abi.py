@@ -122,3 +122,53 @@ def test_validation_without_gpu(gist):
     assert L.gist_ssdc_dpr_encode(A, B, 100, 12, B + 64, None) == UNSUPPORTED
     assert L.gist_ssdc_dpr_encode(A, None, 100, 8, B + 64, None) == INVALID
     assert L.gist_ssdc_dpr_decode(A, B + 4, 100, 8, B + 64, None) == MISALIGNED
+
+
+def test_pool_geometry_overflow_rejected(gist):
+    """A window whose kh*kw wraps in int32 (kh=3, kw=1431655766 -> 2 mod 2^32) must not pass the
+    4-bit argmax check; huge padded spans must not wrap either."""
+    L = gist.lib
+    P = gist.Pool2d
+    g = P(3, 1431655766, 1, 1, 0, 715827883, 0)
+    assert L.gist_maxpool_fwd_argmax(A, 1, 1, 4, 1, C.byref(g), B, B + 4096, None, None) == UNSUPPORTED
+    assert L.gist_pool_relu_bwd(A, B, None, 1, 1, 4, 1, C.byref(g), B + 4096, None) == UNSUPPORTED
+    g = P(17, 1, 1, 1, 0, 0, 0)
+    assert L.gist_maxpool_fwd_argmax(A, 1, 1, 32, 32, C.byref(g), B, B + 4096, None, None) == UNSUPPORTED
+    Ho, Wo = C.c_int32(), C.c_int32()
+    g = P(3, 3, 1, 1, 1, 1, 0)
+    assert L.gist_pool2d_out_dims(2**31 - 1, 8, C.byref(g), C.byref(Ho), C.byref(Wo)) == OK
+    assert Ho.value == 2**31 - 1 and Wo.value == 8  # (H + 2 - 3)/1 + 1 computed without wrapping
+
+
+def test_binding_rejects_wrong_dtypes_and_devices(gist):
+    """The C ABI sees raw pointers only; the binding checks dtype, device and size before the call
+    (a bf16 map read as fp32 would run 2x past its buffer)."""
+    import torch
+    with pytest.raises(ValueError):
+        gist._ptr(torch.zeros(4), gist._F32, name="y")  # CPU tensor: no fallback
+    meta = torch.empty(8, dtype=torch.bfloat16, device="meta")
+    with pytest.raises(ValueError):
+        gist._ptr(meta, gist._F32, name="y")
+
+
+def test_many_calls_validation_without_gpu(gist):
+    L = gist.lib
+    J = gist.SsdcJob
+    assert L.gist_ssdc_encode_many(None, 0, None, 0, None) == OK
+    assert L.gist_ssdc_encode_many(None, 1, None, 0, None) == INVALID
+    assert L.gist_ssdc_decode_many(None, 0, None) == OK
+    assert L.gist_dpr_encode_many(None, 0, 16, None) == OK
+    assert L.gist_dpr_encode_many(None, 0, 12, None) == UNSUPPORTED
+    jobs = (J * 2)()
+    jobs[0] = J(A, 1024, B, B + 4096, B + 8192, 1024, B + 16384, None)
+    jobs[1] = J(A + 4, 1024, B + 32768, B + 36864, B + 40960, 1024, B + 49152, None)  # misaligned x
+    ws = gist.lib.gist_ssdc_workspace_bytes_many(jobs, 2)
+    assert ws == 128 + 8 * 2
+    assert L.gist_ssdc_encode_many(jobs, 2, B + (1 << 20), ws, None) == MISALIGNED
+    jobs[1] = J(A + 8192, 1024, B + 32768, B + 36864, B + 40960, 1024, B + 49152, B + 16384)  # chained: ok so far
+    assert L.gist_ssdc_encode_many(jobs, 2, B + (1 << 20), 8, None) == INVALID  # workspace too small
+    jobs[1] = J(A + 8192, 1024, B + 32768, B + 36864, B + 40960, 1024, B + 49152, B + 49152)  # own nnz
+    assert L.gist_ssdc_encode_many(jobs, 2, B + (1 << 20), ws, None) == INVALID
+    D = gist.DprJob
+    dj = (D * 1)(D(A, 100, A + 16))  # overlapping in/out
+    assert L.gist_dpr_encode_many(dj, 1, 16, None) == INVALID

@@ -413,3 +413,114 @@ def test_ssdc_values_dpr(gist, ref, cuda, bits, n):
     dense = gist.gist_ssdc_decode(row_end, col, back[:max(k, 1)], n)
     expect = ref.ssdc_decode(r_row_end, r_col, ref.dpr_decode(r_packed, k, bits), n)
     assert_bits_equal(host(dense), expect, "ssdc_decode(dpr^-1(dpr(val)))")
+
+
+# ------------------------------------------------------------------------ full-size code paths (round 2)
+def test_full_size_dpr_decode_all_widths(gist, ref, cuda):
+    """a7 at the bench's full size (VGG16 relu1_1 b64, 205.5 M values): the unrolled multi-group
+    decode loops (u >= 1) and the FP10 multi-pass chunk loop, element by element vs the oracle."""
+    s = _vgg_site("relu1_1")
+    x = WL.dpr_map((64,) + s.chw, 3_000_000 + 7, cuda)
+    sp = WL.dpr_specials().to(cuda)
+    x.view(-1)[: sp.numel()] = sp
+    xh = host(x).reshape(-1)
+    n = x.numel()
+    for bits in (16, 10, 8):
+        packed = gist.gist_dpr_encode(x, bits)
+        r_packed = ref.dpr_encode(xh, bits)
+        assert_bits_equal(host(packed), r_packed, f"fp{bits} packed")
+        back = gist.gist_dpr_decode(packed, n, bits)
+        assert_bits_equal(host(back), ref.dpr_decode(r_packed, n, bits), f"fp{bits} decode")
+        del packed, back, r_packed
+
+
+FULL_3X3 = [("alexnet", "relu1", 128), ("nin", "relu_cccp2", 256), ("googlenet", "relu_conv1", 64),
+            ("alexnet", "relu5", 128), ("googlenet", "inc3b_out", 64)]
+
+
+@pytest.mark.parametrize("net,site,batch", FULL_3X3, ids=lambda v: str(v))
+def test_full_size_3x3_pools(gist, ref, cuda, net, site, batch):
+    """3x3/s2 floor (AlexNet) and ceil (NiN, GoogLeNet) at the configs' full batch: the generic
+    forward and the 3x3/s2 block backward run their grid-stride loops past one pass of the capped
+    grid.  Forward with and without the mask, backward with the mask and pool-only."""
+    s = next(t for t in WL.NETS[net] if t.name == site)
+    shape = (batch,) + s.chw
+    y = WL.relu_map(shape, 0.5, 4_000_000 + batch, cuda)
+    out, arg, mask = gist.gist_maxpool_fwd_argmax(y, s.pool, fuse_mask=True)
+    out2, arg2, _ = gist.gist_maxpool_fwd_argmax(y, s.pool)
+    assert torch.equal(out, out2) and torch.equal(arg, arg2)
+    yh = host(y)
+    r_out, r_arg = ref.maxpool_fwd_argmax(yh, s.pool)
+    r_mask = ref.binarize_encode(yh)
+    del yh
+    assert_bits_equal(host(out), r_out, "out")
+    assert_bits_equal(host(arg), r_arg, "argmax")
+    assert_bits_equal(host(mask), r_mask, "mask")
+    dout = WL.grad_map(tuple(out.shape), 19, cuda)
+    dh = host(dout)
+    for m, rm in ((mask, r_mask), (None, None)):
+        dx = gist.gist_pool_relu_bwd(dout, arg, m, shape, s.pool)
+        assert_bits_equal(host(dx), ref.pool_relu_bwd(dh, r_arg, rm, shape, s.pool),
+                          "dx" + (" (pool-only)" if m is None else ""))
+        del dx
+
+
+def test_full_size_2x2_pair_kernels_without_mask(gist, ref, cuda):
+    """The 2x2/s2 pair forward (no mask requested) and the pool-only pair backward at the C3 size."""
+    s = _vgg_site("relu1_2")
+    shape = (64,) + s.chw
+    y = WL.relu_map(shape, 0.8, 3_000_000 + 11, cuda)
+    out, arg, mask = gist.gist_maxpool_fwd_argmax(y, s.pool)
+    assert mask is None
+    r_out, r_arg = ref.maxpool_fwd_argmax(host(y), s.pool)
+    assert_bits_equal(host(out), r_out, "out")
+    assert_bits_equal(host(arg), r_arg, "argmax")
+    dout = WL.grad_map(tuple(out.shape), 23, cuda)
+    dx = gist.gist_pool_relu_bwd(dout, arg, None, shape, s.pool)
+    assert_bits_equal(host(dx), ref.pool_relu_bwd(host(dout), r_arg, None, shape, s.pool), "dx (pool-only)")
+
+
+@pytest.mark.parametrize("g", GEOMS, ids=gid)
+@pytest.mark.parametrize("shape", [(2, 3, 13, 13), (1, 64, 56, 56), (3, 7, 28, 28), (1, 1, 2, 2050)],
+                         ids=lambda s: "x".join(map(str, s)))
+def test_relu_maxpool_then_fused_bwd(gist, ref, cuda, g, shape):
+    """f3 -> a3: the backward fed by the in-place-ReLU forward's argmax and mask equals the
+    oracle's backward of relu(x), and torch CPU autograd of relu -> max_pool2d where torch
+    supports the geometry (the f3 docstring's promise)."""
+    N, Cc, H, W = shape
+    if H + 2 * g[4] < g[0] or W + 2 * g[5] < g[1]:
+        pytest.skip("window larger than padded input")
+    gen = torch.Generator(device=cuda).manual_seed(sum(shape) + 29)
+    x = torch.round(torch.randn(shape, device=cuda, generator=gen) * 2) / 2
+    out, arg, mask = gist.gist_relu_maxpool_fwd_argmax(x, g)
+    y = torch.relu(x.cpu()).numpy()
+    r_out, r_arg = ref.maxpool_fwd_argmax(y, g)
+    r_mask = ref.binarize_encode(y)
+    dout = WL.grad_map(tuple(out.shape), 31, cuda)
+    dx = gist.gist_pool_relu_bwd(dout, arg, mask, shape, g)
+    r_dx = ref.pool_relu_bwd(host(dout), r_arg, r_mask, shape, g)
+    assert_bits_equal(host(dx), r_dx, "dx from f3 encodings")
+    kh, kw, sh, sw, ph, pw, cm = g
+    xc = x.cpu().requires_grad_()
+    oc = torch.nn.functional.max_pool2d(torch.relu(xc), (kh, kw), (sh, sw), (ph, pw), ceil_mode=bool(cm))
+    oc.backward(dout.cpu())
+    assert_bits_equal(host(out), oc.detach().numpy(), "out vs torch")
+    assert_bits_equal(host(dx), xc.grad.numpy(), "dx vs torch autograd")
+
+
+def test_binding_checks_dtype_device_and_size(gist, cuda):
+    """a bf16 map (autocast) read as fp32 would overrun its buffer; the binding refuses it."""
+    y16 = torch.zeros(64, 16, 16, device=cuda, dtype=torch.bfloat16).view(1, 64, 16, 16)
+    with pytest.raises(ValueError):
+        gist.gist_binarize_encode(y16)
+    with pytest.raises(ValueError):
+        gist.gist_maxpool_fwd_argmax(y16, (2, 2, 2, 2, 0, 0, 0))
+    with pytest.raises(ValueError):
+        gist.gist_ssdc_encode(y16)
+    with pytest.raises(ValueError):
+        gist.gist_dpr_encode(y16, 16)
+    y = torch.zeros(1, 64, 16, 16, device=cuda)
+    with pytest.raises(ValueError):  # mask too small
+        gist.gist_maxpool_fwd_argmax(y, (2, 2, 2, 2, 0, 0, 0), mask=torch.zeros(3, dtype=torch.int32, device=cuda))
+    with pytest.raises(ValueError):  # float argmax words
+        gist.gist_maxpool_fwd_argmax(y, (2, 2, 2, 2, 0, 0, 0), argmax=torch.zeros(1024, device=cuda))

@@ -1,0 +1,26 @@
+"""compute-sanitizer as a test target: memcheck and synccheck over every kernel on
+small ragged shapes (scripts/sanitize.py), including the odd-W / n % 32 == 0 pool shapes where
+a mask read one word past the buffer was possible.  racecheck is run by scripts/gpu_sanitize.sh;
+its only reports are the SSDC encoder's mbarrier-ordered role hand-offs."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "synccheck"])
+def test_compute_sanitizer_clean(gist, cuda, tool):
+    cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+    if not os.path.exists(cs):
+        pytest.skip("compute-sanitizer not installed")
+    r = subprocess.run([cs, "--tool", tool, "--error-exitcode", "9", sys.executable,
+                        os.path.join(ROOT, "scripts", "sanitize.py")],
+                       capture_output=True, text=True, timeout=900, cwd=ROOT)
+    tail = (r.stdout + r.stderr)[-3000:]
+    assert r.returncode == 0, tail
+    assert "ERROR SUMMARY: 0 errors" in r.stdout + r.stderr, tail

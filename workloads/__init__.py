@@ -193,6 +193,24 @@ def seed_for(config_index: int, site_index: int, rank: int = 0) -> int:
     return 1_000_000 * config_index + 1000 * site_index + rank
 
 
+def image_seed(config_index: int, site_index: int, image: int, grad: bool = False) -> int:
+    """Per-image seed: 1_000_000*config + 1000*site + image (+500 for the upstream
+    gradient).  Inputs are drawn image by image from GLOBAL image indices, so the union of the
+    ranks' minibatch shards is exactly the single-GPU minibatch (C4 strong scaling)."""
+    if not 0 <= image < 500:
+        raise ValueError("image index must be in [0, 500)")
+    return 1_000_000 * config_index + 1000 * site_index + (500 if grad else 0) + image
+
+
+def per_image(fn, chw, images, seed0: int, device="cpu", **kw) -> torch.Tensor:
+    """Stack fn((1,) + chw, seed0 + image, device, **kw) over the global image indices `images`."""
+    images = list(images)
+    out = torch.empty((len(images),) + tuple(chw), dtype=torch.float32, device=device)
+    for k, img in enumerate(images):
+        out[k:k + 1] = fn((1,) + tuple(chw), seed0 + img, device, **kw)
+    return out
+
+
 def _gen(seed: int, device) -> torch.Generator:
     g = torch.Generator(device=device)
     g.manual_seed(seed)
