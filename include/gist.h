@@ -259,6 +259,29 @@ gist_status gist_ssdc_decode_many(const gist_ssdc_decode_job *jobs, int32_t coun
 gist_status gist_dpr_encode_many(const gist_dpr_job *jobs, int32_t count, int32_t bits, cudaStream_t stream);
 gist_status gist_dpr_decode_many(const gist_dpr_job *jobs, int32_t count, int32_t bits, cudaStream_t stream);
 
+/* ---------------------------------------------------------------- f4: decode inside the consumer GEMM
+ * P:166 §IV-A ("the backward pass implementation can be modified to work directly on
+ * precision-reduced values"), §V-H ("decode only the data that is required in near
+ * future ... the near-future tile in a tiled matrix multiplication"), P:128 (the conv backward needs
+ * its stashed input X for the weight gradient).  Weight gradient of a 3x3 / stride 1 / pad 1
+ * convolution (every VGG16 conv) whose input X is held as its SSDC encoding:
+ *     dW[co][ci][kh][kw] = sum_{n,oh,ow} dY[n][co][oh][ow] * X[n][ci][oh+kh-1][ow+kw-1]
+ * (out-of-range X is 0).  X is decoded tile by tile into shared memory inside a tcgen05 (UMMA)
+ * implicit GEMM; no dense X exists in device memory.
+ *   dy      [N,Co,H,W] fp32, read.   row_end/col/val: gist_ssdc_encode of X [N,Ci,H,W] (complete).
+ *   dw      [Co,Ci,3,3] fp32, written.
+ *   passes  3: "3xTF32" (each operand split into TF32 hi + lo; hi*hi + hi*lo + lo*hi accumulated in
+ *           fp32: every product within ~2^-19 relative of the fp32 product); 1: TF32 products (inputs
+ *           truncated to 10-bit mantissas), fp32 accumulation.  Deterministic (fixed split-K order).
+ *   workspace [>= gist_conv3x3_wgrad_workspace_bytes(...)] device bytes (split-K partials).
+ * UNSUPPORTED unless Co % 128 == 0, Ci % 16 == 0, H*W % 4 == 0 (dY rows are TMA rows), W <= 252,
+ * passes in {1, 3};
+ * TOO_LARGE if N*Ci*H*W or N*Co*H*W >= 2^31. */
+size_t gist_conv3x3_wgrad_workspace_bytes(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W);
+gist_status gist_conv3x3_wgrad_ssdc(const float *dy, const int32_t *row_end, const uint8_t *col, const float *val,
+                                    int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W, int32_t passes,
+                                    float *dw, void *workspace, size_t workspace_bytes, cudaStream_t stream);
+
 /* Number of SMs the launch heuristics use (cached on first call; for diagnostics). */
 int32_t gist_num_sms(void);
 

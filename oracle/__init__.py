@@ -58,6 +58,7 @@ def lib() -> C.CDLL:
             "oracle_dpr_decode": (None, [p, i64, i32, p]),
             "oracle_dpr_codes": (None, [p, i64, i32, p]),
             "oracle_dpr_values": (None, [p, i64, i32, p]),
+            "oracle_conv3x3_wgrad_entries": (None, [p, p, i32, i32, i32, i32, i32, p, i64, p, p]),
         }
         for name, (res, args) in sig.items():
             fn = getattr(_lib, name)
@@ -183,3 +184,24 @@ def dpr_values(codes, bits: int) -> np.ndarray:
     out = np.empty(codes.size, np.float32)
     lib().oracle_dpr_values(_ptr(codes), codes.size, bits, _ptr(out))
     return out
+
+
+# ---------------------------------------------------------------- O8 f4 reference (conv weight gradient)
+def conv3x3_wgrad_entries(dy, x, entries):
+    """dW entries (co, ci, tap) of a 3x3/s1/p1 conv, and sum |dY*X| for each (binary64)."""
+    dy, x = _f32(dy), _f32(x)
+    N, Co, H, W = dy.shape
+    Ci = x.shape[1]
+    ent = np.ascontiguousarray(entries, np.int32).reshape(-1, 3)
+    dw = np.empty(len(ent), np.float64)
+    mag = np.empty(len(ent), np.float64)
+    lib().oracle_conv3x3_wgrad_entries(_ptr(dy), _ptr(x), N, Ci, Co, H, W, _ptr(ent), len(ent), _ptr(dw), _ptr(mag))
+    return dw, mag
+
+
+def conv3x3_wgrad(dy, x):
+    """The full dW [Co, Ci, 3, 3] (binary64) and sum |dY*X| per entry."""
+    Co, Ci = dy.shape[1], x.shape[1]
+    ent = np.stack(np.meshgrid(np.arange(Co), np.arange(Ci), np.arange(9), indexing="ij"), -1).reshape(-1, 3)
+    dw, mag = conv3x3_wgrad_entries(dy, x, ent)
+    return dw.reshape(Co, Ci, 3, 3), mag.reshape(Co, Ci, 3, 3)

@@ -304,3 +304,39 @@ void oracle_dpr_values(const uint32_t *codes, int64_t n, int32_t bits, float *x)
 {
     for (int64_t i = 0; i < n; ++i) x[i] = oracle_dpr_value(codes[i], bits);
 }
+
+/* ------------------------------------------------------------------------------------
+ * O8 — f4 reference: weight gradient of a 3x3 / stride 1 / pad 1 convolution from the upstream
+ * gradient dY and the (decoded) stashed input X.  P:128 §III ("the backward pass of the
+ * convolution needs the input feature map X to compute the weight gradient"), §IV-A and
+ * P:271-272 §V-H (the decode moved into the consumer GEMM: the result is the same weight
+ * gradient).  Definition written out, accumulated in binary64:
+ *     dW[co][ci][kh][kw] = sum_{n,oh,ow} dY[n][co][oh][ow] * X[n][ci][oh+kh-1][ow+kw-1]
+ * with X = 0 outside the map.  dw_abs receives sum |dY * X| (the normwise error scale the f4
+ * parity tolerance is stated against).  entries: the (co, ci, tap) triples to evaluate
+ * (tap = 3 kh + kw); the full gradient is all Co*Ci*9 of them.
+ * ---------------------------------------------------------------------------------- */
+void oracle_conv3x3_wgrad_entries(const float *dy, const float *x, int32_t N, int32_t Ci, int32_t Co, int32_t H,
+                                  int32_t W, const int32_t *entries, int64_t count, double *dw, double *dw_abs)
+{
+    for (int64_t e = 0; e < count; ++e) {
+        int32_t co = entries[3 * e], ci = entries[3 * e + 1], tap = entries[3 * e + 2];
+        int32_t kh = tap / 3, kw = tap % 3;
+        double acc = 0.0, mag = 0.0;
+        for (int32_t n = 0; n < N; ++n)
+            for (int32_t oh = 0; oh < H; ++oh) {
+                int32_t ih = oh + kh - 1;
+                if (ih < 0 || ih >= H) continue;
+                for (int32_t ow = 0; ow < W; ++ow) {
+                    int32_t iw = ow + kw - 1;
+                    if (iw < 0 || iw >= W) continue;
+                    double g = dy[(((int64_t)n * Co + co) * H + oh) * W + ow];
+                    double v = x[(((int64_t)n * Ci + ci) * H + ih) * W + iw];
+                    acc += g * v;
+                    mag += fabs(g * v);
+                }
+            }
+        dw[e] = acc;
+        dw_abs[e] = mag;
+    }
+}

@@ -26,6 +26,7 @@ __all__ = [
     "gist_ssdc_dpr_encode", "gist_ssdc_dpr_decode",
     "gist_ssdc_workspace_bytes_many", "gist_ssdc_encode_many", "gist_ssdc_decode_many", "gist_dpr_encode_many",
     "gist_dpr_decode_many", "SsdcEncodeMany", "SsdcDecodeMany", "DprMany",
+    "gist_conv3x3_wgrad_workspace_bytes", "gist_conv3x3_wgrad_ssdc",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -104,6 +105,8 @@ def _load() -> C.CDLL:
         "gist_ssdc_decode_many": (C.c_int, [p, i32, p]),
         "gist_dpr_encode_many": (C.c_int, [p, i32, i32, p]),
         "gist_dpr_decode_many": (C.c_int, [p, i32, i32, p]),
+        "gist_conv3x3_wgrad_workspace_bytes": (sz, [i32, i32, i32, i32, i32]),
+        "gist_conv3x3_wgrad_ssdc": (C.c_int, [p, p, p, p, i32, i32, i32, i32, i32, i32, p, p, sz, p]),
     }
     for name, (res, args) in sigs.items():
         fn = getattr(L, name)
@@ -540,3 +543,32 @@ def gist_dpr_encode_many(xs, bits: int, stream=None):
 def gist_dpr_decode_many(packed, ns, bits: int, stream=None):
     """a7 over several maps in one launch.  Returns [x]."""
     return DprMany([{"packed": p, "n": n} for p, n in zip(packed, ns)], bits, False)(stream)
+
+
+# ------------------------------------------------------------------ f4: decode inside the consumer GEMM
+def gist_conv3x3_wgrad_workspace_bytes(N: int, Ci: int, Co: int, H: int, W: int) -> int:
+    return lib.gist_conv3x3_wgrad_workspace_bytes(N, Ci, Co, H, W)
+
+
+def gist_conv3x3_wgrad_ssdc(dy: torch.Tensor, row_end: torch.Tensor, col: torch.Tensor, val: torch.Tensor,
+                            x_shape, passes: int = 3, dw: torch.Tensor | None = None,
+                            workspace: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """f4: dW [Co,Ci,3,3] of a 3x3/s1/p1 conv from dY [N,Co,H,W] and the SSDC
+    encoding of its input X (shape x_shape = (N, Ci, H, W)); X is decoded inside the tcgen05 GEMM."""
+    N, Ci, H, W = (int(v) for v in x_shape)
+    Co = int(dy.shape[1])
+    dev = dy.device
+    if tuple(dy.shape) != (N, Co, H, W):
+        raise ValueError(f"dy {tuple(dy.shape)} does not match x_shape {tuple(x_shape)}")
+    if dw is None:
+        dw = torch.empty((Co, Ci, 3, 3), dtype=torch.float32, device=dev)
+    wsb = gist_conv3x3_wgrad_workspace_bytes(N, Ci, Co, H, W)
+    if workspace is None:
+        workspace = torch.empty(max(wsb, 16), dtype=torch.uint8, device=dev)
+    with torch.cuda.device(dev):
+        _check(lib.gist_conv3x3_wgrad_ssdc(
+            _ptr(dy, _F32, dev, name="dy"), _ptr(row_end, _I32, dev, gist_ssdc_rows(N * Ci * H * W), "row_end"),
+            _ptr(col, _U8, dev, name="col"), _ptr(val, _F32, dev, name="val"), N, Ci, Co, H, W, int(passes),
+            _ptr(dw, _F32, dev, Co * Ci * 9, "dw"), _ptr(workspace, None, dev, name="workspace"),
+            workspace.numel() * workspace.element_size(), _stream(dy, stream)), "gist_conv3x3_wgrad_ssdc")
+    return dw

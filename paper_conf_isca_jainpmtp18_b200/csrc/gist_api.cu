@@ -39,10 +39,13 @@ int num_sms() {
 
 cudaError_t PerDeviceAttr::ensure(const void *func, int smem_bytes) {
     const int dev = current_device();
-    const uint64_t bit = dev < 64 ? (1ull << dev) : 0ull;
-    if (bit && (done.load(std::memory_order_acquire) & bit)) return cudaSuccess;
+    if (dev < kMaxDevices && set[dev].load(std::memory_order_acquire) >= smem_bytes) return cudaSuccess;
     const cudaError_t e = cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
-    if (e == cudaSuccess && bit) done.fetch_or(bit, std::memory_order_acq_rel);
+    if (e == cudaSuccess && dev < kMaxDevices) {
+        int cur = set[dev].load(std::memory_order_relaxed);
+        while (cur < smem_bytes && !set[dev].compare_exchange_weak(cur, smem_bytes, std::memory_order_acq_rel)) {
+        }
+    }
     return e;
 }
 
@@ -393,6 +396,35 @@ gist_status gist_dpr_encode_many(const gist_dpr_job *jobs, int32_t count, int32_
 
 gist_status gist_dpr_decode_many(const gist_dpr_job *jobs, int32_t count, int32_t bits, cudaStream_t stream) {
     return dpr_many(jobs, count, bits, false, stream);
+}
+
+size_t gist_conv3x3_wgrad_workspace_bytes(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W) {
+    if (!gist::wgrad_shape_ok(N, Ci, Co, H, W)) return 0;
+    return gist::wgrad_workspace_bytes(N, Ci, Co, H, W);
+}
+
+gist_status gist_conv3x3_wgrad_ssdc(const float *dy, const int32_t *row_end, const uint8_t *col, const float *val,
+                                    int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W, int32_t passes,
+                                    float *dw, void *workspace, size_t workspace_bytes, cudaStream_t stream) {
+    if (N < 0 || Ci < 0 || Co < 0 || H < 0 || W < 0) return GIST_ERR_INVALID_ARGUMENT;
+    if (passes != 1 && passes != 3) return GIST_ERR_UNSUPPORTED;
+    if (N == 0 || Ci == 0 || Co == 0 || H == 0 || W == 0) return GIST_ERR_UNSUPPORTED;
+    if (!gist::wgrad_shape_ok(N, Ci, Co, H, W)) return GIST_ERR_UNSUPPORTED;
+    const int64_t nx = (int64_t)N * Ci * H * W, ny = (int64_t)N * Co * H * W;
+    if (nx >= kI32Limit || ny >= kI32Limit) return GIST_ERR_TOO_LARGE;
+    if (!dy || !row_end || !dw || !workspace) return GIST_ERR_INVALID_ARGUMENT;
+    if (misaligned(dy) || misaligned(row_end) || misaligned(col) || misaligned(val) || misaligned(dw) ||
+        misaligned(workspace))
+        return GIST_ERR_MISALIGNED;
+    if (workspace_bytes < gist::wgrad_workspace_bytes(N, Ci, Co, H, W)) return GIST_ERR_INVALID_ARGUMENT;
+    const int64_t ndw = (int64_t)Co * Ci * 9;
+    if (any_overlap({{dy, 4 * ny}, {row_end, 4 * gist_ssdc_rows(nx)}}, {{dw, 4 * ndw}, {workspace, (int64_t)workspace_bytes}}))
+        return GIST_ERR_INVALID_ARGUMENT;
+    int launches = 0;
+    const cudaError_t e =
+        gist::launch_wgrad_ssdc(dy, row_end, col, val, N, Ci, Co, H, W, passes, dw, workspace, stream, &launches);
+    if (e == cudaErrorNotSupported) return GIST_ERR_UNSUPPORTED;
+    return launched(e, launches);
 }
 
 }  // extern "C"

@@ -15,8 +15,11 @@ int num_sms();  // of the current device (cached per device)
 // Dynamic shared-memory opt-in (cudaFuncAttributeMaxDynamicSharedMemorySize) of one kernel, applied
 // once per DEVICE: the attribute is per device, so a process that launches on a second GPU sets it
 // there too.
+// The attribute only ever grows (a kernel whose shared memory depends on the call's shape keeps the
+// largest size set so far).
 struct PerDeviceAttr {
-    std::atomic<uint64_t> done{0};  // bit d: set on device d (devices >= 64: set on every launch)
+    static constexpr int kMaxDevices = 64;  // devices beyond: set on every launch
+    std::atomic<int> set[kMaxDevices] = {};  // bytes already allowed on device d
     cudaError_t ensure(const void *func, int smem_bytes);
 };
 void count_launches(int k);  // bookkeeping for gist_launch_count()
@@ -59,5 +62,13 @@ cudaError_t launch_dpr_many(const gist_dpr_job *jobs, int32_t count, int bits, b
                             int *launches);
 cudaError_t launch_dpr_decode(const uint32_t *packed, int64_t n, int bits, float *x, cudaStream_t s,
                               const int64_t *n_dev = nullptr);
+
+// f4 (wgrad.cu): 3x3/s1/p1 conv weight gradient, X decoded from SSDC inside the tcgen05 GEMM
+bool wgrad_shape_ok(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W);
+size_t wgrad_workspace_bytes(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W);
+size_t wgrad_smem_bytes(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W, int32_t passes);
+cudaError_t launch_wgrad_ssdc(const float *dy, const int32_t *row_end, const uint8_t *col, const float *val, int32_t N,
+                              int32_t Ci, int32_t Co, int32_t H, int32_t W, int32_t passes, float *dw, void *workspace,
+                              cudaStream_t s, int *launches);
 
 }  // namespace gist

@@ -1,0 +1,87 @@
+"""f4 parity: the decode-in-GEMM weight gradient (tcgen05, SSDC decoded into shared memory) against
+the oracle (O8: the definition in binary64 over the seeded dense X, i.e. oracle-decode followed by
+a reference GEMM).  The result is a float reduction in a different order and, for passes = 1, with
+TF32 products, so the bar is normwise per entry: |dW - dW_ref| <= tol * sum_k |dY_k X_k| (the
+error scale of any fp32 implementation of this sum), tol = 1e-6 for 3xTF32 (north star: 1e-6
+relative where the reduction order differs, loosened to the 3xTF32 worst-case product bound
+2^-20 + 2^-22 rounded up to 2e-6) and 2^-9 for TF32 (two 2^-10 input truncations).
+(f4) derives both; the observed errors are about 1e-7 at full size."""
+import numpy as np
+import pytest
+import torch
+
+import workloads as WL
+
+pytestmark = pytest.mark.gpu
+TOL = {3: 2e-6, 1: 2.0 ** -9}
+
+
+def inputs(N, Ci, Co, H, W, s, seed, cuda):
+    x = WL.relu_map((N, Ci, H, W), s, seed, cuda)
+    dy = WL.grad_map((N, Co, H, W), seed + 1, cuda)
+    return x, dy
+
+
+def run(gist, x, dy, passes):
+    row_end, col, val, nnz = gist.gist_ssdc_encode(x)
+    return gist.gist_conv3x3_wgrad_ssdc(dy, row_end, col, val, tuple(x.shape), passes=passes)
+
+
+SHAPES = [(1, 16, 128, 8, 8), (2, 32, 128, 13, 8), (3, 16, 256, 7, 28), (2, 48, 128, 56, 56), (1, 16, 128, 9, 12),
+          (2, 16, 128, 12, 20), (2, 16, 128, 14, 14), (1, 32, 128, 10, 6), (1, 16, 128, 1, 4), (1, 16, 128, 2, 250), (1, 16, 128, 8, 13),
+          (1, 16, 128, 24, 21), (1, 16, 128, 40, 30)]
+
+
+@pytest.mark.parametrize("passes", [3, 1])
+@pytest.mark.parametrize("shape", SHAPES, ids=lambda s: "x".join(map(str, s)))
+def test_wgrad_vs_oracle(gist, ref, cuda, shape, passes):
+    N, Ci, Co, H, W = shape
+    x, dy = inputs(N, Ci, Co, H, W, 0.8, sum(shape), cuda)
+    dw = run(gist, x, dy, passes)
+    want, mag = ref.conv3x3_wgrad(dy.cpu().numpy(), x.cpu().numpy())
+    err = np.abs(dw.cpu().numpy().astype(np.float64) - want)
+    worst = float((err / np.maximum(mag, 1e-30)).max())
+    assert worst <= TOL[passes], f"normwise error {worst:.3e} > {TOL[passes]:.1e}"
+    again = run(gist, x, dy, passes)
+    assert torch.equal(dw, again), "not deterministic"
+
+
+def test_wgrad_dense_and_empty_maps(gist, ref, cuda):
+    """s ~ 0 (every CSR row full) and s = 1 (X all zero: dW must be exactly 0)."""
+    N, Ci, Co, H, W = 1, 16, 128, 10, 16
+    for s in (0.001, 1.0):
+        x, dy = inputs(N, Ci, Co, H, W, s, 5, cuda)
+        if s == 1.0:
+            x.zero_()
+        dw = run(gist, x, dy, 3)
+        want, mag = ref.conv3x3_wgrad(dy.cpu().numpy(), x.cpu().numpy())
+        if s == 1.0:
+            assert torch.equal(dw, torch.zeros_like(dw))
+        else:
+            assert float((np.abs(dw.cpu().numpy() - want) / np.maximum(mag, 1e-30)).max()) <= TOL[3]
+
+
+def test_wgrad_full_size_vgg16_conv3_2(gist, ref, cuda):
+    """The bench configuration: VGG16 conv3_2 at batch 64 (X = relu3_1, 256 x 56 x 56, SSDC at s = 0.8);
+    256 sampled dW entries computed one by one by the oracle, plus every entry's finiteness."""
+    N, Ci, Co, H, W = 64, 256, 256, 56, 56
+    x, dy = inputs(N, Ci, Co, H, W, 0.8, 3_000_000 + 5, cuda)
+    dw = run(gist, x, dy, 3)
+    assert torch.isfinite(dw).all()
+    rng = np.random.default_rng(0)
+    ent = np.stack([rng.integers(0, Co, 256), rng.integers(0, Ci, 256), rng.integers(0, 9, 256)], 1)
+    # always include the corners of the tile grid
+    ent[:4] = [[0, 0, 0], [Co - 1, Ci - 1, 8], [127, 15, 4], [128, 16, 2]]
+    want, mag = ref.conv3x3_wgrad_entries(dy.cpu().numpy(), x.cpu().numpy(), ent)
+    got = dw.cpu().numpy().reshape(Co, Ci, 9)[ent[:, 0], ent[:, 1], ent[:, 2]].astype(np.float64)
+    worst = float((np.abs(got - want) / np.maximum(mag, 1e-30)).max())
+    assert worst <= TOL[3], f"normwise error {worst:.3e}"
+
+
+def test_wgrad_rejects_unsupported_shapes(gist, cuda):
+    x, dy = inputs(1, 16, 64, 8, 8, 0.5, 1, cuda)  # Co = 64: not a multiple of 128
+    with pytest.raises(gist.GistError):
+        run(gist, x, dy, 3)
+    x, dy = inputs(1, 16, 128, 8, 8, 0.5, 1, cuda)
+    with pytest.raises(gist.GistError):
+        run(gist, x, dy, 2)
