@@ -49,17 +49,24 @@ struct FastDiv {
 };
 
 // Programmatic dependent launch (PDL): every libgist kernel is launched with programmatic
-// stream serialization and starts with pdl_enter(): it lets the next kernel in the stream be
-// scheduled at once (its CTAs' launch and prologue overlap this kernel's tail) and then waits
-// until the previous kernel has completed and its memory is visible (griddepcontrol.wait) before
-// touching global memory.  Stream order of the results is unchanged.  GIST_PDL=0 builds plain
-// <<<>>> launches (A/B knob).
+// stream serialization and starts with pdl_enter(), which waits until the previous kernel has
+// completed and its memory is visible (griddepcontrol.wait) before touching global memory.  No
+// kernel triggers its dependents early (GIST_PDL_EARLY=0): the next grid is launched as this
+// one's CTAs exit, so its launch overlaps only this kernel's drain.  An early trigger (at kernel
+// start) let the next grid's CTAs take SM slots from this grid's later waves and cost 5-16% per
+// step (C3 2.100 -> 1.815 ms, C5o 0.646 -> 0.547 ms, C4 1.997 -> 1.945 ms when removed; plain
+// launches, GIST_PDL=0: C3 1.849, C4 2.020).  Stream order of the results is unchanged.
 #ifndef GIST_PDL
 #define GIST_PDL 1
 #endif
+#ifndef GIST_PDL_EARLY
+#define GIST_PDL_EARLY 0
+#endif
 __device__ __forceinline__ void pdl_enter() {
 #if GIST_PDL
+#if GIST_PDL_EARLY
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+#endif
     asm volatile("griddepcontrol.wait;" ::: "memory");
 #endif
 }

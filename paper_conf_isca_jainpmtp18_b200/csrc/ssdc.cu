@@ -34,6 +34,7 @@
 #include "common.cuh"
 #include "kernels.h"
 #include "tma.cuh"
+#include "tcgen05.cuh"  // named_bar
 
 
 namespace gist {
@@ -73,7 +74,8 @@ constexpr int kStages = GIST_SSDC_STAGES;
 constexpr int kQ = GIST_SSDC_Q;
 constexpr int kProd = 0, kCount = 1, kPub = kCount + kParts, kGather = kPub + 1, kWriter0 = kGather + 1;
 constexpr int kEncThreads = 32 * (kWriter0 + kWriters);  // 23 warps = 736 threads
-constexpr int kStage = kWRows * kRow + 16;  // staged entries per writer warp (+ 16-entry phase)
+constexpr int kStage = kTileRows * kRow + 16;  // staged entries per tile (+ 16-entry phase)
+constexpr int kWriterThreads = 32 * kWriters;
 constexpr int kGatherPer = 8;                     // totals per lane per gather round (256 per warp)
 constexpr int kMaxEncJobs = 48;                   // maps per encode launch (job table in kernel params)
 // Workspace (zeroed once by the caller, left reusable by every call): u32 words ticket [0],
@@ -116,8 +118,8 @@ static_assert(sizeof(EncJobs) + 16 <= 4096, "kernel parameters must fit 4 KB");
 
 struct __align__(128) EncSmem {
     float raw[kStages][kPartElems];  // TMA ring (parts of tiles)
-    uint32_t vst[kWriters][kStage];  // per-writer compacted value bits (congruent to the output mod 4)
-    uint8_t cst[kWriters][kStage];   // per-writer compacted columns (bytes, same index)
+    uint32_t vst[2][kStage];         // compacted value bits of a tile (congruent to the output mod 16),
+    uint8_t cst[2][kStage];          // and its columns (bytes, same index); double-buffered by tile
     uint32_t rcnt[kQ][kTileRows];   // per-row nonzero counts
     uint32_t rinc[kQ][kTileRows];   // tile-local inclusive row ends
     int64_t base[kQ];                // global offset of the tile
@@ -150,29 +152,18 @@ __device__ __forceinline__ uint32_t nz4(const uint4 &a) {  // nonzero bit patter
     return min1(a.x) + min1(a.y) + min1(a.z) + min1(a.w);
 }
 
-// Writer: compact the rows held in lo/hi (queue slot q) to val/col.  The lane counts (0..8) of
-// both rows are scanned together (two 16-bit fields, one 5-step shuffle scan); then each lane's
-// nonzeros go to consecutive staging slots (value word and column byte at the same index).
-// The staging is congruent to the output mod 16 entries, so the whole 16-entry groups of val
-// (64 B) and col (16 B) leave as two 1-D bulk copies (cp.async.bulk shared -> global) issued
-// by lane 0; the ragged head and tail (< 16 entries each) by lanes 0..15 and 16..31.
-__device__ __forceinline__ void write_rows(EncSmem &S, int q, int w, int lane, const uint4 (&lo)[kWRows],
-                                           const uint4 (&hi)[kWRows], const EncJobs &J) {
-    const EncJob &jb = J.j[S.job[q]];
-    uint8_t *__restrict__ col = jb.col;
-    float *__restrict__ val = jb.val;
-    const int64_t capacity = jb.capacity;
+// Writer: stage the nonzeros of the rows held in lo/hi (queue slot q) into the tile's staging
+// buffer sb.  The lane counts (0..8) of both rows are scanned together (two 16-bit fields, one
+// 5-step shuffle scan); then each lane's nonzeros go to consecutive staging slots (value word and
+// column byte at the same index).  The staging index of output entry e is e - (tile base & ~15),
+// so after all writers have staged, the tile's whole 16-entry groups of val (64 B) and col (16 B)
+// leave as ONE pair of 1-D bulk copies (store_tile).
+__device__ __forceinline__ void stage_rows(EncSmem &S, int q, int sb, int w, int lane, const uint4 (&lo)[kWRows],
+                                           const uint4 (&hi)[kWRows]) {
     const int rw = w * kWRows;
-    const int64_t tile_base = S.base[q];
     const uint32_t w_excl = rw ? S.rinc[q][rw - 1] : 0u;
-    const uint32_t w_cnt = S.rinc[q][rw + kWRows - 1] - w_excl;
-    const int64_t off = tile_base + w_excl;
-    if (w_cnt == 0 || off >= capacity) return;
-    uint32_t *vs = S.vst[w];
-    uint8_t *cs = S.cst[w];
-    if (lane == 0) bulk_wait_read();  // the previous tile's bulk copies have read the staging
-    __syncwarp();
-    const uint32_t p = (uint32_t)(off & 15);
+    if (S.rinc[q][rw + kWRows - 1] == w_excl) return;  // no nonzeros in these rows
+    const uint32_t p = (uint32_t)(S.base[q] & 15) + w_excl;  // staging index of the writer's first entry
     // lane prefix of both rows' lane counts in one warp scan (16-bit fields: row counts <= 256)
     static_assert(kWRows == 2, "the packed scan carries two rows");
     const uint32_t cnt0 = nz4(lo[0]) + nz4(hi[0]), cnt1 = nz4(lo[1]) + nz4(hi[1]);
@@ -188,7 +179,7 @@ __device__ __forceinline__ void write_rows(EncSmem &S, int q, int w, int lane, c
     for (int r = 0; r < kWRows; ++r) {
         const uint32_t v[8] = {lo[r].x, lo[r].y, lo[r].z, lo[r].w, hi[r].x, hi[r].y, hi[r].z, hi[r].w};
         const uint32_t i = p + excl[r];
-        uint32_t addr = smem_u32(vs + i), caddr = smem_u32(cs + i);
+        uint32_t addr = smem_u32(S.vst[sb] + i), caddr = smem_u32(S.cst[sb] + i);
         const uint32_t c0 = 8u * lane;
 #pragma unroll
         for (int k = 0; k < 8; ++k) {
@@ -204,33 +195,41 @@ __device__ __forceinline__ void write_rows(EncSmem &S, int q, int w, int lane, c
                 : "memory");
         }
     }
-    const int64_t lim = (off + w_cnt < capacity) ? off + w_cnt : capacity;
+}
+
+// Writer warp 0, once every writer has staged the tile: the whole 16-entry groups leave as two
+// bulk copies issued by lane 0; the ragged head and tail (< 16 entries each) by lanes 0..15 and
+// 16..31.  Entries at or past the job's capacity are not written.
+__device__ __forceinline__ void store_tile(EncSmem &S, int q, int sb, int lane, const EncJobs &J) {
+    const EncJob &jb = J.j[S.job[q]];
+    const int64_t off = S.base[q];
+    const int64_t cnt = S.rinc[q][kTileRows - 1];
+    const int64_t lim = (off + cnt < jb.capacity) ? off + cnt : jb.capacity;
+    if (lim <= off) return;
+    const uint32_t *vs = S.vst[sb];
+    const uint8_t *cs = S.cst[sb];
     const int64_t base16 = off & ~15ll;                     // staging index of entry e: e - base16
     const int64_t g_lo = (off + 15) >> 4, g_hi = lim >> 4;  // whole 16-entry groups [g_lo, g_hi)
-    fence_proxy_async_smem();  // generic staging writes -> async-proxy bulk reads
-    __syncwarp();
     if (g_hi > g_lo) {
         if (lane == 0) {
             const int s0 = (int)(16 * g_lo - base16);
             const uint32_t ng = (uint32_t)(g_hi - g_lo);
-            tma_store_1d(val + 16 * g_lo, vs + s0, 64u * ng);
-            tma_store_1d(col + 16 * g_lo, cs + s0, 16u * ng);
+            tma_store_1d(jb.val + 16 * g_lo, vs + s0, 64u * ng);
+            tma_store_1d(jb.col + 16 * g_lo, cs + s0, 16u * ng);
             bulk_commit();
         }
-        // head [off, 16 g_lo) by lanes 0..15, tail [16 g_hi, lim) by lanes 16..31
         const int64_t e = lane < 16 ? 16 * g_lo - 16 + lane : 16 * g_hi + lane - 16;
         if (e >= off && e < lim) {
-            val[e] = __uint_as_float(vs[e - base16]);
-            col[e] = cs[e - base16];
+            jb.val[e] = __uint_as_float(vs[e - base16]);
+            jb.col[e] = cs[e - base16];
         }
     } else {
         // no whole 16-entry group: fewer than 32 entries
         for (int64_t e = off + lane; e < lim; e += 32) {
-            val[e] = __uint_as_float(vs[e - base16]);
-            col[e] = cs[e - base16];
+            jb.val[e] = __uint_as_float(vs[e - base16]);
+            jb.col[e] = cs[e - base16];
         }
     }
-    __syncwarp();
 }
 
 #ifdef GIST_SSDC_TRACE
@@ -262,7 +261,7 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
     // Prologue before the programmatic-dependency wait touches shared memory only (the barrier
     // initialisation overlaps the previous kernel's tail); after it, the first ticket claim and
     // the read of the counter line (epoch, magic) are issued together.
-#if GIST_PDL
+#if GIST_PDL && GIST_PDL_EARLY
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 #endif
     if (threadIdx.x == 0) {
@@ -482,11 +481,22 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
             }
             return t;
         };
+        // tile jj stages into buffer jj & 1.  One named barrier per tile among the writers: after
+        // it, the tile is fully staged (writer 0 then stores it), and writer 0's bulk copies of the
+        // previous tile, which it waited on just before, have read buffer (jj - 1) & 1, so tile
+        // jj + 1 may overwrite it.
         auto retire = [&](int64_t jj, int64_t t, const uint4 (&l)[kWRows], const uint4 (&h)[kWRows]) {
             const int q = (int)(jj % kQ);
+            const int sb = (int)(jj & 1);
             mbar_wait_sleep(&S.resolved[q], (uint32_t)(jj / kQ) & 1u);
-            write_rows(S, q, w, lane, l, h, J);
-            __syncwarp();
+            stage_rows(S, q, sb, w, lane, l, h);
+            fence_proxy_async_smem();  // generic staging writes -> async-proxy bulk reads
+            if (w == 0 && lane == 0) bulk_wait_read();
+            named_bar(1, kWriterThreads);
+            if (w == 0) {
+                store_tile(S, q, sb, lane, J);
+                __syncwarp();
+            }
             if (lane == 0) {
                 if (w == 0) TRACE(jj, 3);
                 mbar_arrive1(&S.freed[q]);

@@ -113,7 +113,9 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
     }
     if (warp == 0) tmem_alloc<kTmemCols>(&S.tmem_base);
 #if GIST_PDL
+#if GIST_PDL_EARLY
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+#endif
     asm volatile("griddepcontrol.wait;" ::: "memory");
 #endif
     tc_fence_before();

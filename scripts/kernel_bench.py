@@ -57,6 +57,8 @@ def main():
     dev = torch.device("cuda:0")
     peak, src = bench.hbm_peak()
     res = []
+    clocks = bench.ClockSampler(dev)
+    clocks.__enter__()
 
     def rep(row, name, nbytes, fn, extra=None):
         if only and row not in only:
@@ -142,10 +144,13 @@ def main():
         rep("a6", f"fp{bits} 205.5M elems", b, lambda: gist.gist_dpr_encode(x, bits, packed=packed))
         rep("a7", f"fp{bits} 205.5M elems", b, lambda: gist.gist_dpr_decode(packed, n, bits, x=xd))
         del packed
+    clocks.__exit__(None, None, None)
+    clk = clocks.summary()
+    print(json.dumps({"clocks": clk}), flush=True)
     if args.json:
         with open(args.json, "w") as f:
             json.dump({"peak_GBps": peak, "peak_source": src, "gpu": torch.cuda.get_device_name(dev),
-                       "results": res}, f, indent=1)
+                       "clocks": clk, "results": res}, f, indent=1)
 
 
 if __name__ == "__main__":

@@ -76,8 +76,9 @@ def test_ssdc_chained_arena(gist, ref, cuda, start):
     sizes = [256 * 32 * 40 + 7, 5000, 1, 256 * 33, 777_777]
     xs = maps(sizes, 5, cuda)
     cap = start + sum(sizes)
-    col = torch.zeros(cap, dtype=torch.uint8, device=cuda)
-    val = torch.zeros(cap, dtype=torch.float32, device=cuda)
+    extra = 9999  # room for the single-job append at the end
+    col = torch.zeros(cap + extra, dtype=torch.uint8, device=cuda)
+    val = torch.zeros(cap + extra, dtype=torch.float32, device=cuda)
     offs = torch.zeros(len(sizes) + 1, dtype=torch.int64, device=cuda)
     offs[0] = start
     jobs = [{"x": x, "col": col, "val": val, "capacity": cap, "offset": offs[k:k + 1], "nnz": offs[k + 1:k + 2]}
@@ -96,12 +97,16 @@ def test_ssdc_chained_arena(gist, ref, cuda, start):
     for x, b in zip(xs, backs):
         assert torch.equal(b.view(torch.int32), x.view(torch.int32))
     # single-job append mode (offset known from an earlier call)
-    more = WL.relu_map((9999,), 0.6, 99, cuda)
+    more = WL.relu_map((extra,), 0.6, 99, cuda)
     tail = torch.zeros(1, dtype=torch.int64, device=cuda)
-    rows = gist.gist_ssdc_encode_many([{"x": more, "col": col, "val": val, "capacity": cap + 9999,
+    rows = gist.gist_ssdc_encode_many([{"x": more, "col": col, "val": val, "capacity": cap + extra,
                                         "offset": offs[-1:], "nnz": tail}])
-    assert int(tail.item()) - o[-1] == int((more.view(torch.int32) != 0).sum().item()) or \
-        int(tail.item()) > cap  # entries past capacity are dropped, the true end is still published
+    t = int(tail.item())
+    r_row_end, r_col, r_val = ref.ssdc_encode(host(more))
+    assert t - o[-1] == r_col.size
+    same(host(rows[0][0]), (r_row_end.astype(np.int64) + o[-1]).astype(np.int32), "append row_end")
+    same(host(col[o[-1]:t]), r_col, "append col")
+    same(host(val[o[-1]:t]), r_val, "append val")
 
 
 @pytest.mark.parametrize("bits", [16, 10, 8])
