@@ -725,7 +725,7 @@ def main():
         "data": "synthetic",
         "config": workload_config(args, cfg, batch if not strong else cfg.batch, strong=strong, world=world),
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": round(dom_gbs, 1), "peak": peak, "unit": "GB/s",
-                     "frac": round(dom_gbs / peak, 4), "traffic": traffic_for(dom), "peak_source": peak_src},
+                     "frac": round(dom_gbs / peak, 4), "traffic": traffic_for(args, dom), "peak_source": peak_src},
         "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": launches,
@@ -744,14 +744,19 @@ def main():
         dist.destroy_process_group()
 
 
-def traffic_for(kind):
-    """DRAM bytes per launch from the committed ncu --set full capture, if one exists."""
+def traffic_for(args, kind):
+    """DRAM bytes per launch of the dominant kernel, from the committed ncu --set full capture of
+    THIS configuration's launch (profiles/ncu_traffic.json, keyed "<config>:<kernel>:<many|per-site>"
+    at the config's default batch, sparsity and DPR width); None when no such capture exists."""
+    if args.batch is not None or args.sparsity is not None or args.dpr_bits is not None:
+        return None
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if not os.path.exists(p):
         return None
     with open(p) as f:
         t = json.load(f)
-    return t.get(kind, {}).get("dram_bytes_per_launch")
+    key = f"{args.config}:{kind}:{'many' if args.many else 'per-site'}"
+    return t.get(key, {}).get("dram_bytes_per_launch")
 
 
 if __name__ == "__main__":

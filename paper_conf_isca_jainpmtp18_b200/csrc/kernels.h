@@ -63,6 +63,16 @@ cudaError_t launch_dpr_many(const gist_dpr_job *jobs, int32_t count, int bits, b
 cudaError_t launch_dpr_decode(const uint32_t *packed, int64_t n, int bits, float *x, cudaStream_t s,
                               const int64_t *n_dev = nullptr);
 
+// pool3.cu: 3x3 windows (stride 1/2, pad 0/1, floor/ceil) through plane tiles in shared memory;
+// cudaErrorNotSupported when a plane does not fit (the caller falls back)
+bool pool3_ok(const gist_pool2d &p);
+cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p,
+                             int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, uint32_t *mask, bool relu,
+                             cudaStream_t s);
+cudaError_t launch_pool3_bwd(const float *dout, const uint32_t *argmax, const uint32_t *mask, int32_t N, int32_t C,
+                             int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo, float *dx,
+                             cudaStream_t s);
+
 // f4 (wgrad.cu): 3x3/s1/p1 conv weight gradient, X decoded from SSDC inside the tcgen05 GEMM
 bool wgrad_shape_ok(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W);
 size_t wgrad_workspace_bytes(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W);

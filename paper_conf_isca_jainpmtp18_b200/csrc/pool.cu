@@ -31,6 +31,9 @@ constexpr int kPoolThreads = 256;
 #define GIST_POOL_GEN_CTAS 32  // generic-geometry kernels: grid cap in CTAs per SM (8 resident); 32-64 measured
                                // 8-14% faster than 8 on the 3x3/s2 maps (AlexNet, NiN), 4 and 1000 slower
 #endif
+#ifndef GIST_POOL3
+#define GIST_POOL3 1  // 3x3 windows through the plane-tiled kernels of pool3.cu (0: the L1 kernels below)
+#endif
 #ifndef GIST_POOL_BWD_CTAS
 #define GIST_POOL_BWD_CTAS 6
 #endif
@@ -756,6 +759,13 @@ cudaError_t launch_relu_maxpool_fwd(const float *x, int32_t N, int32_t C, int32_
     // geometries use the L1 forward with relu on load and the caller adds binarize(x).
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
     *mask_fused = false;
+    if (GIST_POOL3 && pool3_ok(p)) {
+        const cudaError_t e = launch_pool3_fwd(x, N, C, H, W, p, Ho, Wo, out, argmax, mask, true, s);
+        if (e != cudaErrorNotSupported) {
+            *mask_fused = mask != nullptr;
+            return e;
+        }
+    }
     if (is_k2s2_exact(p, H, W, Ho, Wo) && H == 2 * Ho) {
         const int V = (W % 4 == 0) ? 4 : 2;
         const int ipr = W / V;
@@ -787,6 +797,14 @@ cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, 
                                bool *mask_fused) {
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
     if (mask_fused) *mask_fused = false;
+    if (GIST_POOL3 && pool3_ok(p)) {
+        const cudaError_t e = launch_pool3_fwd(y, N, C, H, W, p, Ho, Wo, out, argmax, mask_fused ? mask : nullptr,
+                                               false, s);
+        if (e != cudaErrorNotSupported) {
+            if (mask_fused) *mask_fused = mask != nullptr;
+            return e;
+        }
+    }
     if (mask && is_k2s2_exact(p, H, W, Ho, Wo) && H == 2 * Ho) {
         // units of BR whole row blocks with BR*W = 0 mod 16 (word-aligned), ~256 items each
         const int V = (W % 4 == 0) ? 4 : 2;
@@ -824,6 +842,10 @@ cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uin
                             int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo, float *dx,
                             cudaStream_t s) {
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
+    if (GIST_POOL3 && pool3_ok(p)) {
+        const cudaError_t e = launch_pool3_bwd(dout, argmax, mask, N, C, H, W, p, Ho, Wo, dx, s);
+        if (e != cudaErrorNotSupported) return e;
+    }
     if (is_k2s2_exact(p, H, W, Ho, Wo) && W % 4 == 0) {
         const unsigned g2 = grid_for(ceil_div(a.n_out / 2, kPairU), kPoolThreads, GIST_POOL_BWD_CTAS);
         if (H == 2 * Ho) launch_k(pool_bwd_k2s2_pair_kernel<true>, g2, kPoolThreads, 0, s, dout, argmax, mask, a, dx);

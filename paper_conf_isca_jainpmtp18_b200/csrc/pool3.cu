@@ -1,0 +1,592 @@
+// pool3.cu — a2 (+a1 fused) and a3 for 3x3 windows, stride 1 or 2, padding 0 or 1, floor or ceil
+// mode: the AlexNet / NiN / GoogLeNet pools (§III-A, P:151-P:156 §IV-A).
+//
+// Plane tiles through a TMA ring.  A tile is G whole planes; their input (forward) or their dY,
+// argmax words and mask words (backward) are contiguous ranges of the maps, so one persistent CTA
+// per (half) SM streams tile after tile into a kRS-deep shared-memory ring with 1-D bulk copies
+// (cp.async.bulk, issued by one thread) while its 256 threads compute the current tile from shared
+// memory: HBM sees each byte once, and the loads of the next tiles are in flight during compute.
+//   forward, stride 2: one thread per output (lanes = consecutive outputs); taps outside the input
+//     read as -inf (never selected under the strict '>' rule, R3), the argmax starts at the
+//     window's first in-bounds position, so an all -inf window gives the oracle's index.  8-lane
+//     groups OR their nibbles into one argmax word.
+//   forward, stride 1: separable.  One thread per output column of a plane walks down the rows,
+//     keeping the row-wise (max, index) of the last three input rows: each input row is scanned
+//     once, not three times.  Scanning rows, then combining the row results in row order with the
+//     same rule, is the row-major scan of the window (last NaN wins, else first maximum).
+//     Nibbles go to shared memory (one byte per output) and are packed into words afterwards.
+//   the a1 mask (forward, when requested): one thread per mask word reads its 32 staged floats.
+//   backward, stride 2: one thread per 2x2 input block: its 4 candidate windows (A-1,b-1), (A-1,b),
+//     (A,b-1), (A,b) route fixed nibbles to fixed block positions, in ascending output order (R6).
+//   backward, stride 1: one thread per input element, its 9 candidate windows in ascending output
+//     order; both select with the mask bit (R7).
+// Word ownership (forward): a tile owns the argmax words whose first output lies in its planes and
+// the mask words whose first element does; the tail of its last word may lie in the next plane, so
+// the tile also stages the first rows of plane p0+G.  Tiles never share an output word.
+#include <math_constants.h>
+
+#include <algorithm>
+
+#include "common.cuh"
+#include "kernels.h"
+#include "tma.cuh"
+
+namespace gist {
+
+namespace {
+
+#ifndef GIST_POOL3_THREADS
+#define GIST_POOL3_THREADS 512  // 256: 10-40% slower, 1024: 5-25% slower (3x3/s1 maps, GoogLeNet b64)
+#endif
+constexpr int kRT = GIST_POOL3_THREADS;  // threads per CTA
+constexpr int kRS = 3;    // ring stages
+#ifndef GIST_POOL3_STAGE_KB
+#define GIST_POOL3_STAGE_KB 32  // KB per ring stage (3 stages + extras < 113 KB: 2 CTAs per SM)
+#endif
+constexpr int kStageBytes = GIST_POOL3_STAGE_KB * 1024;
+constexpr int kStageFloats = kStageBytes / 4;
+constexpr int kNbBytes = 12 * 1024;  // nibble bytes of one tile (stride-1 forward, backward)
+
+struct P3Args {
+    int32_t H, W, Ho, Wo, S, P;
+    int32_t HW, HoWo;
+    int32_t G;       // planes per tile
+    int32_t xrows;   // forward: input rows of plane p0+G a tile may need (0: none)
+    int32_t hb, wb;  // stride-2 backward: 2x2 blocks per plane (rows, columns)
+    int32_t PR, PC;  // backward: padded nibble-byte plane (rows, columns)
+    int32_t a_off, m_off;  // backward stage layout (floats): dY at 0, argmax words, mask words
+    int64_t NC, tiles, n_in, n_out;
+    FastDiv div_hw, div_w, div_howo, div_wo, div_blk, div_wb;
+};
+
+__device__ __forceinline__ void take3(float v, int idx, float &best, int &bi) {
+    if (v > best || v != v) {  // R3: strict '>' keeps the first maximum; NaN always wins
+        best = v;
+        bi = idx;
+    }
+}
+
+template <bool RELU>
+__device__ __forceinline__ float act3(float v) {
+    return RELU ? (v < 0.0f ? 0.0f : v) : v;  // f3 in-place ReLU (R21)
+}
+
+// The bulk copy of floats [lo, hi) of g: from the 16-B aligned sb = lo & ~3, the whole quads; the
+// ragged <= 3 elements at the end are loaded by the consumers (tail_fill).
+__device__ __forceinline__ uint32_t ring_bytes(int64_t lo, int64_t hi) {
+    return (uint32_t)(((hi - (lo & ~3ll)) & ~3ll) * 4);
+}
+
+__device__ __forceinline__ void ring_copy(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    constexpr uint32_t kChunk = 16 * 1024;  // several copies in flight per stage
+    for (uint32_t off = 0; off < bytes; off += kChunk)
+        tma_load_1d(static_cast<char *>(dst) + off, static_cast<const char *>(src) + off,
+                    bytes - off < kChunk ? bytes - off : kChunk, bar);
+}
+
+// Loads the ragged tail (elements past the bulk-copied quads) of [lo, hi) with threads tid0..tid0+2.
+template <typename T>
+__device__ __forceinline__ bool tail_fill(T *dst, const T *__restrict__ src, int64_t lo, int64_t hi, int tid0) {
+    const int64_t sb = lo & ~3ll, te = sb + ((hi - sb) & ~3ll);
+    const int t = (int)threadIdx.x - tid0;
+    if (t >= 0 && t < hi - te) {
+        dst[te - sb + t] = src[te + t];
+        return true;
+    }
+    return false;
+}
+
+struct FwdTile {
+    int64_t p0, lo, hi, oa, ob, ia, ib;
+    int np;
+};
+
+__device__ __forceinline__ FwdTile fwd_tile(const P3Args &a, int64_t k) {
+    FwdTile t;
+    t.p0 = k * a.G;
+    t.np = (int)min((int64_t)a.G, a.NC - t.p0);
+    const bool last = t.p0 + t.np == a.NC;
+    t.oa = (t.p0 * a.HoWo + 7) & ~7ll;
+    t.ob = last ? a.n_out : (((t.p0 + t.np) * a.HoWo + 7) & ~7ll);
+    t.ia = (t.p0 * a.HW + 31) & ~31ll;
+    t.ib = last ? a.n_in : (((t.p0 + t.np) * a.HW + 31) & ~31ll);
+    t.lo = t.p0 * a.HW;
+    const int64_t end = t.lo + (int64_t)t.np * a.HW;
+    t.hi = last ? end : min(a.n_in, end + max((int64_t)a.xrows * a.W, t.ib - end));
+    return t;
+}
+
+// Row-wise scan of input row ih over columns iw0 .. iw0+2 (stride 1): (max, column index).
+template <bool RELU>
+__device__ __forceinline__ void hscan(const float *row, int ih, int iw0, const P3Args &a, float &v, int &x) {
+    v = -CUDART_INF_F;
+    x = max(0, -iw0);
+    if (ih < 0 || ih >= a.H) return;
+#pragma unroll
+    for (int dx = 0; dx < 3; ++dx) {
+        const int iw = iw0 + dx;
+        if (iw >= 0 && iw < a.W) take3(act3<RELU>(row[iw]), dx, v, x);
+    }
+}
+
+template <int S, bool MASK, bool RELU, bool CHECK>
+__global__ void __launch_bounds__(kRT)
+pool3_fwd_kernel(const float *__restrict__ y, P3Args a, float *__restrict__ out, uint32_t *__restrict__ arg,
+                 uint32_t *__restrict__ mask) {
+    pdl_enter();
+    extern __shared__ __align__(128) unsigned char smp[];
+    float *ring = reinterpret_cast<float *>(smp);
+    uint8_t *nbs = smp + kRS * kStageBytes;  // stride 1: nibble bytes of the tile
+    uint64_t *full = reinterpret_cast<uint64_t *>(smp + kRS * kStageBytes + (S == 1 ? kNbBytes : 0));
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const float ninf = -CUDART_INF_F;
+    if (tid == 0) {
+        for (int s = 0; s < kRS; ++s) mbar_init(&full[s], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const int64_t mine = a.tiles > blockIdx.x ? (a.tiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+    auto issue = [&](int64_t j) {
+        const FwdTile t = fwd_tile(a, blockIdx.x + j * gridDim.x);
+        const int st = (int)(j % kRS);
+        const uint32_t b = ring_bytes(t.lo, t.hi);
+        mbar_arrive_expect_tx(&full[st], b);
+        if (b) ring_copy(ring + (size_t)st * kStageFloats, y + (t.lo & ~3ll), b, &full[st]);
+    };
+    if (tid == 0)
+        for (int64_t j = 0; j < kRS && j < mine; ++j) issue(j);
+    for (int64_t j = 0; j < mine; ++j) {
+        const int st = (int)(j % kRS);
+        float *R = ring + (size_t)st * kStageFloats;
+        const FwdTile t = fwd_tile(a, blockIdx.x + j * gridDim.x);
+        const int64_t sb = t.lo & ~3ll;  // stage index of element e: e - sb
+        mbar_wait(&full[st], (uint32_t)(j / kRS) & 1u);
+        if (tail_fill(R, y, t.lo, t.hi, 0)) fence_proxy_async_smem();
+        __syncthreads();
+        // a1 mask words [ia/32, ib/32) (relu(y) > 0 iff y > 0): one staged float4 per lane, the 8
+        // lanes of a word OR their bits together (conflict-free 128-bit shared loads)
+        if (MASK) {
+            const int64_t q0 = t.ia >> 2, q1 = ((t.ib + 31) >> 5) << 3;  // quads of the owned words
+            for (int64_t qb = q0; qb < q1; qb += kRT) {
+                const int64_t q = qb + tid;  // q0 % 8 == 0 and kRT % 8 == 0: lanes 8g..8g+7 = one word
+                uint32_t bits = 0;
+                if (q < q1) {
+                    const float4 f = *reinterpret_cast<const float4 *>(R + (4 * q - sb));
+                    const int64_t e = 4 * q;  // O1: y > 0 (NaN, -0.0 -> 0); elements past the map read 0
+                    bits = (f.x > 0.0f && e < t.hi ? 1u : 0u) | (f.y > 0.0f && e + 1 < t.hi ? 2u : 0u) |
+                           (f.z > 0.0f && e + 2 < t.hi ? 4u : 0u) | (f.w > 0.0f && e + 3 < t.hi ? 8u : 0u);
+                }
+                bits <<= 4 * (lane & 7);
+                bits |= __shfl_xor_sync(kFull, bits, 1);
+                bits |= __shfl_xor_sync(kFull, bits, 2);
+                bits |= __shfl_xor_sync(kFull, bits, 4);
+                if ((lane & 7) == 0 && q < q1) mask[q >> 3] = bits;
+            }
+        }
+        const int64_t olo = t.p0 * a.HoWo;
+        if (S == 2) {
+            // one thread per owned output, 32 consecutive outputs per warp (oa % 8 == 0)
+            const int la = (int)(t.oa - olo), lb = (int)(t.ob - olo);
+            for (int c = la + warp * 32; c < lb; c += kRT) {
+                const int l = c + lane;
+                uint32_t nib = 0;
+                if (l < lb) {
+                    uint32_t pl, rem, oh, ow;
+                    a.div_howo.divmod((uint32_t)l, pl, rem);
+                    a.div_wo.divmod(rem, oh, ow);
+                    const int ih0 = (int)oh * 2 - a.P, iw0 = (int)ow * 2 - a.P;
+                    const float *pb = R + ((t.p0 + pl) * a.HW - sb);
+                    int bi = max(0, -ih0) * 3 + max(0, -iw0);
+                    float best = ninf;
+#pragma unroll
+                    for (int dy = 0; dy < 3; ++dy) {
+                        const int ih = ih0 + dy;
+                        const bool rok = !CHECK || (ih >= 0 && ih < a.H);
+#pragma unroll
+                        for (int dx = 0; dx < 3; ++dx) {
+                            const int iw = iw0 + dx;
+                            const bool ok = rok && (!CHECK || (iw >= 0 && iw < a.W));
+                            const float v = ok ? act3<RELU>(pb[ok ? ih * a.W + iw : 0]) : ninf;
+                            take3(v, 3 * dy + dx, best, bi);
+                        }
+                    }
+                    out[olo + l] = best;
+                    nib = (uint32_t)bi << (4 * (lane & 7));
+                }
+                nib |= __shfl_xor_sync(kFull, nib, 1);
+                nib |= __shfl_xor_sync(kFull, nib, 2);
+                nib |= __shfl_xor_sync(kFull, nib, 4);
+                if ((lane & 7) == 0 && l < lb) arg[(olo + l) >> 3] = nib;
+            }
+        } else {
+            // stride 1 (G * HoWo % 8 == 0: every word whole in the tile): one thread per output column
+            const int items = t.np * a.Wo;
+            for (int it = tid; it < items; it += kRT) {
+                uint32_t pl, ow;
+                a.div_wo.divmod((uint32_t)it, pl, ow);
+                const float *pb = R + ((t.p0 + pl) * a.HW - sb);
+                const int iw0 = (int)ow - a.P;
+                float hv[3];
+                int hx[3];
+                hscan<RELU>(pb - a.P * a.W, -a.P, iw0, a, hv[0], hx[0]);
+                hscan<RELU>(pb + (1 - a.P) * a.W, 1 - a.P, iw0, a, hv[1], hx[1]);
+                const int dx0 = max(0, -iw0);
+                float *op = out + olo + (int64_t)pl * a.HoWo + ow;
+                uint8_t *nb = nbs + pl * a.HoWo + ow;
+                for (int oh = 0; oh < a.Ho; ++oh) {
+                    const int ih2 = oh - a.P + 2;
+                    hscan<RELU>(pb + ih2 * a.W, ih2, iw0, a, hv[2], hx[2]);
+                    float best = ninf;
+                    int bi = max(0, a.P - oh) * 3 + dx0;
+#pragma unroll
+                    for (int dy = 0; dy < 3; ++dy) take3(hv[dy], 3 * dy + hx[dy], best, bi);
+                    op[(int64_t)oh * a.Wo] = best;
+                    nb[oh * a.Wo] = (uint8_t)bi;
+                    hv[0] = hv[1], hx[0] = hx[1];
+                    hv[1] = hv[2], hx[1] = hx[2];
+                }
+            }
+            __syncthreads();
+            // pack: one argmax word per thread (8 nibble bytes, one aligned 64-bit load); only the
+            // map's last word can be partial (its pad nibbles are 0)
+            const int no = t.np * a.HoWo;
+            const int nw = (no + 7) >> 3;
+            for (int w = tid; w < nw; w += kRT) {
+                const uint2 b = *reinterpret_cast<const uint2 *>(nbs + 8 * w);
+                const uint32_t lo4 = (b.x & 0xfu) | ((b.x >> 4) & 0xf0u) | ((b.x >> 8) & 0xf00u) | ((b.x >> 12) & 0xf000u);
+                const uint32_t hi4 = (b.y & 0xfu) | ((b.y >> 4) & 0xf0u) | ((b.y >> 8) & 0xf00u) | ((b.y >> 12) & 0xf000u);
+                const int valid = no - 8 * w;  // nibbles of this word inside the map
+                const uint32_t keep = valid >= 8 ? ~0u : ((1u << (4 * valid)) - 1u);
+                arg[(olo >> 3) + w] = (lo4 | (hi4 << 16)) & keep;
+            }
+        }
+        __syncthreads();  // stage st (and the nibble bytes) consumed
+        if (tid == 0 && j + kRS < mine) issue(j + kRS);
+    }
+}
+
+// ---------------------------------------------------------------- backward
+struct BwdTile {
+    int64_t p0, olo, ohi, ilo, ihi, aw_lo, aw_hi, mw_lo, mw_hi;
+    int np;
+};
+
+__device__ __forceinline__ BwdTile bwd_tile(const P3Args &a, int64_t k) {
+    BwdTile t;
+    t.p0 = k * a.G;
+    t.np = (int)min((int64_t)a.G, a.NC - t.p0);
+    t.olo = t.p0 * a.HoWo;
+    t.ohi = t.olo + (int64_t)t.np * a.HoWo;
+    t.ilo = t.p0 * a.HW;
+    t.ihi = t.ilo + (int64_t)t.np * a.HW;
+    t.aw_lo = t.olo >> 3;
+    t.aw_hi = (t.ohi + 7) >> 3;
+    t.mw_lo = t.ilo >> 5;
+    t.mw_hi = (t.ihi + 31) >> 5;
+    return t;
+}
+
+template <int S, bool MASK>
+__global__ void __launch_bounds__(kRT)
+pool3_bwd_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg, const uint32_t *__restrict__ mask,
+                 P3Args a, float *__restrict__ dx) {
+    pdl_enter();
+    extern __shared__ __align__(128) unsigned char smp[];
+    float *ring = reinterpret_cast<float *>(smp);
+    uint8_t *nbb = smp + kRS * kStageBytes;  // padded nibble-byte planes of the tile
+    uint64_t *full = reinterpret_cast<uint64_t *>(smp + kRS * kStageBytes + kNbBytes);
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        for (int s = 0; s < kRS; ++s) mbar_init(&full[s], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const int64_t mine = a.tiles > blockIdx.x ? (a.tiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+    auto issue = [&](int64_t j) {
+        const BwdTile t = bwd_tile(a, blockIdx.x + j * gridDim.x);
+        const int st = (int)(j % kRS);
+        float *R = ring + (size_t)st * kStageFloats;
+        const uint32_t bd = ring_bytes(t.olo, t.ohi), ba = ring_bytes(t.aw_lo, t.aw_hi);
+        const uint32_t bm = MASK ? ring_bytes(t.mw_lo, t.mw_hi) : 0u;
+        mbar_arrive_expect_tx(&full[st], bd + ba + bm);
+        if (bd) ring_copy(R, dout + (t.olo & ~3ll), bd, &full[st]);
+        if (ba) ring_copy(R + a.a_off, arg + (t.aw_lo & ~3ll), ba, &full[st]);
+        if (bm) ring_copy(R + a.m_off, mask + (t.mw_lo & ~3ll), bm, &full[st]);
+    };
+    if (tid == 0)
+        for (int64_t j = 0; j < kRS && j < mine; ++j) issue(j);
+    for (int64_t j = 0; j < mine; ++j) {
+        const int st = (int)(j % kRS);
+        float *R = ring + (size_t)st * kStageFloats;
+        const BwdTile t = bwd_tile(a, blockIdx.x + j * gridDim.x);
+        mbar_wait(&full[st], (uint32_t)(j / kRS) & 1u);
+        {
+            uint32_t *RA = reinterpret_cast<uint32_t *>(R + a.a_off), *RM = reinterpret_cast<uint32_t *>(R + a.m_off);
+            bool wrote = tail_fill(R, dout, t.olo, t.ohi, 0);
+            wrote |= tail_fill(RA, arg, t.aw_lo, t.aw_hi, 4);
+            if (MASK) wrote |= tail_fill(RM, mask, t.mw_lo, t.mw_hi, 8);
+            if (wrote) fence_proxy_async_smem();
+        }
+        __syncthreads();
+        const float *D = R + (t.olo - (t.olo & ~3ll));  // dY by tile-local output index
+        // argmax / mask words by (tile-local index + phase) >> 3 / >> 5
+        const uint32_t *Aw = reinterpret_cast<const uint32_t *>(R + a.a_off) + (t.aw_lo - (t.aw_lo & ~3ll));
+        const uint32_t *Mw = reinterpret_cast<const uint32_t *>(R + a.m_off) + (t.mw_lo - (t.mw_lo & ~3ll));
+        const int aph = (int)(t.olo & 7), mph = (int)(t.ilo & 31);
+        // nibbles -> one byte per window in padded planes (window (oh, ow) at (oh + OFF, ow + OFF),
+        // OFF = 2 for stride 1, 1 for stride 2); cells holding no window read 0xF (never a hit)
+        constexpr int OFF = S == 1 ? 2 : 1;
+        const int PP = a.PR * a.PC;
+        {
+            uint4 *n4 = reinterpret_cast<uint4 *>(nbb);
+            const int c16 = (t.np * PP + 15) >> 4;
+            for (int i = tid; i < c16; i += kRT) n4[i] = make_uint4(~0u, ~0u, ~0u, ~0u);
+        }
+        __syncthreads();
+        {
+            const int no = t.np * a.HoWo;
+            const int nw = (aph + no + 7) >> 3;
+            for (int w = tid; w < nw; w += kRT) {
+                const uint32_t word = Aw[w];
+                const int l0 = 8 * w - aph;  // tile-local output of nibble 0
+                uint32_t pl, rem, oh, ow;
+                a.div_howo.divmod((uint32_t)(l0 > 0 ? l0 : 0), pl, rem);
+                a.div_wo.divmod(rem, oh, ow);
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    const int l = l0 + k;
+                    if (l >= 0 && l < no) {
+                        nbb[(int)pl * PP + ((int)oh + OFF) * a.PC + (int)ow + OFF] = (uint8_t)((word >> (4 * k)) & 0xfu);
+                        if (++ow == (uint32_t)a.Wo) {
+                            ow = 0;
+                            if (++oh == (uint32_t)a.Ho) {
+                                oh = 0;
+                                ++pl;
+                            }
+                        }
+                    }
+                }
+            }
+        }
+        __syncthreads();
+        auto mbit = [&](int il) { return !MASK || ((Mw[(il + mph) >> 5] >> ((il + mph) & 31)) & 1u); };
+        float *dxt = dx + t.ilo;
+        if (S == 2) {
+            const int nblk = t.np * a.hb * a.wb;
+            for (int q = tid; q < nblk; q += kRT) {
+                uint32_t pl, rem, A, b;
+                a.div_blk.divmod((uint32_t)q, pl, rem);
+                a.div_wb.divmod(rem, A, b);
+                const int c11 = (int)pl * PP + ((int)A + 1) * a.PC + (int)b + 1;  // window (A, b)
+                const unsigned n00 = nbb[c11 - a.PC - 1], n01 = nbb[c11 - a.PC], n10 = nbb[c11 - 1], n11 = nbb[c11];
+                const int o11 = (int)pl * a.HoWo + (int)A * a.Wo + (int)b;  // dY of window (A, b)
+                float a00 = 0.0f, a01 = 0.0f, a10 = 0.0f, a11 = 0.0f;  // +0.0f, then ascending o
+                if (n00 == 8u) a00 = a00 + D[o11 - a.Wo - 1];
+                if (n01 == 6u) a00 = a00 + D[o11 - a.Wo];
+                if (n01 == 7u) a01 = a01 + D[o11 - a.Wo];
+                if (n10 == 2u) a00 = a00 + D[o11 - 1];
+                if (n10 == 5u) a10 = a10 + D[o11 - 1];
+                if (n11 == 0u) a00 = a00 + D[o11];
+                if (n11 == 1u) a01 = a01 + D[o11];
+                if (n11 == 3u) a10 = a10 + D[o11];
+                if (n11 == 4u) a11 = a11 + D[o11];
+                // inputs of the block that exist: ih = 2A + r - P, iw = 2b + c - P
+                const int ih0 = 2 * (int)A - a.P, iw0 = 2 * (int)b - a.P;
+                const bool r0 = ih0 >= 0, r1 = ih0 + 1 < a.H, c0 = iw0 >= 0, c1 = iw0 + 1 < a.W;
+                const int il = (int)pl * a.HW + ih0 * a.W + iw0;
+                if (r0 && c0) dxt[il] = mbit(il) ? a00 : 0.0f;
+                if (r0 && c1) dxt[il + 1] = mbit(il + 1) ? a01 : 0.0f;
+                if (r1 && c0) dxt[il + a.W] = mbit(il + a.W) ? a10 : 0.0f;
+                if (r1 && c1) dxt[il + a.W + 1] = mbit(il + a.W + 1) ? a11 : 0.0f;
+            }
+        } else {
+            // one thread per input element; windows (oh, ow) = (th - dy, tw - dx), th = ih + P, in
+            // ascending output order; the hit nibble is 3 dy + dx
+            const int cnt = t.np * a.HW;
+            for (int l = tid; l < cnt; l += kRT) {
+                const bool on = mbit(l);
+                float acc = 0.0f;  // R6: +0.0f, then ascending output order
+                if (on) {
+                    uint32_t pl, rem, ih, iw;
+                    a.div_hw.divmod((uint32_t)l, pl, rem);
+                    a.div_w.divmod(rem, ih, iw);
+                    const int th = (int)ih + a.P, tw = (int)iw + a.P;
+                    const int cell = (int)pl * PP + (th + 2) * a.PC + tw + 2;  // window (th, tw)
+                    const int ol = (int)pl * a.HoWo + th * a.Wo + tw;          // its dY (when it exists)
+#pragma unroll
+                    for (int dy = 2; dy >= 0; --dy)
+#pragma unroll
+                        for (int dxx = 2; dxx >= 0; --dxx)
+                            if (nbb[cell - dy * a.PC - dxx] == (unsigned)(3 * dy + dxx)) acc = acc + D[ol - dy * a.Wo - dxx];
+                }
+                dxt[l] = on ? acc : 0.0f;
+            }
+        }
+        __syncthreads();  // stage st consumed
+        if (tid == 0 && j + kRS < mine) issue(j + kRS);
+    }
+}
+
+int gcd_i(int a, int b) {
+    while (b) {
+        const int t = a % b;
+        a = b;
+        b = t;
+    }
+    return a;
+}
+
+P3Args p3_args(int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo) {
+    P3Args a{};
+    a.H = H;
+    a.W = W;
+    a.Ho = Ho;
+    a.Wo = Wo;
+    a.S = p.sh;
+    a.P = p.ph;
+    a.HW = H * W;
+    a.HoWo = Ho * Wo;
+    a.NC = (int64_t)N * C;
+    a.n_in = a.NC * a.HW;
+    a.n_out = a.NC * a.HoWo;
+    a.div_hw = FastDiv::make((uint32_t)a.HW);
+    a.div_w = FastDiv::make((uint32_t)W);
+    a.div_howo = FastDiv::make((uint32_t)a.HoWo);
+    a.div_wo = FastDiv::make((uint32_t)Wo);
+    return a;
+}
+
+// Planes per tile: as many as a stage holds (`per_plane` floats each, `fixed` floats of slack),
+// a multiple of `unit`, but no more than keeps ~4 tiles per CTA.  0: one unit does not fit.
+int32_t choose_g(int64_t NC, int64_t per_plane, int64_t fixed, int32_t unit, int64_t ctas) {
+    const int64_t fit = (kStageFloats - fixed) / per_plane;
+    if (fit < unit) return 0;
+    int64_t g = std::min<int64_t>(fit, std::max<int64_t>(1, NC / (4 * ctas)));
+    g = std::max<int64_t>(unit, g / unit * unit);
+    return (int32_t)g;
+}
+
+size_t ring_smem(bool nibble_bytes) { return (size_t)kRS * kStageBytes + (nibble_bytes ? kNbBytes : 0) + 64; }
+
+}  // namespace
+
+// Used for stride 1 (GoogLeNet's in-module pools): forward 16% -> 28% of HBM, backward 12% -> 21%
+// (inc3a b64, isolated).  The stride-2 path is kept for GIST_POOL3_S2=1 only: the L1 kernels of
+// pool.cu measured faster there (AlexNet relu1 b128 forward 52% vs 39%, backward 36% vs 30%).
+#ifndef GIST_POOL3_S2
+#define GIST_POOL3_S2 0
+#endif
+bool pool3_ok(const gist_pool2d &p) {
+    return p.kh == 3 && p.kw == 3 && p.sh == p.sw && (p.sh == 1 || (GIST_POOL3_S2 && p.sh == 2)) && p.ph == p.pw &&
+           p.ph <= 1;
+}
+
+// Forward (+ the a1 mask when mask != NULL, + relu on load when relu).  Returns cudaErrorNotSupported
+// when a plane does not fit a stage (the caller uses the generic kernels).
+cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p,
+                             int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, uint32_t *mask, bool relu,
+                             cudaStream_t s) {
+    P3Args a = p3_args(N, C, H, W, p, Ho, Wo);
+    const int64_t ctas = 2 * (int64_t)num_sms();
+    if (a.S == 1) {
+        // whole argmax (and mask) words per tile; the nibble bytes of a tile fit kNbBytes
+        int32_t unit = 8 / gcd_i(a.HoWo, 8);
+        if (mask) {
+            const int32_t mu = 32 / gcd_i(a.HW, 32);
+            unit = unit * mu / gcd_i(unit, mu);
+        }
+        a.G = choose_g(a.NC, a.HW, 64, unit, ctas);
+        while (a.G > unit && (int64_t)a.G * a.HoWo > kNbBytes) a.G -= unit;
+        if (a.G == 0 || (int64_t)a.G * a.HoWo > kNbBytes) return cudaErrorNotSupported;
+    } else {
+        // rows of the next plane a tile may need: the windows of its last argmax word's (<= 7)
+        // outputs there, and the (<= 31) elements of its last mask word
+        int32_t xr = 0;
+        if (a.HoWo % 8) xr = std::min(H, (std::min(6, a.HoWo - 1) / Wo) * a.S - a.P + 3);
+        if (mask && a.HW % 32) xr = std::max(xr, std::min(H, (30 + W) / W));
+        a.xrows = xr;
+        a.G = choose_g(a.NC, a.HW, 64 + (int64_t)xr * W + 32, 1, ctas);
+        if (a.G == 0) return cudaErrorNotSupported;
+    }
+    a.tiles = ceil_div(a.NC, a.G);
+    // every window inside the input: no bounds tests (AlexNet's floor-mode 3x3/s2)
+    const bool check = !(a.P == 0 && (Ho - 1) * a.S + 3 <= H && (Wo - 1) * a.S + 3 <= W);
+    const size_t smem = ring_smem(a.S == 1);
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(a.tiles, ctas));
+#define P3F(S_, M_, R_, C_)                                                                                 \
+    do {                                                                                                    \
+        static PerDeviceAttr attr;                                                                          \
+        const cudaError_t e =                                                                               \
+            attr.ensure(reinterpret_cast<const void *>(pool3_fwd_kernel<S_, M_, R_, C_>), (int)smem);       \
+        if (e != cudaSuccess) return e;                                                                     \
+        launch_k(pool3_fwd_kernel<S_, M_, R_, C_>, grid, kRT, smem, s, y, a, out, argmax, mask);            \
+    } while (0)
+    const bool m = mask != nullptr;
+    if (a.S == 1) {
+        if (m) {
+            if (relu) P3F(1, true, true, true); else P3F(1, true, false, true);
+        } else {
+            if (relu) P3F(1, false, true, true); else P3F(1, false, false, true);
+        }
+    } else if (check) {
+        if (m) {
+            if (relu) P3F(2, true, true, true); else P3F(2, true, false, true);
+        } else {
+            if (relu) P3F(2, false, true, true); else P3F(2, false, false, true);
+        }
+    } else {
+        if (m) {
+            if (relu) P3F(2, true, true, false); else P3F(2, true, false, false);
+        } else {
+            if (relu) P3F(2, false, true, false); else P3F(2, false, false, false);
+        }
+    }
+#undef P3F
+    return cudaPeekAtLastError();
+}
+
+cudaError_t launch_pool3_bwd(const float *dout, const uint32_t *argmax, const uint32_t *mask, int32_t N, int32_t C,
+                             int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo, float *dx,
+                             cudaStream_t s) {
+    P3Args a = p3_args(N, C, H, W, p, Ho, Wo);
+    const int64_t ctas = 2 * (int64_t)num_sms();
+    if (a.S == 2) {
+        a.hb = (H + a.P + 1) / 2;
+        a.wb = (W + a.P + 1) / 2;
+        a.div_blk = FastDiv::make((uint32_t)(a.hb * a.wb));
+        a.div_wb = FastDiv::make((uint32_t)a.wb);
+        a.PR = std::max(Ho, a.hb) + 1;
+        a.PC = std::max(Wo, a.wb) + 1;
+    } else {
+        a.PR = Ho + 4;
+        a.PC = Wo + 4;
+    }
+    // stage floats per plane: dY (HoWo) + argmax words (HoWo/8) + mask words (HW/32), and the
+    // phases / round-ups of the three ranges
+    const int64_t per_plane = (int64_t)a.HoWo + (a.HoWo + 7) / 8 + (mask ? (a.HW + 31) / 32 : 0) + 1;
+    a.G = choose_g(a.NC, per_plane, 64, 1, ctas);
+    while (a.G > 1 && (int64_t)a.G * a.PR * a.PC > kNbBytes) --a.G;
+    if (a.G == 0 || (int64_t)a.G * a.PR * a.PC > kNbBytes) return cudaErrorNotSupported;
+    a.tiles = ceil_div(a.NC, a.G);
+    const int64_t G = a.G;
+    a.a_off = (int32_t)((G * a.HoWo + 8 + 3) & ~3ll);
+    a.m_off = (int32_t)((a.a_off + (G * a.HoWo + 7) / 8 + 8 + 3) & ~3ll);
+    const size_t smem = ring_smem(true);
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(a.tiles, ctas));
+#define P3B(S_, M_)                                                                                          \
+    do {                                                                                                     \
+        static PerDeviceAttr attr;                                                                           \
+        const cudaError_t e = attr.ensure(reinterpret_cast<const void *>(pool3_bwd_kernel<S_, M_>), (int)smem); \
+        if (e != cudaSuccess) return e;                                                                      \
+        launch_k(pool3_bwd_kernel<S_, M_>, grid, kRT, smem, s, dout, argmax, mask, a, dx);                   \
+    } while (0)
+    if (a.S == 1) {
+        if (mask) P3B(1, true); else P3B(1, false);
+    } else {
+        if (mask) P3B(2, true); else P3B(2, false);
+    }
+#undef P3B
+    return cudaPeekAtLastError();
+}
+
+}  // namespace gist
