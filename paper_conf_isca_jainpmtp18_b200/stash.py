@@ -8,8 +8,12 @@ long forward->backward gap (Fig 2).  Here the same schedule is expressed 
   a2 kernel with the a1 mask fused; autograd saves ONLY the 1-bit mask and the 4-bit argmax
   map (neither the ReLU output nor the pool output), and the backward is the a3 kernel.
 * `relu_conv(x, conv)` / `stashed_conv(y, conv)` — ReLU->Conv and Pool->Conv (SSDC,
-  P:158-164): the conv input is stashed as exact-size 256-column CSR (a4) and densified just
-  before the conv backward (a5); the dense math stays in cuDNN ("dense compute").
+  P:158-164): the conv input is stashed as 256-column CSR (a4) and densified just before the
+  conv backward (a5); the dense math stays in cuDNN ("dense compute").  Inside
+  `ssdc_arena(...)` every stash appends its entries to one chained arena in a single encode
+  pass with device-side offsets (no host synchronization in the forward; one capacity check
+  per step, before the first decode); outside it, each stash is sized exactly by a count pass
+  and a host read of nnz.
 * `dpr_saved_tensors(bits, params)` — every other stashed activation (DPR,
   "applicable to any layer combination") is packed to FP16/FP10/FP8 by the a6 kernel when
   autograd saves it and restored by a7 when the backward unpacks it.
@@ -24,7 +28,8 @@ import torch
 import torch.nn.functional as F
 
 from . import (gist_dpr_decode, gist_dpr_encode, gist_relu_maxpool_fwd_argmax, gist_pool_relu_bwd,
-               gist_ssdc_decode, gist_ssdc_encode, gist_ssdc_rows, gist_ssdc_workspace)
+               gist_ssdc_decode, gist_ssdc_decode_many, gist_ssdc_encode, gist_ssdc_rows, gist_ssdc_workspace,
+               gist_ssdc_workspace_bytes, gist_ssdc_workspace_init, SsdcEncodeMany)
 
 
 def _pool_tuple(kernel_size, stride, padding, ceil_mode):
@@ -55,12 +60,83 @@ def relu_maxpool(x, kernel_size, stride=None, padding=0, ceil_mode=False):
     return _ReLUMaxPool.apply(x, _pool_tuple(kernel_size, stride, padding, ceil_mode))
 
 
+class StashOverflow(RuntimeError):
+    """The step's SSDC entries did not fit the arena; `needed` is the entry count it would take."""
+
+    def __init__(self, needed: int, capacity: int):
+        super().__init__(f"SSDC stash arena overflow: {needed} entries needed, capacity {capacity}")
+        self.needed, self.capacity = needed, capacity
+
+
+class StashArena:
+    """One chained SSDC arena for a training step (the Schedule
+    Builder's preallocated stash): each stash's col/val entries follow the previous stash's, the
+    start offset is a device scalar (the previous encode's nnz output), so an encode is ONE pass
+    over the map with no host synchronization.  Entries past `capacity` are dropped by the kernel
+    (which still publishes the true end); `check()` reads the end once and raises StashOverflow
+    before any stash of an overflowed arena is decoded."""
+
+    def __init__(self, capacity: int, device):
+        self.capacity, self.device = int(capacity), torch.device(device)
+        self.col = torch.empty(max(1, self.capacity), dtype=torch.uint8, device=self.device)
+        self.val = torch.empty(max(1, self.capacity), dtype=torch.float32, device=self.device)
+        self.ws = None
+        self.reset()
+
+    def reset(self):
+        self.head = torch.zeros(1, dtype=torch.int64, device=self.device)
+        self.used = None  # host value once checked
+
+    def _workspace(self, n: int) -> torch.Tensor:
+        need = gist_ssdc_workspace_bytes(n)
+        if self.ws is None or self.ws.numel() < need:
+            self.ws = torch.empty(need, dtype=torch.uint8, device=self.device)
+            gist_ssdc_workspace_init(self.ws)
+        return self.ws
+
+    def append(self, y: torch.Tensor):
+        """Encode y after the current end; returns (row_end, start, end) (start/end on the device)."""
+        n = y.numel()
+        start, end = self.head, torch.empty(1, dtype=torch.int64, device=self.device)
+        row_end = torch.empty(gist_ssdc_rows(n), dtype=torch.int32, device=self.device)
+        SsdcEncodeMany([{"x": y, "row_end": row_end, "col": self.col, "val": self.val, "capacity": self.capacity,
+                         "offset": start, "nnz": end}], workspace=self._workspace(n))()
+        self.head = end
+        return row_end, start, end
+
+    def check(self) -> int:
+        """Entries used by the step (one host read per reset); raises StashOverflow."""
+        if self.used is None:
+            self.used = int(self.head.item())
+        if self.used > self.capacity:
+            raise StashOverflow(self.used, self.capacity)
+        return self.used
+
+
+_ARENA: list = []
+
+
+@contextlib.contextmanager
+def ssdc_arena(arena: StashArena):
+    """Stashes made inside this context append to `arena` (one encode pass each, no host sync)."""
+    _ARENA.append(arena)
+    try:
+        yield arena
+    finally:
+        _ARENA.pop()
+
+
 class CSRStash:
-    """Exact-size SSDC encoding of a dense fp32 map (one count pass, one encode pass)."""
+    """SSDC encoding of a dense fp32 map: appended to the active arena (one pass), else exact-size
+    (one count pass, a host read of nnz, one encode pass)."""
 
     def __init__(self, y: torch.Tensor):
         y = y.contiguous()
         self.shape, self.n = tuple(y.shape), y.numel()
+        self.arena = _ARENA[-1] if _ARENA else None
+        if self.arena is not None:
+            self.row_end, self.start, self.end = self.arena.append(y)
+            return
         ws = gist_ssdc_workspace(self.n, y.device)
         nnz = torch.empty(1, dtype=torch.int64, device=y.device)
         row_end = torch.empty(gist_ssdc_rows(self.n), dtype=torch.int32, device=y.device)
@@ -72,9 +148,16 @@ class CSRStash:
         self.row_end, self.col, self.val, self.nnz = row_end, col, val, k
 
     def nbytes(self) -> int:
-        return 5 * self.nnz + 4 * self.row_end.numel()
+        """Encoded bytes (5 nnz + 4 rows); reads the arena offsets (a host sync) in arena mode."""
+        nnz = int((self.end - self.start).item()) if self.arena is not None else self.nnz
+        return 5 * nnz + 4 * self.row_end.numel()
 
     def dense(self) -> torch.Tensor:
+        if self.arena is not None:
+            self.arena.check()  # never decode entries an overflowed arena dropped
+            (x,) = gist_ssdc_decode_many([{"row_end": self.row_end, "col": self.arena.col, "val": self.arena.val,
+                                           "offset": self.start, "n": self.n}])
+            return x.view(self.shape)
         return gist_ssdc_decode(self.row_end, self.col, self.val, self.n).view(self.shape)
 
 

@@ -23,6 +23,9 @@ import torch.nn.functional as F  # noqa: E402
 from paper_conf_isca_jainpmtp18_b200 import stash  # noqa: E402
 
 CFG = [(3, 64, 2), (64, 128, 2), (128, 256, 3), (256, 512, 3), (512, 512, 3)]
+# SSDC-stashed maps per image in forward_gist: (channels, side) of every relu->conv and pool->conv input
+SSDC_SHAPES = [(cout, 224 >> b) for b, (_, cout, k) in enumerate(CFG) for _ in range(k - 1)] + \
+    [(cin, 224 >> b) for b, (cin, _, _) in enumerate(CFG) if b > 0]
 
 
 class VGG16(nn.Module):
@@ -48,10 +51,14 @@ class VGG16(nn.Module):
         x = F.relu(self.fc7(x))
         return self.fc8(x)
 
-    def forward_gist(self, x, bits, lossless=False):
-        # DPR (lossy) wraps everything; the Binarize/SSDC functions save only their encodings
+    def forward_gist(self, x, bits, lossless=False, arena=None):
+        # DPR (lossy) wraps everything; the Binarize/SSDC functions save only their encodings;
+        # with an arena the SSDC stashes are single-pass appends (no host sync in the forward)
         ctx = stash.dpr_saved_tensors(bits, self.parameters()) if not lossless else _null()
-        with ctx:
+        actx = stash.ssdc_arena(arena) if arena is not None else _null()
+        if arena is not None:
+            arena.reset()
+        with ctx, actx:
             c = 0
             z = self.convs[0](x)  # the input image: an "other" stashed map (DPR)
             c = 1
@@ -80,7 +87,23 @@ class _null:
 
 def step(model, x, target, fwd, marks=None):
     model.zero_grad(set_to_none=True)
-    loss = F.cross_entropy(fwd(x), target)
+    try:
+        loss = F.cross_entropy(fwd(x), target)
+        return _finish(loss, marks)
+    except stash.StashOverflow as e:  # the arena was too small: grow it (once) and redo the step
+        if ARENA.get("arena") is None:
+            raise
+        ARENA["arena"] = stash.StashArena(int(e.needed * 1.05), x.device)
+        ARENA["grown"] = ARENA.get("grown", 0) + 1
+        model.zero_grad(set_to_none=True)
+        loss = F.cross_entropy(fwd(x), target)
+        return _finish(loss, marks)
+
+
+ARENA = {}
+
+
+def _finish(loss, marks):
     if marks is not None:  # the stash: everything alive between the forward and the backward
         torch.cuda.synchronize()
         marks["after_forward_bytes"] = torch.cuda.memory_allocated()
@@ -122,6 +145,8 @@ def main():
     ap.add_argument("--bits", type=int, default=16)
     ap.add_argument("--lossless", action="store_true", help="Binarize + SSDC only (no DPR)")
     ap.add_argument("--json", default=None)
+    ap.add_argument("--no-arena", dest="arena", action="store_false",
+                    help="exact-size SSDC stashes (count pass + host read of nnz per conv) instead of the arena")
     ap.add_argument("--cap-gb", type=float, default=None,
                     help="largest-minibatch mode: cap the process at this many GB (P:38: Gist fits larger "
                          "minibatches) and search the largest batch each arm can train")
@@ -190,13 +215,20 @@ def main():
 
     base = measure(model, x, target, model.forward_baseline)
     g_base = [p.grad.clone() for p in model.parameters()]
-    gist = measure(model, x, target, lambda t: model.forward_gist(t, args.bits, args.lossless))
+    if args.arena:  # start at half the SSDC-stashed elements; an overflow grows it once
+        n_ssdc = sum(x.shape[0] * c * h * h for c, h in SSDC_SHAPES)
+        ARENA["arena"] = stash.StashArena(n_ssdc // 2, dev)
+    gist = measure(model, x, target, lambda t: model.forward_gist(t, args.bits, args.lossless, ARENA.get("arena")))
     g_gist = [p.grad for p in model.parameters()]
     rel = max(float((a - b).abs().max() / (a.abs().max() + 1e-30)) for a, b in zip(g_base, g_gist))
     out = {
         "model": "VGG16 random init", "batch": args.batch, "image": 224,
         "encodings": "Binarize + SSDC" + ("" if args.lossless else f" + DPR-fp{args.bits}"),
         "baseline": base, "gist": gist,
+        "ssdc_stash": ({"mode": "arena (one encode pass per stash, no host sync in the forward)",
+                        "capacity_entries": ARENA["arena"].capacity, "used_entries": ARENA["arena"].check(),
+                        "grown": ARENA.get("grown", 0)} if args.arena else
+                       {"mode": "exact-size (count pass + host read of nnz + encode pass per stash)"}),
         "mfr_peak": round(base["peak_bytes"] / gist["peak_bytes"], 3),
         "mfr_above_inputs": round(base["peak_above_inputs_bytes"] / gist["peak_above_inputs_bytes"], 3),
         "stash_ratio": round(base["stash_bytes"] / gist["stash_bytes"], 3),

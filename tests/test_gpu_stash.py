@@ -85,3 +85,53 @@ def test_csr_stash_is_exact_and_small(gist, cuda):
     s = stash.CSRStash(y)
     assert torch.equal(s.dense().view(torch.int32), y.view(torch.int32))
     assert s.nbytes() < 0.3 * 4 * y.numel()
+
+
+def test_arena_stash_one_pass_no_sync_bit_exact(gist, cuda, deterministic):
+    """f2 single pass: inside ssdc_arena every stash is ONE encode into a chained arena with
+    device-side offsets.  The forward runs under torch's sync debug mode set to "error" (any host
+    synchronization raises), and the gradients still equal plain PyTorch's bit for bit."""
+    from paper_conf_isca_jainpmtp18_b200 import stash
+    torch.manual_seed(0)
+    m = TinyVGG().to(cuda)
+    x = torch.randn(8, 3, 32, 32, device=cuda)
+    y = torch.randint(0, 10, (8,), device=cuda)
+    g0 = grads(m, m.base, x, y)
+    arena = stash.StashArena(8 * 16 * 32 * 32 * 4, cuda)  # >= every SSDC-stashed element of the step
+    launches0 = gist.gist_launch_count()
+    m.zero_grad(set_to_none=True)
+    torch.cuda.synchronize()
+    with stash.ssdc_arena(arena):
+        torch.cuda.set_sync_debug_mode("error")
+        try:
+            logits = m.gist(x, stash)
+        finally:
+            torch.cuda.set_sync_debug_mode("default")
+    assert gist.gist_launch_count() - launches0 >= 3  # the three SSDC stashes were encoded
+    F.cross_entropy(logits, y).backward()
+    g1 = [p.grad.clone() for p in m.parameters()]
+    for (name, _), a, b in zip(m.named_parameters(), g0, g1):
+        assert torch.equal(a.view(torch.int32), b.view(torch.int32)), name
+    used = arena.check()
+    # the arena holds exactly the nonzeros of the three stashed maps
+    assert 0 < used <= arena.capacity
+
+
+def test_arena_overflow_is_reported_before_decode(gist, cuda):
+    from paper_conf_isca_jainpmtp18_b200 import stash
+    y = torch.relu(torch.randn(2, 16, 32, 32, device=cuda))
+    arena = stash.StashArena(100, cuda)  # far too small
+    with stash.ssdc_arena(arena):
+        s = stash.CSRStash(y)
+    with pytest.raises(stash.StashOverflow) as e:
+        s.dense()
+    assert e.value.needed == int((y.view(torch.int32) != 0).sum().item())
+    # a fresh arena large enough round-trips exactly, and reset() reuses it
+    arena = stash.StashArena(y.numel(), cuda)
+    for _ in range(2):
+        arena.reset()
+        with stash.ssdc_arena(arena):
+            s = stash.CSRStash(y)
+            s2 = stash.CSRStash(2 * y)
+        assert torch.equal(s.dense().view(torch.int32), y.view(torch.int32))
+        assert torch.equal(s2.dense().view(torch.int32), (2 * y).view(torch.int32))
