@@ -274,7 +274,8 @@ gist_status gist_dpr_decode_many(const gist_dpr_job *jobs, int32_t count, int32_
  *           fp32: every product within ~2^-19 relative of the fp32 product); 1: TF32 products (inputs
  *           truncated to 10-bit mantissas), fp32 accumulation.  Deterministic (fixed split-K order).
  *   workspace [>= gist_conv3x3_wgrad_workspace_bytes(...)] device bytes (split-K partials).
- * UNSUPPORTED unless Co % 128 == 0, Ci % 16 == 0, H*W % 4 == 0 (dY rows are TMA rows), W <= 252,
+ * UNSUPPORTED unless Co % 128 == 0, Ci % 16 == 0, H*W % 4 == 0 (dY rows are TMA rows), W <= 252 and
+ * the two decode slabs (16 x (R+2) x (W+2) floats each, R ~ 256/W rows) fit shared memory (W <= ~190),
  * passes in {1, 3};
  * TOO_LARGE if N*Ci*H*W or N*Co*H*W >= 2^31. */
 size_t gist_conv3x3_wgrad_workspace_bytes(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W);

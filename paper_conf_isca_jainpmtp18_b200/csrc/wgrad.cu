@@ -38,12 +38,16 @@ constexpr int kTaps = 9;                // 3x3 window
 constexpr int kN = kCiBlk * kTaps;      // 144 GEMM columns: n = tap * 16 + ci
 constexpr int kM = 128;                 // output channels per CTA tile (UMMA M)
 constexpr int kKs = 32;                 // K per pipeline stage = one 128-byte swizzle row of fp32
-constexpr int kProdWarps = 8;
-constexpr int kProdThreads = 32 * kProdWarps;
+constexpr int kBldWarps = 4;                 // operand builders: B = im2col(X) (hi/lo) and A_lo
+constexpr int kBldThreads = 32 * kBldWarps;  // one thread per (ci, 4-position chunk) of a stage
+constexpr int kDecWarps = 4;                 // decoders: CSR rows of X -> the next K-tile's slab
+constexpr int kDecThreads = 32 * kDecWarps;
+constexpr int kBld0 = 2, kDec0 = kBld0 + kBldWarps;
 constexpr int kEpiWarps = 8;                 // two per TMEM lane quarter (taps 0-4 / 5-8)
-constexpr int kEpi0 = 2 + kProdWarps;        // first epilogue warp
-// warp 0: TMA + TMEM owner, warp 1: MMA, 2..9: producers, 10..17: accumulator drain (epilogue)
+constexpr int kEpi0 = kDec0 + kDecWarps;     // first epilogue warp
+// warp 0: TMA + TMEM owner, warp 1: MMA, 2..5: builders, 6..9: decoders, 10..17: accumulator drain
 constexpr int kThreads = 32 * (kEpi0 + kEpiWarps);
+static_assert(kBldThreads == kCiBlk * (kKs / 4), "one builder thread per (ci, chunk)");
 constexpr int kTmemCols = 512;               // two accumulators (K-tile t uses columns 256 (t % 2) + n)
 constexpr int kAccStride = 256;
 constexpr uint32_t kIdesc = idesc_tf32<kM, kN>();
@@ -63,6 +67,8 @@ struct WgArgs {
     int32_t chunk;    // K-tiles per partial (the fp32 register accumulation spans at most this many)
     int32_t units;    // partials per output tile = ceil(T / chunk)
     int64_t T;        // K-tiles in total = N * ktiles
+    int32_t SWP;      // slab row pitch (W + 2 halo columns, rounded up to a multiple of 4)
+    int32_t slab_floats;  // one slab buffer: kCiBlk * (R + 2) * SWP
     FastDiv div_w;
 };
 
@@ -73,12 +79,19 @@ struct __align__(1024) WgSmem {
     float bhi[STAGES][kN * kKs];                    // im2col(X) tiles, same layout
     float blo[PASSES == 3 ? STAGES : 1][PASSES == 3 ? kN * kKs : 256];
     uint64_t a_full[STAGES], b_full[STAGES], empty[STAGES], acc_full[2], acc_empty[2];
+    uint64_t slab_full[2], slab_empty[2];  // decoders -> builders, builders -> decoders (per slab buffer)
     uint32_t tmem_base;
 };
 // every operand tile must start on a 1024-byte boundary (the 128-byte swizzle atom)
 static_assert(sizeof(float) * kM * kKs % 1024 == 0 && sizeof(float) * kN * kKs % 1024 == 0, "tile sizes");
 
-template <int PASSES, int STAGES>
+// Long waits (the TMA lane on a free stage, the epilogue on a finished period, the decoders on a
+// free slab) back off instead of spinning on the issue slots the builders need.
+__device__ __forceinline__ void wait_backoff(uint64_t *bar, uint32_t parity) {
+    while (!mbar_test(bar, parity)) __nanosleep(64);
+}
+
+template <int PASSES, int STAGES, bool VEC>
 __global__ void __launch_bounds__(kThreads, 1)
 wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
     using Smem = WgSmem<PASSES, STAGES>;
@@ -86,7 +99,7 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
     // the 128-byte swizzle repeats every 1024 bytes: align the tiles to that
     const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
     Smem &S = *reinterpret_cast<Smem *>(smem_raw + pad);
-    float *slab = reinterpret_cast<float *>(smem_raw + pad + sizeof(Smem));
+    float *slabs = reinterpret_cast<float *>(smem_raw + pad + sizeof(Smem));  // two slab buffers
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
     const int nb = blockIdx.x % a.n_blocks;
@@ -97,17 +110,19 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
     const int64_t t0 = u0 * a.chunk, t1 = min(a.T, u1 * (int64_t)a.chunk);
     const int co0 = mb * kM, ci0 = nb * kCiBlk;
     const int64_t nst = (t1 - t0) * a.spt;  // pipeline stages of this CTA
-    const int RW = a.R * a.W, SW = a.W + 2, SR = a.R + 2;
+    const int RW = a.R * a.W, SW = a.SWP, SR = a.R + 2;
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(&S.a_full[s], 1);
-            mbar_init(&S.b_full[s], kProdWarps);
+            mbar_init(&S.b_full[s], kBldWarps);
             mbar_init(&S.empty[s], 1);
         }
         for (int b = 0; b < 2; ++b) {
             mbar_init(&S.acc_full[b], 1);
             mbar_init(&S.acc_empty[b], kEpiWarps);
+            mbar_init(&S.slab_full[b], kDecWarps);
+            mbar_init(&S.slab_empty[b], kBldWarps);
         }
         fence_mbar_init();
     }
@@ -129,7 +144,7 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
             prefetch_tmap(&tmap_dy);
             for (int64_t g = 0; g < nst; ++g) {
                 const int st = (int)(g % STAGES);
-                if (g >= STAGES) mbar_wait(&S.empty[st], (uint32_t)((g / STAGES) - 1) & 1u);
+                if (g >= STAGES) wait_backoff(&S.empty[st], (uint32_t)((g / STAGES) - 1) & 1u);
                 const int64_t t = t0 + g / a.spt;
                 const int j = (int)(g % a.spt);
                 const int n = (int)(t / a.ktiles), ty = (int)(t % a.ktiles);
@@ -190,7 +205,7 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
         const int64_t nper = (t1 - t0) * a.pp;
         for (int64_t gp = 0; gp < nper; ++gp) {
             const int b = (int)(gp & 1);
-            mbar_wait(&S.acc_full[b], (uint32_t)(gp / 2) & 1u);
+            wait_backoff(&S.acc_full[b], (uint32_t)(gp / 2) & 1u);
             tc_fence_after();
 #pragma unroll
             for (int i = 0; i < 5; ++i) {
@@ -224,26 +239,27 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                 }
             }
         }
-    } else {
-        // ---- producers: decode X (SSDC) into the slab, build B (im2col, hi/lo) and A_lo
-        const int p = threadIdx.x - 64;
-        const int wp = warp - 2;
-        const int ci_b = p >> 4, ch = (p >> 1) & 7, half = p & 1;  // B chunk owned by this thread
+    } else if (warp >= kDec0) {
+        // ---- decoders: for each K-tile t of this CTA, the input rows [oh0-1, oh0+R] of its image for
+        // the 16 channels, zero-filled then scattered from the CSR rows that cover them, into slab
+        // buffer (t - t0) % 2 while the builders read the other one
+        const int dp = threadIdx.x - 32 * kDec0, dw = warp - kDec0;
         for (int64_t t = t0; t < t1; ++t) {
+            const int64_t tl = t - t0;
+            const int sb = (int)(tl & 1);
+            if (tl >= 2) wait_backoff(&S.slab_empty[sb], (uint32_t)((tl / 2) - 1) & 1u);
+            float *slab = slabs + (size_t)sb * a.slab_floats;
             const int n = (int)(t / a.ktiles), ty = (int)(t % a.ktiles);
             const int oh0 = ty * a.R;
-            named_bar(1, kProdThreads);  // every producer is done reading the previous slab
             {
                 float4 *s4 = reinterpret_cast<float4 *>(slab);
-                const int n4 = kCiBlk * SR * SW / 4;
-                for (int i = p; i < n4; i += kProdThreads) s4[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+                for (int i = dp; i < a.slab_floats / 4; i += kDecThreads) s4[i] = make_float4(0.f, 0.f, 0.f, 0.f);
             }
-            named_bar(1, kProdThreads);
-            // each warp decodes two channels: the CSR rows covering input rows [oh0-1, oh0+R]
-            for (int cc = 0; cc < 2; ++cc) {
-                const int ci = 2 * wp + cc;
+            named_bar(2, kDecThreads);  // the buffer is zero before any scatter
+            const int ih_lo = max(0, oh0 - 1), ih_hi = min(a.H, oh0 + a.R + 1);
+            for (int cc = 0; cc < kCiBlk / kDecWarps; ++cc) {
+                const int ci = dw * (kCiBlk / kDecWarps) + cc;
                 const int64_t plane0 = ((int64_t)n * a.Ci + ci0 + ci) * a.H * a.W;
-                const int ih_lo = max(0, oh0 - 1), ih_hi = min(a.H, oh0 + a.R + 1);
                 const int64_t F0 = plane0 + (int64_t)ih_lo * a.W, F1 = plane0 + (int64_t)ih_hi * a.W;
                 if (F1 <= F0) continue;
                 float *sl = slab + (size_t)ci * SR * SW;
@@ -259,49 +275,83 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                     }
                 }
             }
-            named_bar(1, kProdThreads);
+            __syncwarp();
+            if (lane == 0) mbar_arrive_1(&S.slab_full[sb]);
+        }
+    } else {
+        // ---- builders: per stage, B rows (tap, ci) x 32 positions from the slab (hi and lo parts) and
+        // A_lo; thread p owns channel ci_b and the 4-position chunk ch of every stage
+        const int p = threadIdx.x - 32 * kBld0;
+        const int ci_b = p >> 3, ch = p & 7;
+        for (int64_t t = t0; t < t1; ++t) {
+            const int64_t tl = t - t0;
+            const int sb = (int)(tl & 1);
+            mbar_wait(&S.slab_full[sb], (uint32_t)(tl / 2) & 1u);
+            const float *slab = slabs + (size_t)sb * a.slab_floats;
+            const int oh0 = (int)(t % a.ktiles) * a.R;
             for (int j = 0; j < a.spt; ++j) {
-                const int64_t g = (t - t0) * a.spt + j;
+                const int64_t g = tl * a.spt + j;
                 const int st = (int)(g % STAGES);
                 if (g >= STAGES) mbar_wait(&S.empty[st], (uint32_t)((g / STAGES) - 1) & 1u);
-                // B rows (tap, ci_b), chunk ch = output positions pos .. pos+3 of the K-tile (they may
-                // straddle an output row when W % 4 != 0); slab offset of each for tap (0, 0)
-                const int pos = j * kKs + 4 * ch;
+                const int pos = j * kKs + 4 * ch;  // the chunk's first position in the K-tile
                 uint32_t ohr = 0, ow = 0;
                 a.div_w.divmod((uint32_t)pos, ohr, ow);
-                int off[4];
-                bool ok[4];
-#pragma unroll
-                for (int e = 0; e < 4; ++e) {
-                    ok[e] = pos + e < RW && oh0 + (int)ohr < a.H;
-                    off[e] = ((ci_b * SR) + (int)ohr) * SW + (int)ow;
-                    if (++ow == (uint32_t)a.W) {
-                        ow = 0;
-                        ++ohr;
-                    }
-                }
                 unsigned char *bh = reinterpret_cast<unsigned char *>(S.bhi[st]);
                 unsigned char *bl = reinterpret_cast<unsigned char *>(S.blo[PASSES == 3 ? st : 0]);
+                if constexpr (VEC) {
+                    // W % 4 == 0: the chunk lies in one output row at ow % 4 == 0; slab row kh holds the
+                    // 6 inputs (cols ow .. ow+5) of its 3 taps: two 16-byte loads
+                    const bool valid = pos < RW && oh0 + (int)ohr < a.H;
+                    const float *src = slab + ((size_t)ci_b * SR + ohr) * SW + ow;
 #pragma unroll
-                for (int i = 0; i < 5; ++i) {
-                    const int tap = half ? 5 + i : i;
-                    if (tap >= kTaps) break;
-                    const int kh = tap / 3, kw = tap % 3;
-                    float v[4];
+                    for (int kh = 0; kh < 3; ++kh) {
+                        float4 l0 = make_float4(0.f, 0.f, 0.f, 0.f), l1 = l0;
+                        if (valid) {
+                            l0 = *reinterpret_cast<const float4 *>(src + kh * SW);
+                            l1 = *reinterpret_cast<const float4 *>(src + kh * SW + 4);
+                        }
+                        const float v[6] = {l0.x, l0.y, l0.z, l0.w, l1.x, l1.y};
+                        float hi[6], lo[6];
 #pragma unroll
-                    for (int e = 0; e < 4; ++e) v[e] = ok[e] ? slab[off[e] + kh * SW + kw] : 0.0f;
-                    const uint32_t off = sw128_offset((uint32_t)(tap * kCiBlk + ci_b), (uint32_t)ch);
-                    if constexpr (PASSES == 3) {
-                        float hi[4], lo[4];
-#pragma unroll
-                        for (int e = 0; e < 4; ++e) {
-                            hi[e] = to_tf32(v[e]);
+                        for (int e = 0; e < 6; ++e) {
+                            hi[e] = PASSES == 3 ? to_tf32(v[e]) : v[e];
                             lo[e] = v[e] - hi[e];
                         }
-                        *reinterpret_cast<float4 *>(bh + off) = make_float4(hi[0], hi[1], hi[2], hi[3]);
-                        *reinterpret_cast<float4 *>(bl + off) = make_float4(lo[0], lo[1], lo[2], lo[3]);
-                    } else {
-                        *reinterpret_cast<float4 *>(bh + off) = make_float4(v[0], v[1], v[2], v[3]);
+#pragma unroll
+                        for (int kw = 0; kw < 3; ++kw) {
+                            const uint32_t off = sw128_offset((uint32_t)((3 * kh + kw) * kCiBlk + ci_b), (uint32_t)ch);
+                            *reinterpret_cast<float4 *>(bh + off) = make_float4(hi[kw], hi[kw + 1], hi[kw + 2], hi[kw + 3]);
+                            if constexpr (PASSES == 3)
+                                *reinterpret_cast<float4 *>(bl + off) = make_float4(lo[kw], lo[kw + 1], lo[kw + 2], lo[kw + 3]);
+                        }
+                    }
+                } else {
+                    // any W: the 4 positions may straddle an output row; slab offset of each for tap (0, 0)
+                    int off[4];
+                    bool ok[4];
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) {
+                        ok[e] = pos + e < RW && oh0 + (int)ohr < a.H;
+                        off[e] = ((ci_b * SR) + (int)ohr) * SW + (int)ow;
+                        if (++ow == (uint32_t)a.W) {
+                            ow = 0;
+                            ++ohr;
+                        }
+                    }
+#pragma unroll
+                    for (int tap = 0; tap < kTaps; ++tap) {
+                        const int kh = tap / 3, kw = tap % 3;
+                        float v[4], hi[4], lo[4];
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) {
+                            v[e] = ok[e] ? slab[off[e] + kh * SW + kw] : 0.0f;
+                            hi[e] = PASSES == 3 ? to_tf32(v[e]) : v[e];
+                            lo[e] = v[e] - hi[e];
+                        }
+                        const uint32_t o = sw128_offset((uint32_t)(tap * kCiBlk + ci_b), (uint32_t)ch);
+                        *reinterpret_cast<float4 *>(bh + o) = make_float4(hi[0], hi[1], hi[2], hi[3]);
+                        if constexpr (PASSES == 3)
+                            *reinterpret_cast<float4 *>(bl + o) = make_float4(lo[0], lo[1], lo[2], lo[3]);
                     }
                 }
                 if constexpr (PASSES == 3) {
@@ -311,17 +361,19 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                     float4 *ar = reinterpret_cast<float4 *>(S.a[st]);
                     float4 *al = reinterpret_cast<float4 *>(S.alo[st]);
 #pragma unroll
-                    for (int i = 0; i < kM * kKs / 4 / kProdThreads; ++i) {
-                        const float4 x = ar[p + i * kProdThreads];
+                    for (int i = 0; i < kM * kKs / 4 / kBldThreads; ++i) {
+                        const float4 x = ar[p + i * kBldThreads];
                         const float4 h = make_float4(to_tf32(x.x), to_tf32(x.y), to_tf32(x.z), to_tf32(x.w));
-                        ar[p + i * kProdThreads] = h;
-                        al[p + i * kProdThreads] = make_float4(x.x - h.x, x.y - h.y, x.z - h.z, x.w - h.w);
+                        ar[p + i * kBldThreads] = h;
+                        al[p + i * kBldThreads] = make_float4(x.x - h.x, x.y - h.y, x.z - h.z, x.w - h.w);
                     }
                 }
                 fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
                 __syncwarp();
                 if (lane == 0) mbar_arrive_1(&S.b_full[st]);
             }
+            __syncwarp();
+            if (lane == 0) mbar_arrive_1(&S.slab_empty[sb]);  // this K-tile's slab is no longer read
         }
     }
     tc_fence_before();
@@ -373,9 +425,11 @@ WgPlan wg_plan(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W, int32_t 
     return P;
 }
 
+int32_t slab_pitch(int32_t W) { return (W + 2 + 3) / 4 * 4; }
+
 template <int PASSES, int STAGES>
 size_t wg_smem_bytes(const WgPlan &P, int32_t W) {
-    return sizeof(WgSmem<PASSES, STAGES>) + (size_t)kCiBlk * (P.R + 2) * (W + 2) * 4 + 1024;
+    return sizeof(WgSmem<PASSES, STAGES>) + 2 * (size_t)kCiBlk * (P.R + 2) * slab_pitch(W) * 4 + 1024;
 }
 
 PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
@@ -390,14 +444,15 @@ PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
     return fn;
 }
 
-template <int PASSES, int STAGES>
+template <int PASSES, int STAGES, bool VEC>
 cudaError_t launch_wg(const CUtensorMap &tm, const WgArgs &args, const WgPlan &P, int32_t W, cudaStream_t s) {
     static PerDeviceAttr attr;
     const size_t smem = wg_smem_bytes<PASSES, STAGES>(P, W);
-    const cudaError_t ea = attr.ensure(reinterpret_cast<const void *>(wgrad_ssdc_kernel<PASSES, STAGES>), (int)smem);
+    const cudaError_t ea =
+        attr.ensure(reinterpret_cast<const void *>(wgrad_ssdc_kernel<PASSES, STAGES, VEC>), (int)smem);
     if (ea != cudaSuccess) return ea;
     const unsigned grid = (unsigned)((int64_t)P.m_blocks * P.n_blocks * P.splits);
-    launch_k(wgrad_ssdc_kernel<PASSES, STAGES>, grid, kThreads, smem, s, tm, args);
+    launch_k(wgrad_ssdc_kernel<PASSES, STAGES, VEC>, grid, kThreads, smem, s, tm, args);
     return cudaPeekAtLastError();
 }
 
@@ -461,7 +516,11 @@ cudaError_t launch_wgrad_ssdc(const float *dy, const int32_t *row_end, const uin
     args.units = P.units;
     args.T = P.T;
     args.div_w = FastDiv::make((uint32_t)W);
-    const cudaError_t e = passes == 3 ? launch_wg<3, 2>(tm, args, P, W, s) : launch_wg<1, 4>(tm, args, P, W, s);
+    args.SWP = slab_pitch(W);
+    args.slab_floats = kCiBlk * (P.R + 2) * args.SWP;
+    const bool vec = W % 4 == 0;
+    const cudaError_t e = passes == 3 ? (vec ? launch_wg<3, 2, true>(tm, args, P, W, s) : launch_wg<3, 2, false>(tm, args, P, W, s))
+                                      : (vec ? launch_wg<1, 4, true>(tm, args, P, W, s) : launch_wg<1, 4, false>(tm, args, P, W, s));
     if (e != cudaSuccess) return e;
     ++*launches;
     const int64_t count = (int64_t)Co * Ci * kTaps;

@@ -28,7 +28,7 @@ def run(gist, x, dy, passes):
 
 
 SHAPES = [(1, 16, 128, 8, 8), (2, 32, 128, 13, 8), (3, 16, 256, 7, 28), (2, 48, 128, 56, 56), (1, 16, 128, 9, 12),
-          (2, 16, 128, 12, 20), (2, 16, 128, 14, 14), (1, 32, 128, 10, 6), (1, 16, 128, 1, 4), (1, 16, 128, 2, 250), (1, 16, 128, 8, 13),
+          (2, 16, 128, 12, 20), (2, 16, 128, 14, 14), (1, 32, 128, 10, 6), (1, 16, 128, 1, 4), (1, 16, 128, 4, 124), (1, 16, 128, 4, 61), (1, 16, 128, 8, 13),
           (1, 16, 128, 24, 21), (1, 16, 128, 40, 30)]
 
 
