@@ -292,14 +292,17 @@ dpr_many_kernel(const __grid_constant__ DprJobs J) {
 #ifndef GIST_DPR_CTAS
 #define GIST_DPR_CTAS 8  // grid cap, CTAs per SM
 #endif
+#ifndef GIST_DPR_MANY_CTAS
+#define GIST_DPR_MANY_CTAS 4  // many-map grid cap (C3's four DPR sites: 8 -> 4 CTAs/SM took a6 57% -> 62%, a7 64% -> 73%)
+#endif
 template <int BITS>
-int64_t dpr_blocks(int64_t n) {
+int64_t dpr_blocks(int64_t n, int per_sm = GIST_DPR_CTAS) {
     // one group per thread until the grid cap is reached (the unrolled loops then take several
     // per thread): small maps get every SM instead of 1/U of the threads
     constexpr int GF = (BITS == 10) ? 12 : 4;
     int64_t groups = n / GF + 1;
     int64_t blocks = ceil_div(groups, kDprThreads);
-    const int64_t cap = (int64_t)num_sms() * GIST_DPR_CTAS;
+    const int64_t cap = (int64_t)num_sms() * per_sm;
     return blocks > cap ? cap : blocks;
 }
 
@@ -344,9 +347,9 @@ cudaError_t launch_dpr_many(const gist_dpr_job *jobs, int32_t count, int bits, b
         for (int k = 0; k < J.count; ++k) n_sum += J.j[k].n;
         unsigned grid = 1;
         switch (bits) {
-            case 16: grid = (unsigned)dpr_blocks<16>(n_sum); break;
-            case 10: grid = (unsigned)dpr_blocks<10>(n_sum); break;
-            case 8: grid = (unsigned)dpr_blocks<8>(n_sum); break;
+            case 16: grid = (unsigned)dpr_blocks<16>(n_sum, GIST_DPR_MANY_CTAS); break;
+            case 10: grid = (unsigned)dpr_blocks<10>(n_sum, GIST_DPR_MANY_CTAS); break;
+            case 8: grid = (unsigned)dpr_blocks<8>(n_sum, GIST_DPR_MANY_CTAS); break;
             default: return cudaErrorInvalidValue;
         }
         (void)n_max;
