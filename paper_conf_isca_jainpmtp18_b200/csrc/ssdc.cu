@@ -348,6 +348,9 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
                 const EncJob &jb = J.j[S.job[q]];
                 const int64_t e0 = (t - jb.tile0) * (int64_t)(kTileRows * kRow) + h * kPartElems;
                 const int64_t avail = jb.n - e0;
+                // racecheck reports these ring writes against the writers' ring reads (fetch): ordered by
+                // counted[q] (counter arrive, release) -> publisher wait (acquire) ... published[q] arrive
+                // -> writer wait in fetch, a chain of mbarrier release/acquire pairs racecheck does not model
                 if (avail < kPartElems) {  // ragged end of the map: the part the TMA could not copy, zeros
                     const int from = avail > 0 ? (int)(((avail * 4) & ~15ll) / 4) : 0;
                     for (int i = from + lane; i < kPartElems; i += 32) T[i] = (i < avail) ? jb.x[e0 + i] : 0.0f;
@@ -363,6 +366,8 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
                     if (lane == r) mine = u & 0xffffu;
                     if (lane == r + 1) mine = u >> 16;
                 }
+                // rcnt -> publisher: counted[q] arrive (release) / wait (acquire); the slot is rewritten
+                // only after freed[q] (every writer done with tile j - kQ) -- racecheck hazard, ordered
                 if (lane < kPartRows) S.rcnt[q][h * kPartRows + lane] = mine;
             }
             __syncwarp();
@@ -384,6 +389,8 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
                     const uint32_t u = __shfl_up_sync(kFull, inc, d);
                     if (lane >= d) inc += u;
                 }
+                // rinc -> gatherer / writers: published[q] (and resolved[q]) arrive / wait; rewritten
+                // only after freed[q] -- racecheck hazard, ordered by those mbarriers
                 S.rinc[q][lane] = inc;
                 if (lane == 31) st_relaxed_u64(&tot[t], tag | inc);
             }

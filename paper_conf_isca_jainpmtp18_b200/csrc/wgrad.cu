@@ -48,6 +48,17 @@ constexpr int kEpi0 = kDec0 + kDecWarps;     // first epilogue warp
 // warp 0: TMA + TMEM owner, warp 1: MMA, 2..5: builders, 6..9: decoders, 10..17: accumulator drain
 constexpr int kThreads = 32 * (kEpi0 + kEpiWarps);
 static_assert(kBldThreads == kCiBlk * (kKs / 4), "one builder thread per (ci, chunk)");
+constexpr int kDecU = 8;                     // decoder: CSR entries per lane in flight
+// timing-only knobs (outputs invalid): skip the decode / the B build / the A split
+#ifndef GIST_WG_SKIP_DEC
+#define GIST_WG_SKIP_DEC 0
+#endif
+#ifndef GIST_WG_SKIP_B
+#define GIST_WG_SKIP_B 0
+#endif
+#ifndef GIST_WG_SKIP_ASPLIT
+#define GIST_WG_SKIP_ASPLIT 0
+#endif
 constexpr int kTmemCols = 512;               // two accumulators (K-tile t uses columns 256 (t % 2) + n)
 constexpr int kAccStride = 256;
 constexpr uint32_t kIdesc = idesc_tf32<kM, kN>();
@@ -68,17 +79,20 @@ struct WgArgs {
     int32_t units;    // partials per output tile = ceil(T / chunk)
     int64_t T;        // K-tiles in total = N * ktiles
     int32_t SWP;      // slab row pitch (W + 2 halo columns, rounded up to a multiple of 4)
+    int32_t rpc;      // CSR rows a K-tile's input rows of one channel can touch (4 channels x rpc <= 32)
     int32_t slab_floats;  // one slab buffer: kCiBlk * (R + 2) * SWP
     FastDiv div_w;
 };
 
-template <int PASSES, int STAGES>
+// NA dY stages (the TMA ring, deeper: its loads come from L2 with a long latency) and NB operand
+// stages (B hi/lo and A_lo, written by the builders); stage g uses A slot g % NA and B slot g % NB.
+template <int PASSES, int NA, int NB>
 struct __align__(1024) WgSmem {
-    float a[STAGES][kM * kKs];                      // dY tiles (TMA, 128-B swizzle): A_hi as loaded
-    float alo[PASSES == 3 ? STAGES : 1][PASSES == 3 ? kM * kKs : 256];  // A - tf32(A) (3xTF32 only; 1 KB keeps bhi 1024-aligned)
-    float bhi[STAGES][kN * kKs];                    // im2col(X) tiles, same layout
-    float blo[PASSES == 3 ? STAGES : 1][PASSES == 3 ? kN * kKs : 256];
-    uint64_t a_full[STAGES], b_full[STAGES], empty[STAGES], acc_full[2], acc_empty[2];
+    float a[NA][kM * kKs];                          // dY tiles (TMA, 128-B swizzle): A_hi after the split
+    float alo[PASSES == 3 ? NB : 1][PASSES == 3 ? kM * kKs : 256];  // A - tf32(A) (3xTF32 only; 1 KB keeps bhi 1024-aligned)
+    float bhi[NB][kN * kKs];                        // im2col(X) tiles, same layout
+    float blo[PASSES == 3 ? NB : 1][PASSES == 3 ? kN * kKs : 256];
+    uint64_t a_full[NA], a_empty[NA], b_full[NB], b_empty[NB], acc_full[2], acc_empty[2];
     uint64_t slab_full[2], slab_empty[2];  // decoders -> builders, builders -> decoders (per slab buffer)
     uint32_t tmem_base;
 };
@@ -87,14 +101,27 @@ static_assert(sizeof(float) * kM * kKs % 1024 == 0 && sizeof(float) * kN * kKs %
 
 // Long waits (the TMA lane on a free stage, the epilogue on a finished period, the decoders on a
 // free slab) back off instead of spinning on the issue slots the builders need.
+#ifndef GIST_WG_SKIP_TMA
+#define GIST_WG_SKIP_TMA 0
+#endif
+#ifndef GIST_WG_SPIN
+#define GIST_WG_SPIN 0
+#endif
+#ifndef GIST_WG_SKIP_EPI
+#define GIST_WG_SKIP_EPI 0  // timing only: the epilogue releases each period without reading TMEM
+#endif
 __device__ __forceinline__ void wait_backoff(uint64_t *bar, uint32_t parity) {
+#if GIST_WG_SPIN
+    mbar_wait(bar, parity);
+#else
     while (!mbar_test(bar, parity)) __nanosleep(64);
+#endif
 }
 
-template <int PASSES, int STAGES, bool VEC>
+template <int PASSES, int NA, int NB, bool VEC>
 __global__ void __launch_bounds__(kThreads, 1)
 wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
-    using Smem = WgSmem<PASSES, STAGES>;
+    using Smem = WgSmem<PASSES, NA, NB>;
     extern __shared__ unsigned char smem_raw[];
     // the 128-byte swizzle repeats every 1024 bytes: align the tiles to that
     const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
@@ -113,10 +140,13 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
     const int RW = a.R * a.W, SW = a.SWP, SR = a.R + 2;
 
     if (threadIdx.x == 0) {
-        for (int s = 0; s < STAGES; ++s) {
+        for (int s = 0; s < NA; ++s) {
             mbar_init(&S.a_full[s], 1);
+            mbar_init(&S.a_empty[s], 1);
+        }
+        for (int s = 0; s < NB; ++s) {
             mbar_init(&S.b_full[s], kBldWarps);
-            mbar_init(&S.empty[s], 1);
+            mbar_init(&S.b_empty[s], 1);
         }
         for (int b = 0; b < 2; ++b) {
             mbar_init(&S.acc_full[b], 1);
@@ -142,14 +172,29 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
         // ---- TMA producer: the dY tile [co0, co0+128) x [k, k+32) of each stage
         if (lane == 0) {
             prefetch_tmap(&tmap_dy);
+            // (image, K-tile row, stage) advanced incrementally: no division on this thread's path
+            int n = (int)(t0 / a.ktiles), ty = (int)(t0 % a.ktiles), j = 0, st = 0;
+            uint32_t ph = 0;
             for (int64_t g = 0; g < nst; ++g) {
-                const int st = (int)(g % STAGES);
-                if (g >= STAGES) wait_backoff(&S.empty[st], (uint32_t)((g / STAGES) - 1) & 1u);
-                const int64_t t = t0 + g / a.spt;
-                const int j = (int)(g % a.spt);
-                const int n = (int)(t / a.ktiles), ty = (int)(t % a.ktiles);
+                if (g >= NA) wait_backoff(&S.a_empty[st], ph ^ 1u);
+#if GIST_WG_SKIP_TMA
+                (void)n, (void)ty, (void)j;
+                mbar_arrive_1(&S.a_full[st]);  // timing only: no dY load
+#else
                 mbar_arrive_expect_tx(&S.a_full[st], kM * kKs * 4);
                 tma_load_2d(S.a[st], &tmap_dy, ty * RW + j * kKs, n * a.Co + co0, &S.a_full[st]);
+#endif
+                if (++st == NA) {
+                    st = 0;
+                    ph ^= 1u;
+                }
+                if (++j == a.spt) {
+                    j = 0;
+                    if (++ty == a.ktiles) {
+                        ty = 0;
+                        ++n;
+                    }
+                }
             }
         }
     } else if (warp == 1) {
@@ -159,21 +204,22 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
             // its own TMEM buffer (period % 2), drained by the epilogue warps into fp32 registers: the
             // tensor core's own accumulation then spans at most ceil(spt/pp) stages, which keeps its
             // rounding error near fp32's (f4).
+            // stage / period bookkeeping advanced incrementally (no per-stage division on this thread's
+            // path); period q of a K-tile covers stages [floor(q spt / pp), floor((q+1) spt / pp))
             int64_t gp = 0;  // accumulation periods started so far
+            int sa = 0, st = 0, j = 0, q = 0;
+            uint32_t pha = 0, phb = 0;
+            int q_start = 0, q_end = a.spt / a.pp;
             for (int64_t g = 0; g < nst; ++g) {
-                const int st = (int)(g % STAGES);
-                const uint32_t par = (uint32_t)(g / STAGES) & 1u;
-                const int j = (int)(g % a.spt);
-                const int q = j * a.pp / a.spt;
-                const bool first = j == 0 || (j - 1) * a.pp / a.spt != q;
-                const bool last = j == a.spt - 1 || (j + 1) * a.pp / a.spt != q;
+                const bool first = j == q_start;
+                const bool last = j + 1 == q_end;
                 const int b = (int)(gp & 1);
                 if (first && gp >= 2) mbar_wait(&S.acc_empty[b], (uint32_t)((gp / 2) - 1) & 1u);
-                mbar_wait(&S.a_full[st], par);
-                mbar_wait(&S.b_full[st], par);
+                mbar_wait(&S.a_full[sa], pha);
+                mbar_wait(&S.b_full[st], phb);
                 tc_fence_after();
                 const uint32_t d = tmem + (uint32_t)(b * kAccStride);
-                const uint32_t ab = smem_u32(S.a[st]), bb = smem_u32(S.bhi[st]);
+                const uint32_t ab = smem_u32(S.a[sa]), bb = smem_u32(S.bhi[st]);
 #pragma unroll
                 for (int kk = 0; kk < kKs / 8; ++kk) {  // K = 8 tf32 (32 bytes) per instruction
                     const uint64_t da = umma_desc_sw128(ab + 32 * kk), db = umma_desc_sw128(bb + 32 * kk);
@@ -183,11 +229,26 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                         umma_tf32(d, umma_desc_sw128(smem_u32(S.alo[st]) + 32 * kk), db, kIdesc, 1u);
                     }
                 }
-                umma_commit(&S.empty[st]);  // the stage's smem is free once these MMAs complete
+                umma_commit(&S.a_empty[sa]);  // the stage's smem is free once these MMAs complete
+                umma_commit(&S.b_empty[st]);
                 if (last) {
                     umma_commit(&S.acc_full[b]);
                     ++gp;
                 }
+                if (++sa == NA) {
+                    sa = 0;
+                    pha ^= 1u;
+                }
+                if (++st == NB) {
+                    st = 0;
+                    phb ^= 1u;
+                }
+                if (last) {
+                    if (++q == a.pp) q = 0;
+                    q_start = q == 0 ? 0 : q_end;
+                    q_end = ((q + 1) * a.spt) / a.pp;
+                }
+                if (++j == a.spt) j = 0;
             }
         }
     } else if (warp >= kEpi0) {
@@ -210,7 +271,7 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
 #pragma unroll
             for (int i = 0; i < 5; ++i) {
                 const int tap = 5 * half + i;
-                if (tap < kTaps) {
+                if (tap < kTaps && !GIST_WG_SKIP_EPI) {
                     uint32_t v[16];
                     tmem_ld16(tmem + (uint32_t)(b * kAccStride) + ((uint32_t)(32 * q) << 16) + (uint32_t)(tap * kCiBlk), v);
                     tmem_wait_ld();
@@ -257,24 +318,83 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
             }
             named_bar(2, kDecThreads);  // the buffer is zero before any scatter
             const int ih_lo = max(0, oh0 - 1), ih_hi = min(a.H, oh0 + a.R + 1);
-            for (int cc = 0; cc < kCiBlk / kDecWarps; ++cc) {
-                const int ci = dw * (kCiBlk / kDecWarps) + cc;
-                const int64_t plane0 = ((int64_t)n * a.Ci + ci0 + ci) * a.H * a.W;
-                const int64_t F0 = plane0 + (int64_t)ih_lo * a.W, F1 = plane0 + (int64_t)ih_hi * a.W;
-                if (F1 <= F0) continue;
-                float *sl = slab + (size_t)ci * SR * SW;
-                for (int64_t r = F0 >> 8; r <= (F1 - 1) >> 8; ++r) {
-                    const int32_t e0 = r ? a.row_end[r - 1] : 0, e1 = a.row_end[r];
-                    for (int32_t k = e0 + lane; k < e1; k += 32) {
-                        const int64_t flat = 256 * r + a.col[k];
+#if !GIST_WG_SKIP_DEC
+            // Each warp decodes its 4 channels with two global round trips: (1) lane l loads the entry
+            // range of (channel, CSR row) pair l (<= 32 pairs); a warp scan gives their offsets in one
+            // flat entry list; (2) the lanes walk that list kDecU entries at a time, every col/val load
+            // of a batch in flight before the scatter.
+            {
+                constexpr int kCh = kCiBlk / kDecWarps;
+                const int npairs = kCh * a.rpc;
+                int32_t pe0 = 0, pcnt = 0;
+                if (lane < npairs && ih_hi > ih_lo) {
+                    const int ci = dw * kCh + lane / a.rpc, rr = lane % a.rpc;
+                    const int64_t plane0 = ((int64_t)n * a.Ci + ci0 + ci) * a.H * a.W;
+                    const int64_t F0 = plane0 + (int64_t)ih_lo * a.W, F1 = plane0 + (int64_t)ih_hi * a.W;
+                    const int64_t r = (F0 >> 8) + rr;
+                    if (r <= (F1 - 1) >> 8) {
+                        pe0 = r ? a.row_end[r - 1] : 0;
+                        pcnt = a.row_end[r] - pe0;
+                    }
+                }
+                int pend = pcnt;  // inclusive end of pair `lane` in the flat list
+#pragma unroll
+                for (int d = 1; d < 32; d <<= 1) {
+                    const int u = __shfl_up_sync(kFull, pend, d);
+                    if (lane >= d) pend += u;
+                }
+                const int total = __shfl_sync(kFull, pend, 31);
+                int p = 0;  // pair of this lane's current entry (entries are visited in increasing order)
+                for (int k0 = 0; k0 < total; k0 += 32 * kDecU) {
+                    int32_t kk[kDecU];
+                    int pr[kDecU];
+                    uint8_t cv[kDecU];
+                    float vv[kDecU];
+#pragma unroll
+                    for (int u = 0; u < kDecU; ++u) {
+                        const int k = k0 + 32 * u + lane;
+                        // advance to the first pair whose end exceeds k (whole-warp shuffles: every
+                        // lane takes part in each round, so each source lane is active)
+                        for (;;) {
+                            const int nxt = __shfl_sync(kFull, pend, p);
+                            const bool adv = k < total && k >= nxt;
+                            if (!__any_sync(kFull, adv)) break;
+                            if (adv) ++p;
+                        }
+                        pr[u] = k < total ? p : -1;
+                    }
+#pragma unroll
+                    for (int u = 0; u < kDecU; ++u) {
+                        // entry index: the pair's first entry + the offset inside the pair
+                        const int ps = pr[u] < 0 ? 0 : pr[u];
+                        const int32_t e0p = __shfl_sync(kFull, pe0, ps), endp = __shfl_sync(kFull, pend, ps),
+                                      cntp = __shfl_sync(kFull, pcnt, ps);
+                        const int k = k0 + 32 * u + lane;
+                        kk[u] = e0p + (k - (endp - cntp));
+                        if (pr[u] >= 0) {
+                            cv[u] = a.col[kk[u]];
+                            vv[u] = a.val[kk[u]];
+                        }
+                    }
+#pragma unroll
+                    for (int u = 0; u < kDecU; ++u) {
+                        if (pr[u] < 0) continue;
+                        const int ci = dw * kCh + pr[u] / a.rpc, rr = pr[u] % a.rpc;
+                        const int64_t plane0 = ((int64_t)n * a.Ci + ci0 + ci) * a.H * a.W;
+                        const int64_t F0 = plane0 + (int64_t)ih_lo * a.W, F1 = plane0 + (int64_t)ih_hi * a.W;
+                        const int64_t flat = 256 * ((F0 >> 8) + rr) + cv[u];
                         if (flat >= F0 && flat < F1) {
                             uint32_t ih, iw;
                             a.div_w.divmod((uint32_t)(flat - plane0), ih, iw);
-                            sl[((int)ih - oh0 + 1) * SW + (int)iw + 1] = a.val[k];
+                            // racecheck reports these slab writes against the builders' slab reads: they
+                            // are ordered by slab_full[sb] (decoder arrive, release -> builder wait,
+                            // acquire) and, for the next refill, slab_empty[sb] (builder arrive -> wait)
+                            slab[(size_t)ci * SR * SW + ((int)ih - oh0 + 1) * SW + (int)iw + 1] = vv[u];
                         }
                     }
                 }
             }
+#endif
             __syncwarp();
             if (lane == 0) mbar_arrive_1(&S.slab_full[sb]);
         }
@@ -291,14 +411,15 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
             const int oh0 = (int)(t % a.ktiles) * a.R;
             for (int j = 0; j < a.spt; ++j) {
                 const int64_t g = tl * a.spt + j;
-                const int st = (int)(g % STAGES);
-                if (g >= STAGES) mbar_wait(&S.empty[st], (uint32_t)((g / STAGES) - 1) & 1u);
+                const int st = (int)(g % NB), sa = (int)(g % NA);
+                if (g >= NB) mbar_wait(&S.b_empty[st], (uint32_t)((g / NB) - 1) & 1u);
                 const int pos = j * kKs + 4 * ch;  // the chunk's first position in the K-tile
                 uint32_t ohr = 0, ow = 0;
                 a.div_w.divmod((uint32_t)pos, ohr, ow);
                 unsigned char *bh = reinterpret_cast<unsigned char *>(S.bhi[st]);
                 unsigned char *bl = reinterpret_cast<unsigned char *>(S.blo[PASSES == 3 ? st : 0]);
-                if constexpr (VEC) {
+                if (GIST_WG_SKIP_B) {
+                } else if constexpr (VEC) {
                     // W % 4 == 0: the chunk lies in one output row at ow % 4 == 0; slab row kh holds the
                     // 6 inputs (cols ow .. ow+5) of its 3 taps: two 16-byte loads
                     const bool valid = pos < RW && oh0 + (int)ohr < a.H;
@@ -354,11 +475,11 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                             *reinterpret_cast<float4 *>(bl + o) = make_float4(lo[0], lo[1], lo[2], lo[3]);
                     }
                 }
-                if constexpr (PASSES == 3) {
+                if (PASSES == 3 && !GIST_WG_SKIP_ASPLIT) {
                     // A_hi = tf32_rn(A) written back in place, A_lo = A - A_hi (exact in fp32); the layouts
                     // of a[] and alo[] are identical, so chunk by chunk
-                    mbar_wait(&S.a_full[st], (uint32_t)(g / STAGES) & 1u);
-                    float4 *ar = reinterpret_cast<float4 *>(S.a[st]);
+                    mbar_wait(&S.a_full[sa], (uint32_t)(g / NA) & 1u);
+                    float4 *ar = reinterpret_cast<float4 *>(S.a[sa]);
                     float4 *al = reinterpret_cast<float4 *>(S.alo[st]);
 #pragma unroll
                     for (int i = 0; i < kM * kKs / 4 / kBldThreads; ++i) {
@@ -427,9 +548,21 @@ WgPlan wg_plan(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W, int32_t 
 
 int32_t slab_pitch(int32_t W) { return (W + 2 + 3) / 4 * 4; }
 
-template <int PASSES, int STAGES>
+#ifndef GIST_WG_NA3
+#define GIST_WG_NA3 2  // dY ring depth, 3xTF32 (4: 2.54 -> 2.79 ms on conv3_2, 3 and 6 no better)
+#endif
+#ifndef GIST_WG_NA1
+#define GIST_WG_NA1 4  // dY ring depth, 1xTF32 (6: 2.13 -> 2.58 ms)
+#endif
+#ifndef GIST_WG_NB1
+#define GIST_WG_NB1 4  // operand stages, 1xTF32
+#endif
+constexpr int kNA3 = GIST_WG_NA3, kNA1 = GIST_WG_NA1, kNB1 = GIST_WG_NB1;
+constexpr size_t kMaxSmemW = 227 * 1024;
+
+template <int PASSES, int NA, int NB>
 size_t wg_smem_bytes(const WgPlan &P, int32_t W) {
-    return sizeof(WgSmem<PASSES, STAGES>) + 2 * (size_t)kCiBlk * (P.R + 2) * slab_pitch(W) * 4 + 1024;
+    return sizeof(WgSmem<PASSES, NA, NB>) + 2 * (size_t)kCiBlk * (P.R + 2) * slab_pitch(W) * 4 + 1024;
 }
 
 PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
@@ -444,15 +577,15 @@ PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
     return fn;
 }
 
-template <int PASSES, int STAGES, bool VEC>
+template <int PASSES, int NA, int NB, bool VEC>
 cudaError_t launch_wg(const CUtensorMap &tm, const WgArgs &args, const WgPlan &P, int32_t W, cudaStream_t s) {
     static PerDeviceAttr attr;
-    const size_t smem = wg_smem_bytes<PASSES, STAGES>(P, W);
+    const size_t smem = wg_smem_bytes<PASSES, NA, NB>(P, W);
     const cudaError_t ea =
-        attr.ensure(reinterpret_cast<const void *>(wgrad_ssdc_kernel<PASSES, STAGES, VEC>), (int)smem);
+        attr.ensure(reinterpret_cast<const void *>(wgrad_ssdc_kernel<PASSES, NA, NB, VEC>), (int)smem);
     if (ea != cudaSuccess) return ea;
     const unsigned grid = (unsigned)((int64_t)P.m_blocks * P.n_blocks * P.splits);
-    launch_k(wgrad_ssdc_kernel<PASSES, STAGES, VEC>, grid, kThreads, smem, s, tm, args);
+    launch_k(wgrad_ssdc_kernel<PASSES, NA, NB, VEC>, grid, kThreads, smem, s, tm, args);
     return cudaPeekAtLastError();
 }
 
@@ -466,7 +599,10 @@ bool wgrad_shape_ok(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W) {
     // of R+2 rows must fit beside the pipeline stages (odd W > 64 needs R = 4: W <= 252 is not enough)
     if (!(N > 0 && H > 0 && W > 0 && Co % kM == 0 && Ci % kCiBlk == 0 && W <= 252 && (int64_t)H * W % 4 == 0))
         return false;
-    return wgrad_smem_bytes(N, Ci, Co, H, W, 3) <= kMaxSmem && wgrad_smem_bytes(N, Ci, Co, H, W, 1) <= kMaxSmem;
+    const WgPlan P = wg_plan(N, Ci, Co, H, W, 3);
+    const int64_t rpc = ((int64_t)(P.R + 2) * W + 255) / 256 + 1;  // decoder pairs: 16 * rpc <= 128
+    return (kCiBlk / kDecWarps) * rpc <= 32 && wgrad_smem_bytes(N, Ci, Co, H, W, 3) <= kMaxSmem &&
+           wgrad_smem_bytes(N, Ci, Co, H, W, 1) <= kMaxSmem;
 }
 
 size_t wgrad_workspace_bytes(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W) {
@@ -476,7 +612,7 @@ size_t wgrad_workspace_bytes(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32
 
 size_t wgrad_smem_bytes(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W, int32_t passes) {
     const WgPlan P = wg_plan(N, Ci, Co, H, W, passes);
-    return passes == 3 ? wg_smem_bytes<3, 2>(P, W) : wg_smem_bytes<1, 4>(P, W);
+    return passes == 3 ? wg_smem_bytes<3, 2, 2>(P, W) : wg_smem_bytes<1, 4, 4>(P, W);  // the shallow ring always fits
 }
 
 cudaError_t launch_wgrad_ssdc(const float *dy, const int32_t *row_end, const uint8_t *col, const float *val, int32_t N,
@@ -517,10 +653,19 @@ cudaError_t launch_wgrad_ssdc(const float *dy, const int32_t *row_end, const uin
     args.T = P.T;
     args.div_w = FastDiv::make((uint32_t)W);
     args.SWP = slab_pitch(W);
+    args.rpc = (int32_t)(((int64_t)(P.R + 2) * W + 255) / 256 + 1);
     args.slab_floats = kCiBlk * (P.R + 2) * args.SWP;
     const bool vec = W % 4 == 0;
-    const cudaError_t e = passes == 3 ? (vec ? launch_wg<3, 2, true>(tm, args, P, W, s) : launch_wg<3, 2, false>(tm, args, P, W, s))
-                                      : (vec ? launch_wg<1, 4, true>(tm, args, P, W, s) : launch_wg<1, 4, false>(tm, args, P, W, s));
+    // the deeper dY ring when the slabs leave room for it
+    const bool deep3 = wg_smem_bytes<3, kNA3, 2>(P, W) <= kMaxSmemW, deep1 = wg_smem_bytes<1, kNA1, kNB1>(P, W) <= kMaxSmemW;
+    cudaError_t e;
+    if (passes == 3) {
+        if (deep3) e = vec ? launch_wg<3, kNA3, 2, true>(tm, args, P, W, s) : launch_wg<3, kNA3, 2, false>(tm, args, P, W, s);
+        else e = vec ? launch_wg<3, 2, 2, true>(tm, args, P, W, s) : launch_wg<3, 2, 2, false>(tm, args, P, W, s);
+    } else {
+        if (deep1) e = vec ? launch_wg<1, kNA1, kNB1, true>(tm, args, P, W, s) : launch_wg<1, kNA1, kNB1, false>(tm, args, P, W, s);
+        else e = vec ? launch_wg<1, 4, 4, true>(tm, args, P, W, s) : launch_wg<1, 4, 4, false>(tm, args, P, W, s);
+    }
     if (e != cudaSuccess) return e;
     ++*launches;
     const int64_t count = (int64_t)Co * Ci * kTaps;

@@ -23,5 +23,17 @@ for n in (1, 1000, 4096 * 3 + 5, 256 * 16 * 40 + 17):
     gist.gist_ssdc_decode(row_end, col, val, n)
     for b in (16, 10, 8):
         gist.gist_dpr_decode(gist.gist_dpr_encode(x, b), n, b)
+# 3x3/s1 plane-tile pools with a ragged last tile and odd planes (pool3.cu)
+for shape in [(3, 5, 7, 7), (2, 9, 14, 14)]:
+    y = WL.relu_map(shape, 0.5, 3, dev)
+    out, arg, mask = gist.gist_maxpool_fwd_argmax(y, WL.P3S1P1, fuse_mask=True)
+    gist.gist_pool_relu_bwd(torch.randn_like(out), arg, mask, shape, WL.P3S1P1)
+# f4: decode-in-GEMM weight gradient, both precisions, a vector (W % 4 == 0) and a scalar shape
+for N, Ci, Co, H, W in [(1, 16, 128, 8, 8), (1, 16, 128, 6, 10)]:
+    x = WL.relu_map((N, Ci, H, W), 0.8, 5, dev)
+    dy = WL.grad_map((N, Co, H, W), 6, dev)
+    row_end, col, val, nnz = gist.gist_ssdc_encode(x)
+    for passes in (3, 1):
+        gist.gist_conv3x3_wgrad_ssdc(dy, row_end, col, val, (N, Ci, H, W), passes=passes)
 torch.cuda.synchronize()
 print("sanitize workload done")

@@ -2,10 +2,10 @@
 the oracle (O8: the definition in binary64 over the seeded dense X, i.e. oracle-decode followed by
 a reference GEMM).  The result is a float reduction in a different order and, for passes = 1, with
 TF32 products, so the bar is normwise per entry: |dW - dW_ref| <= tol * sum_k |dY_k X_k| (the
-error scale of any fp32 implementation of this sum), tol = 1e-6 for 3xTF32 (north star: 1e-6
-relative where the reduction order differs, loosened to the 3xTF32 worst-case product bound
-2^-20 + 2^-22 rounded up to 2e-6) and 2^-9 for TF32 (two 2^-10 input truncations).
-(f4) derives both; the observed errors are about 1e-7 at full size."""
+error scale of any fp32 implementation of this sum), tol = 1e-6 for 3xTF32 (the north star's
+1e-6 relative where the reduction order differs) and 2^-9 for TF32 (two 2^-10 input truncations).
+DESIGN.md §6 (f4) derives both; measured (scripts/wgrad_accuracy.py, profiles/r2_f4_accuracy.json):
+3xTF32 max 1.0e-7 .. 3.9e-7, cuDNN's own fp32 weight gradient 3.7e-8 .. 9.1e-8, TF32 1.1e-4 .. 4.7e-4."""
 import numpy as np
 import pytest
 import torch
@@ -13,7 +13,7 @@ import torch
 import workloads as WL
 
 pytestmark = pytest.mark.gpu
-TOL = {3: 2e-6, 1: 2.0 ** -9}
+TOL = {3: 1e-6, 1: 2.0 ** -9}
 
 
 def inputs(N, Ci, Co, H, W, s, seed, cuda):
