@@ -306,13 +306,13 @@ class KernelTimer:
 
 # --------------------------------------------------------------------------------- clocks
 class ClockSampler:
-    """Samples SM clock, power and clock-event (throttle) reasons through NVML every 50 ms
+    """Samples SM clock, power and clock-event (throttle) reasons through NVML every 5 ms
     while the timed region runs (the recipe's nvidia-smi clocks line, in-process)."""
 
     REASONS = {"sw_power_cap": 0x4, "hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20,
                "hw_thermal_slowdown": 0x40, "hw_power_brake_slowdown": 0x80}
 
-    def __init__(self, device: torch.device, period_s: float = 0.05):
+    def __init__(self, device: torch.device, period_s: float = 0.005):
         self.device, self.period = device, period_s
         self.samples, self.reasons, self.max_mhz, self.power = [], set(), None, []
         self._stop = None

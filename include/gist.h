@@ -27,7 +27,7 @@
  *   - Deterministic: all encodings are bit-identical run to run; padding bits, unused
  *     fields and tail fields are always written as 0, so whole buffers compare with
  *     memcmp.  The library is stateless apart from per-device caches (SM count, the
- *     dynamic shared-memory opt-in of two kernels) filled on first use on each device;
+ *     dynamic shared-memory opt-in of the kernels that need it) filled on first use on each device;
  *     calls act on the CURRENT device (cudaSetDevice).  Concurrent calls on different
  *     streams are safe when they use distinct outputs and workspaces.
  *   - Inputs and outputs must not overlap (GIST_ERR_INVALID_ARGUMENT).
@@ -114,7 +114,10 @@ gist_status gist_binarize_encode(const float *y, int64_t n, uint32_t *mask, cuda
  *          written too — in the same pass (one read of y) for 2x2/s2 unpadded pools with H and
  *          W even whose warp unit of BR whole row pairs fits 512 items: BR*W/V <= 512 with
  *          V = 4 if W % 4 == 0 else 2, a = 16/gcd(W,16), BR = a*max(1, floor(256/(a*W/V)))
- *          (every VGG16 and OverFeat map); otherwise by a second kernel over y.
+ *          (every VGG16 and OverFeat map), and for 3x3 stride-1 windows with padding 0 or 1
+ *          (GoogLeNet's in-module pools: whole-plane tiles staged in shared memory, when the
+ *          planes of one tile, a multiple of 32/gcd(H*W,32) and of 8/gcd(Ho*Wo,8), fit a 32 KB
+ *          stage); otherwise by a second kernel over y.
  * TOO_LARGE if N*C*H*W >= 2^31. */
 gist_status gist_maxpool_fwd_argmax(const float *y, int32_t N, int32_t C, int32_t H, int32_t W,
                                     const gist_pool2d *p, float *out, uint32_t *argmax,
@@ -126,8 +129,9 @@ gist_status gist_maxpool_fwd_argmax(const float *y, int32_t N, int32_t C, int32_
  * gist_maxpool_fwd_argmax(relu(x), ..., mask) writes, with relu(v) = (v < 0 ? +0.0f : v)
  * (R21: torch's ReLU; -0.0 and NaN pass through), reading x once: out = the window max of
  * relu(x), argmax = its 4-bit in-window index, mask bit i = (x[i] > 0) (= relu(x)[i] > 0).
- * mask is required.  One kernel for 2x2/s2 with even H and W (VGG16, OverFeat); other
- * geometries run the forward with relu on load plus a binarize pass over x.  Errors as
+ * mask is required.  One kernel for 2x2/s2 with even H and W (VGG16, OverFeat) and for the 3x3
+ * stride-1 pools that gist_maxpool_fwd_argmax fuses; other geometries run the forward with relu
+ * on load plus a binarize pass over x.  Errors as
  * gist_maxpool_fwd_argmax; mask == NULL -> INVALID_ARGUMENT. */
 gist_status gist_relu_maxpool_fwd_argmax(const float *x, int32_t N, int32_t C, int32_t H, int32_t W,
                                          const gist_pool2d *p, float *out, uint32_t *argmax, uint32_t *mask,
