@@ -48,7 +48,7 @@ constexpr int kEpi0 = kDec0 + kDecWarps;     // first epilogue warp
 // warp 0: TMA + TMEM owner, warp 1: MMA, 2..5: builders, 6..9: decoders, 10..17: accumulator drain
 constexpr int kThreads = 32 * (kEpi0 + kEpiWarps);
 static_assert(kBldThreads == kCiBlk * (kKs / 4), "one builder thread per (ci, chunk)");
-constexpr int kDecU = 8;                     // decoder: CSR entries per lane in flight
+constexpr int kDecU = 8;                     // decoder: CSR entries per lane in flight (16: more spills, slower)
 // timing-only knobs (outputs invalid): skip the decode / the B build / the A split
 #ifndef GIST_WG_SKIP_DEC
 #define GIST_WG_SKIP_DEC 0
@@ -92,7 +92,7 @@ struct __align__(1024) WgSmem {
     float alo[PASSES == 3 ? NB : 1][PASSES == 3 ? kM * kKs : 256];  // A - tf32(A) (3xTF32 only; 1 KB keeps bhi 1024-aligned)
     float bhi[NB][kN * kKs];                        // im2col(X) tiles, same layout
     float blo[PASSES == 3 ? NB : 1][PASSES == 3 ? kN * kKs : 256];
-    uint64_t a_full[NA], a_empty[NA], b_full[NB], b_empty[NB], acc_full[2], acc_empty[2];
+    uint64_t a_full[NA], b_full[NB], b_empty[NB], acc_full[2], acc_empty[2];
     uint64_t slab_full[2], slab_empty[2];  // decoders -> builders, builders -> decoders (per slab buffer)
     uint32_t tmem_base;
 };
@@ -121,6 +121,7 @@ __device__ __forceinline__ void wait_backoff(uint64_t *bar, uint32_t parity) {
 template <int PASSES, int NA, int NB, bool VEC>
 __global__ void __launch_bounds__(kThreads, 1)
 wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
+    static_assert(NA == NB, "one empty barrier per stage serves the dY ring and the operand stages");
     using Smem = WgSmem<PASSES, NA, NB>;
     extern __shared__ unsigned char smem_raw[];
     // the 128-byte swizzle repeats every 1024 bytes: align the tiles to that
@@ -140,10 +141,7 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
     const int RW = a.R * a.W, SW = a.SWP, SR = a.R + 2;
 
     if (threadIdx.x == 0) {
-        for (int s = 0; s < NA; ++s) {
-            mbar_init(&S.a_full[s], 1);
-            mbar_init(&S.a_empty[s], 1);
-        }
+        for (int s = 0; s < NA; ++s) mbar_init(&S.a_full[s], 1);
         for (int s = 0; s < NB; ++s) {
             mbar_init(&S.b_full[s], kBldWarps);
             mbar_init(&S.b_empty[s], 1);
@@ -176,7 +174,7 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
             int n = (int)(t0 / a.ktiles), ty = (int)(t0 % a.ktiles), j = 0, st = 0;
             uint32_t ph = 0;
             for (int64_t g = 0; g < nst; ++g) {
-                if (g >= NA) wait_backoff(&S.a_empty[st], ph ^ 1u);
+                if (g >= NA) wait_backoff(&S.b_empty[st], ph ^ 1u);  // NA == NB: one empty barrier per stage
 #if GIST_WG_SKIP_TMA
                 (void)n, (void)ty, (void)j;
                 mbar_arrive_1(&S.a_full[st]);  // timing only: no dY load
@@ -215,7 +213,8 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                 const bool last = j + 1 == q_end;
                 const int b = (int)(gp & 1);
                 if (first && gp >= 2) mbar_wait(&S.acc_empty[b], (uint32_t)((gp / 2) - 1) & 1u);
-                mbar_wait(&S.a_full[sa], pha);
+                // one wait per stage: the builders arrive on b_full only after the stage's dY tile has
+                // landed (a_full), so b_full covers both operands
                 mbar_wait(&S.b_full[st], phb);
                 tc_fence_after();
                 const uint32_t d = tmem + (uint32_t)(b * kAccStride);
@@ -229,8 +228,7 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                         umma_tf32(d, umma_desc_sw128(smem_u32(S.alo[st]) + 32 * kk), db, kIdesc, 1u);
                     }
                 }
-                umma_commit(&S.a_empty[sa]);  // the stage's smem is free once these MMAs complete
-                umma_commit(&S.b_empty[st]);
+                umma_commit(&S.b_empty[st]);  // the stage's smem (A and B) is free once these MMAs complete
                 if (last) {
                     umma_commit(&S.acc_full[b]);
                     ++gp;
@@ -305,6 +303,27 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
         // the 16 channels, zero-filled then scattered from the CSR rows that cover them, into slab
         // buffer (t - t0) % 2 while the builders read the other one
         const int dp = threadIdx.x - 32 * kDec0, dw = warp - kDec0;
+        constexpr int kCh = kCiBlk / kDecWarps;
+        const int npairs = kCh * a.rpc;
+        // lane l's (channel, CSR row) pair of K-tile t: the row's entry range [e0, e1), issued one
+        // K-tile ahead so that its latency hides under the previous K-tile's entry loads
+        auto pair_range = [&](int64_t t, int32_t &e0, int32_t &e1) {
+            e0 = e1 = 0;
+            if (t >= t1 || lane >= npairs) return;
+            const int n = (int)(t / a.ktiles), oh0 = (int)(t % a.ktiles) * a.R;
+            const int ih_lo = max(0, oh0 - 1), ih_hi = min(a.H, oh0 + a.R + 1);
+            if (ih_hi <= ih_lo) return;
+            const int ci = dw * kCh + lane / a.rpc, rr = lane % a.rpc;
+            const int64_t plane0 = ((int64_t)n * a.Ci + ci0 + ci) * a.H * a.W;
+            const int64_t F0 = plane0 + (int64_t)ih_lo * a.W, F1 = plane0 + (int64_t)ih_hi * a.W;
+            const int64_t r = (F0 >> 8) + rr;
+            if (r <= (F1 - 1) >> 8) {
+                e0 = r ? a.row_end[r - 1] : 0;
+                e1 = a.row_end[r];
+            }
+        };
+        int32_t cur_e0, cur_e1;
+        pair_range(t0, cur_e0, cur_e1);
         for (int64_t t = t0; t < t1; ++t) {
             const int64_t tl = t - t0;
             const int sb = (int)(tl & 1);
@@ -319,24 +338,11 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
             named_bar(2, kDecThreads);  // the buffer is zero before any scatter
             const int ih_lo = max(0, oh0 - 1), ih_hi = min(a.H, oh0 + a.R + 1);
 #if !GIST_WG_SKIP_DEC
-            // Each warp decodes its 4 channels with two global round trips: (1) lane l loads the entry
-            // range of (channel, CSR row) pair l (<= 32 pairs); a warp scan gives their offsets in one
-            // flat entry list; (2) the lanes walk that list kDecU entries at a time, every col/val load
-            // of a batch in flight before the scatter.
+            // Each warp decodes its 4 channels: lane l holds the entry range of (channel, CSR row) pair
+            // l (<= 32 pairs, loaded one K-tile ahead); a warp scan flattens the pairs into one entry
+            // list, and the lanes load kDecU entries each (all in flight) before scattering them.
             {
-                constexpr int kCh = kCiBlk / kDecWarps;
-                const int npairs = kCh * a.rpc;
-                int32_t pe0 = 0, pcnt = 0;
-                if (lane < npairs && ih_hi > ih_lo) {
-                    const int ci = dw * kCh + lane / a.rpc, rr = lane % a.rpc;
-                    const int64_t plane0 = ((int64_t)n * a.Ci + ci0 + ci) * a.H * a.W;
-                    const int64_t F0 = plane0 + (int64_t)ih_lo * a.W, F1 = plane0 + (int64_t)ih_hi * a.W;
-                    const int64_t r = (F0 >> 8) + rr;
-                    if (r <= (F1 - 1) >> 8) {
-                        pe0 = r ? a.row_end[r - 1] : 0;
-                        pcnt = a.row_end[r] - pe0;
-                    }
-                }
+                const int32_t pe0 = cur_e0, pcnt = cur_e1 - cur_e0;
                 int pend = pcnt;  // inclusive end of pair `lane` in the flat list
 #pragma unroll
                 for (int d = 1; d < 32; d <<= 1) {
@@ -376,6 +382,7 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                             vv[u] = a.val[kk[u]];
                         }
                     }
+                    if (k0 == 0) pair_range(t + 1, cur_e0, cur_e1);  // the next K-tile's ranges, in flight now
 #pragma unroll
                     for (int u = 0; u < kDecU; ++u) {
                         if (pr[u] < 0) continue;
@@ -393,7 +400,10 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                         }
                     }
                 }
+                if (total == 0) pair_range(t + 1, cur_e0, cur_e1);
             }
+#else
+            pair_range(t + 1, cur_e0, cur_e1);
 #endif
             __syncwarp();
             if (lane == 0) mbar_arrive_1(&S.slab_full[sb]);
@@ -489,6 +499,7 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                         al[p + i * kBldThreads] = make_float4(x.x - h.x, x.y - h.y, x.z - h.z, x.w - h.w);
                     }
                 }
+                if constexpr (PASSES == 1) mbar_wait(&S.a_full[sa], (uint32_t)(g / NA) & 1u);  // b_full implies A
                 fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
                 __syncwarp();
                 if (lane == 0) mbar_arrive_1(&S.b_full[st]);
@@ -548,16 +559,10 @@ WgPlan wg_plan(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W, int32_t 
 
 int32_t slab_pitch(int32_t W) { return (W + 2 + 3) / 4 * 4; }
 
-#ifndef GIST_WG_NA3
-#define GIST_WG_NA3 2  // dY ring depth, 3xTF32 (4: 2.54 -> 2.79 ms on conv3_2, 3 and 6 no better)
+#ifndef GIST_WG_NS1
+#define GIST_WG_NS1 4  // pipeline stages, 1xTF32 (3xTF32: 2; a deeper dY-only ring measured slower)
 #endif
-#ifndef GIST_WG_NA1
-#define GIST_WG_NA1 4  // dY ring depth, 1xTF32 (6: 2.13 -> 2.58 ms)
-#endif
-#ifndef GIST_WG_NB1
-#define GIST_WG_NB1 4  // operand stages, 1xTF32
-#endif
-constexpr int kNA3 = GIST_WG_NA3, kNA1 = GIST_WG_NA1, kNB1 = GIST_WG_NB1;
+constexpr int kNS1 = GIST_WG_NS1;
 constexpr size_t kMaxSmemW = 227 * 1024;
 
 template <int PASSES, int NA, int NB>
@@ -657,13 +662,12 @@ cudaError_t launch_wgrad_ssdc(const float *dy, const int32_t *row_end, const uin
     args.slab_floats = kCiBlk * (P.R + 2) * args.SWP;
     const bool vec = W % 4 == 0;
     // the deeper dY ring when the slabs leave room for it
-    const bool deep3 = wg_smem_bytes<3, kNA3, 2>(P, W) <= kMaxSmemW, deep1 = wg_smem_bytes<1, kNA1, kNB1>(P, W) <= kMaxSmemW;
+    const bool deep1 = wg_smem_bytes<1, kNS1, kNS1>(P, W) <= kMaxSmemW;
     cudaError_t e;
     if (passes == 3) {
-        if (deep3) e = vec ? launch_wg<3, kNA3, 2, true>(tm, args, P, W, s) : launch_wg<3, kNA3, 2, false>(tm, args, P, W, s);
-        else e = vec ? launch_wg<3, 2, 2, true>(tm, args, P, W, s) : launch_wg<3, 2, 2, false>(tm, args, P, W, s);
+        e = vec ? launch_wg<3, 2, 2, true>(tm, args, P, W, s) : launch_wg<3, 2, 2, false>(tm, args, P, W, s);
     } else {
-        if (deep1) e = vec ? launch_wg<1, kNA1, kNB1, true>(tm, args, P, W, s) : launch_wg<1, kNA1, kNB1, false>(tm, args, P, W, s);
+        if (deep1) e = vec ? launch_wg<1, kNS1, kNS1, true>(tm, args, P, W, s) : launch_wg<1, kNS1, kNS1, false>(tm, args, P, W, s);
         else e = vec ? launch_wg<1, 4, 4, true>(tm, args, P, W, s) : launch_wg<1, 4, 4, false>(tm, args, P, W, s);
     }
     if (e != cudaSuccess) return e;
