@@ -39,6 +39,12 @@ namespace {
 #define GIST_POOL3_THREADS 512  // 256: 10-40% slower, 1024: 5-25% slower (3x3/s1 maps, GoogLeNet b64)
 #endif
 constexpr int kRT = GIST_POOL3_THREADS;  // threads per CTA
+#ifndef GIST_POOL3_BWD_SEG
+#define GIST_POOL3_BWD_SEG 0  // 1: row segments for tiles with few columns (measured slower in the C4 step)
+#endif
+#ifndef GIST_POOL3_BWD_STRIP
+#define GIST_POOL3_BWD_STRIP 1  // stride-1 backward: column strips for tiles of >= kRT/2 columns (0: never)
+#endif
 constexpr int kRS = 3;    // ring stages
 #ifndef GIST_POOL3_STAGE_KB
 #define GIST_POOL3_STAGE_KB 32  // KB per ring stage (3 stages + extras < 113 KB: 2 CTAs per SM)
@@ -400,6 +406,59 @@ pool3_bwd_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ ar
                 if (r1 && c1) dxt[il + a.W + 1] = mbit(il + a.W + 1) ? a11 : 0.0f;
             }
         } else {
+            if (GIST_POOL3_BWD_STRIP) {
+            // one thread per input column segment (segr rows) of a plane walks down its rows; a tile with
+            // few columns (GoogLeNet's 28x28 planes) is cut into row segments so every thread has work.  Input (ih, iw) is position
+            // (dy, dx) = (th - oh, tw - ow) of the windows oh in [th-2, th], ow in [tw-2, tw] (th = ih + P):
+            // padded nibble rows th, th+1, th+2 (dy = 2, 1, 0) x columns tw, tw+1, tw+2 (dx = 2, 1, 0),
+            // visited in that order = ascending output order (R6).  Moving down one row shifts the
+            // rows by one, so each window row's three nibbles are loaded once per column, not three times.
+            const int cols = t.np * a.W;
+            const int nseg = (!GIST_POOL3_BWD_SEG || cols >= kRT / 2) ? 1 : (kRT + cols - 1) / cols;  // row segments
+            const int segr = (a.H + nseg - 1) / nseg;
+            for (int it = tid; it < cols * nseg; it += kRT) {
+                const int sg = it / cols;
+                uint32_t pl, iw;
+                a.div_w.divmod((uint32_t)(it - sg * cols), pl, iw);
+                const int tw = (int)iw + a.P;
+                const int ih_beg = sg * segr, ih_end = min(a.H, ih_beg + segr);
+                const unsigned char *nb = nbb + (int)pl * PP + tw;  // padded column tw of row 0
+                const float *Dp = D + (int)pl * a.HoWo + tw;          // dY of window (0, tw)
+                unsigned n0[3], n1[3], n2[3];
+#pragma unroll
+                for (int c = 0; c < 3; ++c) {
+                    n0[c] = nb[(ih_beg + a.P) * a.PC + c];
+                    n1[c] = nb[(ih_beg + a.P + 1) * a.PC + c];
+                }
+                const int il0 = (int)pl * a.HW + (int)iw;
+                for (int ih = ih_beg; ih < ih_end; ++ih) {
+                    const int th = ih + a.P;
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) n2[c] = nb[(th + 2) * a.PC + c];
+                    const int il = il0 + ih * a.W;
+                    const bool on = mbit(il);
+                    float acc = 0.0f;  // R6: +0.0f, then ascending output order
+                    if (on) {
+                        const float *d0 = Dp + (th - 2) * a.Wo;  // window row th-2: dY at column tw - 2 + c
+#pragma unroll
+                        for (int c = 0; c < 3; ++c)
+                            if (n0[c] == 8u - c) acc = acc + d0[c - 2];
+#pragma unroll
+                        for (int c = 0; c < 3; ++c)
+                            if (n1[c] == 5u - c) acc = acc + d0[a.Wo + c - 2];
+#pragma unroll
+                        for (int c = 0; c < 3; ++c)
+                            if (n2[c] == 2u - c) acc = acc + d0[2 * a.Wo + c - 2];
+                    }
+                    dxt[il] = on ? acc : 0.0f;
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) {
+                        n0[c] = n1[c];
+                        n1[c] = n2[c];
+                    }
+                }
+            }
+            } else {
             // one thread per input element; windows (oh, ow) = (th - dy, tw - dx), th = ih + P, in
             // ascending output order; the hit nibble is 3 dy + dx
             const int cnt = t.np * a.HW;
@@ -420,6 +479,7 @@ pool3_bwd_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ ar
                             if (nbb[cell - dy * a.PC - dxx] == (unsigned)(3 * dy + dxx)) acc = acc + D[ol - dy * a.Wo - dxx];
                 }
                 dxt[l] = on ? acc : 0.0f;
+            }
             }
         }
         __syncthreads();  // stage st consumed
