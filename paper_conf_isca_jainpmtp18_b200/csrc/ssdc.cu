@@ -55,6 +55,9 @@ constexpr int kRow = 256;
 #ifndef GIST_SSDC_DEC_CTAS
 #define GIST_SSDC_DEC_CTAS 3  // decode CTAs per SM (grid cap); 4-6 measured slower in isolation
 #endif
+#ifndef GIST_SSDC_LPRE
+#define GIST_SSDC_LPRE 0  // 1: the counters also scan the writers' lane counts (writers skip count + scan): 0.228 -> 0.265 ms, the counters then pace the prefix chain
+#endif
 #ifndef GIST_SSDC_WROWS
 #define GIST_SSDC_WROWS 2
 #endif
@@ -121,6 +124,9 @@ struct __align__(128) EncSmem {
     uint32_t vst[2][kStage];         // compacted value bits of a tile (congruent to the output mod 16),
     uint8_t cst[2][kStage];          // and its columns (bytes, same index); double-buffered by tile
     uint32_t rcnt[kQ][kTileRows];   // per-row nonzero counts
+#if GIST_SSDC_LPRE
+    uint32_t lpre[kQ][kWriters][32];  // per writer lane: row-0 | row-1 exclusive offsets (16 bits each)
+#endif
     uint32_t rinc[kQ][kTileRows];   // tile-local inclusive row ends
     int64_t base[kQ];                // global offset of the tile
     int64_t tile[kQ];                // tile claimed in this slot (>= tiles: no more work)
@@ -164,8 +170,13 @@ __device__ __forceinline__ void stage_rows(EncSmem &S, int q, int sb, int w, int
     const uint32_t w_excl = rw ? S.rinc[q][rw - 1] : 0u;
     if (S.rinc[q][rw + kWRows - 1] == w_excl) return;  // no nonzeros in these rows
     const uint32_t p = (uint32_t)(S.base[q] & 15) + w_excl;  // staging index of the writer's first entry
-    // lane prefix of both rows' lane counts in one warp scan (16-bit fields: row counts <= 256)
     static_assert(kWRows == 2, "the packed scan carries two rows");
+#if GIST_SSDC_LPRE
+    // the counters scanned this writer's lane counts (published with the tile, ordered by published[q])
+    const uint32_t pk = S.lpre[q][w][lane];
+    const uint32_t excl[2] = {pk & 0xffffu, pk >> 16};
+#else
+    // lane prefix of both rows' lane counts in one warp scan (16-bit fields: row counts <= 256)
     const uint32_t cnt0 = nz4(lo[0]) + nz4(hi[0]), cnt1 = nz4(lo[1]) + nz4(hi[1]);
     uint32_t inc = cnt0 | (cnt1 << 16);
 #pragma unroll
@@ -175,6 +186,7 @@ __device__ __forceinline__ void stage_rows(EncSmem &S, int q, int sb, int w, int
     }
     const uint32_t row0_tot = __shfl_sync(kFull, inc, 31) & 0xffffu;
     const uint32_t excl[2] = {(inc & 0xffffu) - cnt0, row0_tot + (inc >> 16) - cnt1};
+#endif
 #pragma unroll
     for (int r = 0; r < kWRows; ++r) {
         const uint32_t v[8] = {lo[r].x, lo[r].y, lo[r].z, lo[r].w, hi[r].x, hi[r].y, hi[r].z, hi[r].w};
@@ -358,6 +370,27 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
                     __syncwarp();
                 }
                 uint32_t mine = 0;
+#if GIST_SSDC_LPRE
+                // in the writers' layout (lane l: columns 8l .. 8l+7 of each row): the row pair of writer
+                // w = part * 4 + r/2 is scanned here, its per-lane exclusive offsets left in lpre
+#pragma unroll
+                for (int r = 0; r < kPartRows; r += 2) {
+                    const uint4 *r0 = reinterpret_cast<const uint4 *>(T + r * kRow), *r1 = r0 + kRow / 4;
+                    const uint32_t cnt0 = nz4(r0[2 * lane]) + nz4(r0[2 * lane + 1]);
+                    const uint32_t cnt1 = nz4(r1[2 * lane]) + nz4(r1[2 * lane + 1]);
+                    uint32_t inc = cnt0 | (cnt1 << 16);
+#pragma unroll
+                    for (int d = 1; d < 32; d <<= 1) {
+                        const uint32_t u = __shfl_up_sync(kFull, inc, d);
+                        if (lane >= d) inc += u;
+                    }
+                    const uint32_t tot = __shfl_sync(kFull, inc, 31);
+                    const uint32_t row0_tot = tot & 0xffffu;
+                    S.lpre[q][(h * kPartRows + r) / kWRows][lane] = ((inc & 0xffffu) - cnt0) | ((row0_tot + (inc >> 16) - cnt1) << 16);
+                    if (lane == r) mine = row0_tot;
+                    if (lane == r + 1) mine = tot >> 16;
+                }
+#else
 #pragma unroll
                 for (int r = 0; r < kPartRows; r += 2) {  // two rows per reduction (16-bit fields)
                     const uint4 *row4 = reinterpret_cast<const uint4 *>(T + r * kRow);
@@ -366,6 +399,7 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
                     if (lane == r) mine = u & 0xffffu;
                     if (lane == r + 1) mine = u >> 16;
                 }
+#endif
                 // rcnt -> publisher: counted[q] arrive (release) / wait (acquire); the slot is rewritten
                 // only after freed[q] (every writer done with tile j - kQ) -- racecheck hazard, ordered
                 if (lane < kPartRows) S.rcnt[q][h * kPartRows + lane] = mine;
