@@ -76,18 +76,26 @@ class StashArena:
     (which still publishes the true end); `check()` reads the end once and raises StashOverflow
     before any stash of an overflowed arena is decoded."""
 
-    def __init__(self, capacity: int, device):
+    def __init__(self, capacity: int, device, plan=None):
         self.capacity, self.device = int(capacity), torch.device(device)
         self.col = torch.empty(max(1, self.capacity), dtype=torch.uint8, device=self.device)
         self.val = torch.empty(max(1, self.capacity), dtype=torch.float32, device=self.device)
-        self.ws = None
+        self.ws, self.plan = None, plan
         self.reset()
 
     def reset(self):
         self.head = torch.zeros(1, dtype=torch.int64, device=self.device)
         self.used = None  # host value once checked
 
+    def head_ref(self):
+        """A callable returning the arena's current end (device tensor) without keeping the arena's
+        buffers alive (ArenaPlan reads it after the backward has released them)."""
+        box = self._box = [self.head]
+        return lambda: box[0]
+
     def _workspace(self, n: int) -> torch.Tensor:
+        if self.plan is not None:
+            return self.plan.workspace(n)
         need = gist_ssdc_workspace_bytes(n)
         if self.ws is None or self.ws.numel() < need:
             self.ws = torch.empty(need, dtype=torch.uint8, device=self.device)
@@ -102,6 +110,8 @@ class StashArena:
         SsdcEncodeMany([{"x": y, "row_end": row_end, "col": self.col, "val": self.val, "capacity": self.capacity,
                          "offset": start, "nnz": end}], workspace=self._workspace(n))()
         self.head = end
+        if getattr(self, "_box", None) is not None:
+            self._box[0] = end
         return row_end, start, end
 
     def check(self) -> int:
@@ -111,6 +121,46 @@ class StashArena:
         if self.used > self.capacity:
             raise StashOverflow(self.used, self.capacity)
         return self.used
+
+
+class ArenaPlan:
+    """Per-group arenas for one training step, sized from the previous step (no host sync in the
+    forward).  Each group (e.g. a VGG block) gets a fresh StashArena when `arena(g)` is called; the
+    arena is freed by the allocator once the group's last stash has been decoded in the backward, so
+    the stash memory shrinks as the backward proceeds (as exact-size stashes do).  `update()`, after
+    the backward, reads every arena's end in ONE host synchronization and resizes the groups for the
+    next step (used x `slack`); a group that overflowed raises StashOverflow at its first decode."""
+
+    def __init__(self, device, initial: dict | None = None, slack: float = 1.05, floor: int = 1 << 16):
+        self.device, self.slack, self.floor = torch.device(device), slack, floor
+        self.cap = dict(initial or {})
+        self.live = {}
+        self.ws = None  # one encode workspace shared by the plan's arenas (stream-ordered reuse)
+
+    def workspace(self, n: int) -> torch.Tensor:
+        need = gist_ssdc_workspace_bytes(n)
+        if self.ws is None or self.ws.numel() < need:
+            self.ws = torch.empty(need, dtype=torch.uint8, device=self.device)
+            gist_ssdc_workspace_init(self.ws)
+        return self.ws
+
+    def arena(self, group, default_capacity: int) -> "StashArena":
+        cap = self.cap.get(group, default_capacity)
+        a = StashArena(cap, self.device, plan=self)
+        self.live[group] = (a.head_ref(), cap)
+        return a
+
+    def update(self):
+        if not self.live:
+            return {}
+        groups = list(self.live)
+        used = torch.cat([self.live[g][0]() for g in groups]).cpu().tolist()  # one synchronization
+        out = {}
+        for g, u in zip(groups, used):
+            self.cap[g] = max(self.floor, int(u * self.slack))
+            out[g] = (int(u), self.live[g][1])
+        self.live = {}
+        return out
 
 
 _ARENA: list = []

@@ -51,25 +51,27 @@ class VGG16(nn.Module):
         x = F.relu(self.fc7(x))
         return self.fc8(x)
 
-    def forward_gist(self, x, bits, lossless=False, arena=None):
+    def forward_gist(self, x, bits, lossless=False, plan=None):
         # DPR (lossy) wraps everything; the Binarize/SSDC functions save only their encodings;
-        # with an arena the SSDC stashes are single-pass appends (no host sync in the forward)
+        # with an arena plan each block's SSDC stashes are single-pass appends into the block's own
+        # arena (no host sync in the forward; freed once the block's backward has decoded them)
         ctx = stash.dpr_saved_tensors(bits, self.parameters()) if not lossless else _null()
-        actx = stash.ssdc_arena(arena) if arena is not None else _null()
-        if arena is not None:
-            arena.reset()
-        with ctx, actx:
+        with ctx:
             c = 0
             z = self.convs[0](x)  # the input image: an "other" stashed map (DPR)
             c = 1
-            for b, (_, _, k) in enumerate(CFG):
-                for i in range(1 if b == 0 else 0, k):
-                    conv = self.convs[c]
-                    c += 1
-                    if i == 0:  # pool -> conv: SSDC of the pool output
-                        z = stash.stashed_conv(z, conv)
-                    else:  # relu -> conv: SSDC of the ReLU output
-                        z = stash.relu_conv(z, conv)
+            for b, (cin, cout, k) in enumerate(CFG):
+                side = 224 >> b
+                default = x.shape[0] * side * side * ((k - 1) * cout + (cin if b else 0)) * 6 // 10
+                actx = stash.ssdc_arena(plan.arena(b, default)) if plan is not None else _null()
+                with actx:
+                    for i in range(1 if b == 0 else 0, k):
+                        conv = self.convs[c]
+                        c += 1
+                        if i == 0:  # pool -> conv: SSDC of the pool output
+                            z = stash.stashed_conv(z, conv)
+                        else:  # relu -> conv: SSDC of the ReLU output
+                            z = stash.relu_conv(z, conv)
                 z = stash.relu_maxpool(z, 2, 2)  # relu -> maxpool: Binarize
             z = torch.flatten(z, 1)
             z = F.relu(self.fc6(z))
@@ -87,17 +89,22 @@ class _null:
 
 def step(model, x, target, fwd, marks=None):
     model.zero_grad(set_to_none=True)
+    plan = ARENA.get("plan")
     try:
         loss = F.cross_entropy(fwd(x), target)
-        return _finish(loss, marks)
-    except stash.StashOverflow as e:  # the arena was too small: grow it (once) and redo the step
-        if ARENA.get("arena") is None:
+        out = _finish(loss, marks)
+    except stash.StashOverflow:  # a block's arena was too small: resize from this step's ends, redo
+        if plan is None:
             raise
-        ARENA["arena"] = stash.StashArena(int(e.needed * 1.05), x.device)
+        loss = None
+        ARENA["last"] = plan.update()
         ARENA["grown"] = ARENA.get("grown", 0) + 1
         model.zero_grad(set_to_none=True)
         loss = F.cross_entropy(fwd(x), target)
-        return _finish(loss, marks)
+        out = _finish(loss, marks)
+    if plan is not None:
+        ARENA["last"] = plan.update()  # one host read per step, after the backward
+    return out
 
 
 ARENA = {}
@@ -215,19 +222,19 @@ def main():
 
     base = measure(model, x, target, model.forward_baseline)
     g_base = [p.grad.clone() for p in model.parameters()]
-    if args.arena:  # start at half the SSDC-stashed elements; an overflow grows it once
-        n_ssdc = sum(x.shape[0] * c * h * h for c, h in SSDC_SHAPES)
-        ARENA["arena"] = stash.StashArena(n_ssdc // 2, dev)
-    gist = measure(model, x, target, lambda t: model.forward_gist(t, args.bits, args.lossless, ARENA.get("arena")))
+    if args.arena:  # per-block arenas sized from the previous step (60% of the elements at first)
+        ARENA["plan"] = stash.ArenaPlan(dev)
+    gist = measure(model, x, target, lambda t: model.forward_gist(t, args.bits, args.lossless, ARENA.get("plan")))
     g_gist = [p.grad for p in model.parameters()]
     rel = max(float((a - b).abs().max() / (a.abs().max() + 1e-30)) for a, b in zip(g_base, g_gist))
     out = {
         "model": "VGG16 random init", "batch": args.batch, "image": 224,
         "encodings": "Binarize + SSDC" + ("" if args.lossless else f" + DPR-fp{args.bits}"),
         "baseline": base, "gist": gist,
-        "ssdc_stash": ({"mode": "arena (one encode pass per stash, no host sync in the forward)",
-                        "capacity_entries": ARENA["arena"].capacity, "used_entries": ARENA["arena"].check(),
-                        "grown": ARENA.get("grown", 0)} if args.arena else
+        "ssdc_stash": ({"mode": "per-block arenas (one encode pass per stash, no host sync in the forward; "
+                                "capacities from the previous step, one host read per step after the backward)",
+                        "blocks_used_capacity": {str(k): v for k, v in ARENA.get("last", {}).items()},
+                        "regrown_steps": ARENA.get("grown", 0)} if args.arena else
                        {"mode": "exact-size (count pass + host read of nnz + encode pass per stash)"}),
         "mfr_peak": round(base["peak_bytes"] / gist["peak_bytes"], 3),
         "mfr_above_inputs": round(base["peak_above_inputs_bytes"] / gist["peak_above_inputs_bytes"], 3),

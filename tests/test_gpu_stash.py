@@ -135,3 +135,35 @@ def test_arena_overflow_is_reported_before_decode(gist, cuda):
             s2 = stash.CSRStash(2 * y)
         assert torch.equal(s.dense().view(torch.int32), y.view(torch.int32))
         assert torch.equal(s2.dense().view(torch.int32), (2 * y).view(torch.int32))
+
+
+def test_arena_plan_per_group_resizes_and_stays_exact(gist, cuda, deterministic):
+    """ArenaPlan: one arena per group, sized from the previous step.  A first step with a too-small
+    capacity raises StashOverflow at the first decode; update() reads every group's end in one
+    synchronization, and the redone step is bit-exact to plain PyTorch."""
+    from paper_conf_isca_jainpmtp18_b200 import stash
+    torch.manual_seed(0)
+    m = TinyVGG().to(cuda)
+    x = torch.randn(8, 3, 32, 32, device=cuda)
+    y = torch.randint(0, 10, (8,), device=cuda)
+    g0 = grads(m, m.base, x, y)
+    plan = stash.ArenaPlan(cuda, floor=16)
+
+    def fwd(t):
+        with stash.ssdc_arena(plan.arena("a", 64)):
+            z = stash.relu_conv(m.c1(t), m.c2)
+        z = stash.relu_maxpool(z, 2)
+        with stash.ssdc_arena(plan.arena("b", 64)):
+            z = stash.relu_conv(stash.stashed_conv(z, m.c3), m.c4)
+        z = stash.relu_maxpool(z, 2)
+        return m.fc(torch.flatten(z, 1))
+
+    with pytest.raises(stash.StashOverflow):
+        grads(m, fwd, x, y)
+    sizes = plan.update()
+    assert set(sizes) == {"a", "b"} and all(used > cap for used, cap in sizes.values())
+    g1 = grads(m, fwd, x, y)
+    after = plan.update()
+    assert all(used <= cap for used, cap in after.values())
+    for (name, _), a, b in zip(m.named_parameters(), g0, g1):
+        assert torch.equal(a.view(torch.int32), b.view(torch.int32)), name
