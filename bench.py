@@ -280,11 +280,35 @@ class _Null:
         return False
 
 
-class KernelTimer:
-    """CUDA events around every launch, on the stream the kernels are launched on."""
+def site_label(kind, d):
+    """`<kernel kind>:<site name>` (a many-map launch: `<kind>:<first site>+<n-1>`)."""
+    if isinstance(d, list):
+        return f"{kind}:{d[0]['site'].name}+{len(d) - 1}" if d else kind
+    return f"{kind}:{d['site'].name}"
 
-    def __init__(self, stream):
+
+class NvtxRanges:
+    """An NVTX range per call site (`--nvtx`: named ranges in nsys / ncu --nvtx timelines)."""
+
+    def __call__(self, kind, d):
+        class _Ctx:
+            def __enter__(self_inner):
+                torch.cuda.nvtx.range_push(site_label(kind, d))
+                return self_inner
+
+            def __exit__(self_inner, *a):
+                torch.cuda.nvtx.range_pop()
+                return False
+        return _Ctx()
+
+
+class KernelTimer:
+    """CUDA events around every launch, on the stream the kernels are launched on (and an NVTX range
+    per call site when nvtx is set)."""
+
+    def __init__(self, stream, nvtx=False):
         self.stream = stream
+        self.nvtx = nvtx
         self.records = []  # (kind, site dict, start, end)
 
     def __call__(self, kind, d):
@@ -292,6 +316,8 @@ class KernelTimer:
 
         class _Ctx:
             def __enter__(self_inner):
+                if timer.nvtx:
+                    torch.cuda.nvtx.range_push(site_label(kind, d))
                 self_inner.s = torch.cuda.Event(enable_timing=True)
                 self_inner.e = torch.cuda.Event(enable_timing=True)
                 self_inner.s.record(timer.stream)
@@ -299,6 +325,8 @@ class KernelTimer:
 
             def __exit__(self_inner, *a):
                 self_inner.e.record(timer.stream)
+                if timer.nvtx:
+                    torch.cuda.nvtx.range_pop()
                 timer.records.append((kind, d, self_inner.s, self_inner.e))
                 return False
         return _Ctx()
@@ -569,6 +597,9 @@ def main():
     ap.add_argument("--no-fuse-mask", dest="fuse_mask", action="store_false",
                     help="call a1 separately instead of passing the mask to the a2 call")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--nvtx", action="store_true", help="an NVTX range per call site (timed and instrumented steps)")
+    ap.add_argument("--metrics-jsonl", default=None,
+                    help="write per-(config, site, kernel, rank) device times and GB/s of the instrumented pass here")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--kernels-out", default=None, help="write the per-kernel breakdown JSON here")
     ap.add_argument("--same-device", action="store_true",
@@ -622,14 +653,15 @@ def main():
     # (an event recorded between two kernels would cut their programmatic-dependent-launch overlap),
     # clocks sampled.  Then K more steps with an event pair around every launch give the per-kernel
     # breakdown and the roofline numbers.
-    timer = KernelTimer(stream)
+    timer = KernelTimer(stream, nvtx=args.nvtx)
+    nvtx_ranges = NvtxRanges() if args.nvtx else None
     launches0 = gist.gist_launch_count()
     with ClockSampler(dev) as clocks:
         barrier()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev0.record(stream)
         for _ in range(args.steps):
-            wl.step()
+            wl.step(nvtx_ranges)
         ev1.record(stream)
         barrier()
         launches = gist.gist_launch_count() - launches0
@@ -651,11 +683,18 @@ def main():
         if d["site"].kind == "ssdc":
             nnz_of[id(d)] = int(nnz[k])
             k += 1
+    per_site = {}  # (kind, site label) -> [ms, launches, algorithmic bytes]
     for kind, d, s, e in timer.records:
         r = per.setdefault(kind, {"ms": 0.0, "launches": 0, "algo_bytes": 0})
-        r["ms"] += s.elapsed_time(e)
+        ms = s.elapsed_time(e)
+        b = wl.algo_bytes(kind, d, nnz_of if isinstance(d, list) else nnz_of.get(id(d)))
+        r["ms"] += ms
         r["launches"] += 1
-        r["algo_bytes"] += wl.algo_bytes(kind, d, nnz_of if isinstance(d, list) else nnz_of.get(id(d)))
+        r["algo_bytes"] += b
+        ps = per_site.setdefault((kind, site_label(kind, d)), [0.0, 0, 0])
+        ps[0] += ms
+        ps[1] += 1
+        ps[2] += b
     peak, peak_src = hbm_peak()
     step_kernel_ms = sum(r["ms"] for r in per.values())
     kernels = {}
@@ -666,6 +705,15 @@ def main():
                          "frac_hbm": round(gbs / peak, 4)}
     dom = max(per, key=lambda kk: per[kk]["ms"])
     dom_gbs = per[dom]["algo_bytes"] / (per[dom]["ms"] * 1e-3) / 1e9
+    if args.metrics_jsonl:  # one line per (config, site, kernel, rank) (SURVEY.md §5 metrics)
+        with open(args.metrics_jsonl if world == 1 else f"{args.metrics_jsonl}.rank{rank}", "w") as f:
+            for (kind, label), (ms, n_l, b) in per_site.items():
+                gbs = b / (ms * 1e-3) / 1e9 if ms > 0 else 0.0
+                f.write(json.dumps({"config": cfg.key, "site": label.split(":", 1)[1], "kernel": kind, "rank": rank,
+                                    "world": world, "launches": n_l, "ms_per_launch": round(ms / n_l, 5),
+                                    "algo_bytes_per_launch": int(b // n_l), "algo_GBps": round(gbs, 1),
+                                    "frac_hbm": round(gbs / peak, 4),
+                                    "sm_mhz": clocks.summary().get("sm_mhz")}) + "\n")
 
     # ---- multi-rank: max time over ranks, sum of bytes (one collective, outside the timed region)
     tdev = torch.device("cpu") if (dist is not None and args.same_device) else dev
