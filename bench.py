@@ -607,6 +607,8 @@ def main():
                          "path on a 1-GPU box)")
     args = ap.parse_args()
     cfg = WL.CONFIGS[args.config]
+    args.default_workload = args.batch is None and args.sparsity in (None, cfg.sparsity) and \
+        args.dpr_bits in (None, cfg.dpr_bits)
     args.sparsity = cfg.sparsity if args.sparsity is None else args.sparsity
     args.dpr_bits = cfg.dpr_bits if args.dpr_bits is None else args.dpr_bits
     batch = args.batch or cfg.batch
@@ -816,7 +818,7 @@ def traffic_for(args, kind):
     """DRAM bytes per launch of the dominant kernel, from the committed ncu --set full capture of
     THIS configuration's launch (profiles/ncu_traffic.json, keyed "<config>:<kernel>:<many|per-site>"
     at the config's default batch, sparsity and DPR width); None when no such capture exists."""
-    if args.batch is not None or args.sparsity is not None or args.dpr_bits is not None:
+    if not getattr(args, "default_workload", False):
         return None
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if not os.path.exists(p):
