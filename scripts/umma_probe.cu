@@ -14,7 +14,7 @@ using namespace gist;
 // MODE 0: back-to-back MMAs; 1: a tcgen05.commit after every 4 MMAs (a K = 32-float stage);
 // 2: as 1, and before each stage wait for the commit of the stage D = 4 stages earlier (the
 // operand-ring back-pressure of a pipelined kernel); 3: D = 8; 4: D = 1 (wait for the previous
-// stage's commit: the commit round-trip latency is exposed)
+// stage's commit: the commit round-trip latency is exposed); 5: as 2 with a test_wait polling loop
 template <int N, bool BF16, int MODE>
 __global__ void probe(long long *cycles, int iters) {
     extern __shared__ __align__(1024) unsigned char smem[];
@@ -43,7 +43,10 @@ __global__ void probe(long long *cycles, int iters) {
             const uint32_t kk = (uint32_t)(i & 3);
             const int stage = i >> 2;
             constexpr int D = MODE == 3 ? 8 : MODE == 4 ? 1 : 4;
-            if (MODE >= 2 && kk == 0 && stage >= D) mbar_wait(&sbar[stage % D], (uint32_t)((stage / D) - 1) & 1u);
+            if (MODE >= 2 && MODE != 5 && kk == 0 && stage >= D) mbar_wait(&sbar[stage % D], (uint32_t)((stage / D) - 1) & 1u);
+            if (MODE == 5 && kk == 0 && stage >= D)  // the same wait with non-blocking test_wait polling
+                while (!mbar_test(&sbar[stage % D], (uint32_t)((stage / D) - 1) & 1u)) {
+                }
             const uint64_t da = umma_desc_sw128(a_addr + 32 * kk), db = umma_desc_sw128(b_addr + 32 * kk);
             if (BF16)
                 asm volatile(
@@ -54,6 +57,7 @@ __global__ void probe(long long *cycles, int iters) {
             else
                 umma_tf32(tmem_base, da, db, idesc, i > 0 ? 1u : 0u);
             if (MODE >= 1 && kk == 3) umma_commit(&sbar[stage % (MODE == 3 ? 8 : MODE == 4 ? 1 : 4)]);
+            if (MODE == 6 && kk == 3) asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         }
         umma_commit(&bar);
         mbar_wait(&bar, 0);
@@ -101,5 +105,6 @@ int main() {
     run<144, false, 2>("tf32");
     run<144, false, 3>("tf32");
     run<144, false, 4>("tf32");
+    run<144, false, 5>("tf32");
     return 0;
 }
