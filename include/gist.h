@@ -281,7 +281,8 @@ gist_status gist_dpr_decode_many(const gist_dpr_job *jobs, int32_t count, int32_
  * UNSUPPORTED unless Co % 128 == 0, Ci % 16 == 0, H*W % 4 == 0 (dY rows are TMA rows), W <= 252 and
  * the two decode slabs (16 x (R+2) x (W+2) floats each, R ~ 256/W rows) fit shared memory (W <= ~190),
  * passes in {1, 3};
- * TOO_LARGE if N*Ci*H*W or N*Co*H*W >= 2^31. */
+ * TOO_LARGE if N*Ci*H*W or N*Co*H*W >= 2^31.  N, H or W == 0: dW is set to 0 (an empty sum) with
+ * cudaMemsetAsync; Ci or Co == 0: nothing to write. */
 size_t gist_conv3x3_wgrad_workspace_bytes(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W);
 gist_status gist_conv3x3_wgrad_ssdc(const float *dy, const int32_t *row_end, const uint8_t *col, const float *val,
                                     int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W, int32_t passes,

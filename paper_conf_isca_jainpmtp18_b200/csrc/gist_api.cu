@@ -408,7 +408,14 @@ gist_status gist_conv3x3_wgrad_ssdc(const float *dy, const int32_t *row_end, con
                                     float *dw, void *workspace, size_t workspace_bytes, cudaStream_t stream) {
     if (N < 0 || Ci < 0 || Co < 0 || H < 0 || W < 0) return GIST_ERR_INVALID_ARGUMENT;
     if (passes != 1 && passes != 3) return GIST_ERR_UNSUPPORTED;
-    if (N == 0 || Ci == 0 || Co == 0 || H == 0 || W == 0) return GIST_ERR_UNSUPPORTED;
+    if (Ci == 0 || Co == 0) return GIST_OK;  // empty dW
+    if (Co % 128 || Ci % 16) return GIST_ERR_UNSUPPORTED;
+    if (N == 0 || H == 0 || W == 0) {  // no positions: dW = 0 (an empty sum)
+        if (!dw) return GIST_ERR_INVALID_ARGUMENT;
+        if (misaligned(dw)) return GIST_ERR_MISALIGNED;
+        return cudaMemsetAsync(dw, 0, (size_t)Co * Ci * 9 * sizeof(float), stream) == cudaSuccess ? GIST_OK
+                                                                                                  : GIST_ERR_CUDA;
+    }
     if (!gist::wgrad_shape_ok(N, Ci, Co, H, W)) return GIST_ERR_UNSUPPORTED;
     const int64_t nx = (int64_t)N * Ci * H * W, ny = (int64_t)N * Co * H * W;
     if (nx >= kI32Limit || ny >= kI32Limit) return GIST_ERR_TOO_LARGE;

@@ -124,6 +124,30 @@ def test_validation_without_gpu(gist):
     assert L.gist_ssdc_dpr_decode(A, B + 4, 100, 8, B + 64, None) == MISALIGNED
 
 
+def test_wgrad_validation_without_gpu(gist):
+    """f4 (gist_conv3x3_wgrad_ssdc): host-side validation returns the documented codes, no launch."""
+    L = gist.lib
+    N, Ci, Co, H, W = 2, 16, 128, 8, 8
+    ws = gist.gist_conv3x3_wgrad_workspace_bytes(N, Ci, Co, H, W)
+    assert ws > 0
+    args = lambda **k: [k.get("dy", A), B, B + 4096, B + 8192, k.get("N", N), k.get("Ci", Ci), k.get("Co", Co),
+                        k.get("H", H), k.get("W", W), k.get("passes", 3), k.get("dw", B + (1 << 20)),
+                        k.get("ws", B + (1 << 21)), k.get("wsb", ws), None]
+    assert L.gist_conv3x3_wgrad_ssdc(*args(passes=2)) == UNSUPPORTED
+    assert L.gist_conv3x3_wgrad_ssdc(*args(Co=64)) == UNSUPPORTED      # M tile of 128 output channels
+    assert L.gist_conv3x3_wgrad_ssdc(*args(Ci=24)) == UNSUPPORTED      # 16 input channels per N tile
+    assert L.gist_conv3x3_wgrad_ssdc(*args(W=300)) == UNSUPPORTED      # decode slab does not fit
+    assert L.gist_conv3x3_wgrad_ssdc(*args(H=7, W=7)) == UNSUPPORTED   # H*W % 4: dY rows are TMA rows
+    assert L.gist_conv3x3_wgrad_ssdc(*args(N=-1)) == INVALID
+    assert L.gist_conv3x3_wgrad_ssdc(*args(dy=None)) == INVALID
+    assert L.gist_conv3x3_wgrad_ssdc(*args(dy=A + 4)) == MISALIGNED
+    assert L.gist_conv3x3_wgrad_ssdc(*args(wsb=ws - 1)) == INVALID      # workspace too small
+    assert L.gist_conv3x3_wgrad_ssdc(*args(Ci=0)) == OK                 # empty dW: nothing to write
+    big = (1 << 31) // (Ci * H * W) + 1
+    assert L.gist_conv3x3_wgrad_ssdc(*args(N=big, wsb=1 << 40)) == TOO_LARGE
+    assert gist.gist_conv3x3_wgrad_workspace_bytes(N, Ci, 64, H, W) == 0
+
+
 def test_pool_geometry_overflow_rejected(gist):
     """A window whose kh*kw wraps in int32 (kh=3, kw=1431655766 -> 2 mod 2^32) must not pass the
     4-bit argmax check; huge padded spans must not wrap either."""

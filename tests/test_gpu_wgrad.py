@@ -85,3 +85,15 @@ def test_wgrad_rejects_unsupported_shapes(gist, cuda):
     x, dy = inputs(1, 16, 128, 8, 8, 0.5, 1, cuda)
     with pytest.raises(gist.GistError):
         run(gist, x, dy, 2)
+
+
+def test_wgrad_empty_batch_gives_zero(gist, cuda):
+    """No positions (N = 0): dW is the empty sum, written as zeros."""
+    dw = torch.full((128, 16, 3, 3), 7.0, device=cuda)
+    dy = torch.empty((0, 128, 8, 8), device=cuda)
+    e_i = torch.empty(0, dtype=torch.int32, device=cuda)
+    e_u = torch.empty(0, dtype=torch.uint8, device=cuda)
+    e_f = torch.empty(0, dtype=torch.float32, device=cuda)
+    out = gist.gist_conv3x3_wgrad_ssdc(dy, e_i, e_u, e_f, (0, 16, 8, 8), dw=dw)
+    torch.cuda.synchronize()
+    assert torch.equal(out, torch.zeros_like(dw))
