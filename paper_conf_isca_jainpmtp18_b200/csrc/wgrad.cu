@@ -33,6 +33,10 @@ namespace gist {
 
 namespace {
 
+#ifndef GIST_WG_ATMEM
+#define GIST_WG_ATMEM 1  // 3xTF32: A_hi / A_lo in tensor memory (the MMAs read only B from shared memory)
+#endif
+
 constexpr int kCiBlk = 16;              // input channels per CTA tile
 constexpr int kTaps = 9;                // 3x3 window
 constexpr int kN = kCiBlk * kTaps;      // 144 GEMM columns: n = tap * 16 + ci
@@ -59,8 +63,11 @@ constexpr int kDecU = 8;                     // decoder: CSR entries per lane in
 #ifndef GIST_WG_SKIP_ASPLIT
 #define GIST_WG_SKIP_ASPLIT 0
 #endif
-constexpr int kTmemCols = 512;               // two accumulators (K-tile t uses columns 256 (t % 2) + n)
-constexpr int kAccStride = 256;
+constexpr int kTmemCols = 512;               // two accumulators, then (3xTF32) the A stages
+constexpr int kAccStride = kN;               // accumulator b at columns [144 b, 144 b + 144)
+// 3xTF32 with A in tensor memory: stage s's A_hi at columns [288 + 64 s, +32), A_lo at the next 32
+// (lane = output channel, column = k), after the two accumulators: up to 3 stages in 512 columns
+__host__ __device__ constexpr uint32_t a_tmem_col(int s) { return 2u * kN + 64u * (uint32_t)s; }
 constexpr uint32_t kIdesc = idesc_tf32<kM, kN>();
 static_assert(kN % 16 == 0 && kN <= 256, "UMMA M=128 needs N % 16 == 0, N <= 256");
 
@@ -89,7 +96,7 @@ struct WgArgs {
 template <int PASSES, int NA, int NB>
 struct __align__(1024) WgSmem {
     float a[NA][kM * kKs];                          // dY tiles (TMA, 128-B swizzle): A_hi after the split
-    float alo[PASSES == 3 ? NB : 1][PASSES == 3 ? kM * kKs : 256];  // A - tf32(A) (3xTF32 only; 1 KB keeps bhi 1024-aligned)
+    float alo[PASSES == 3 && !GIST_WG_ATMEM ? NB : 1][PASSES == 3 && !GIST_WG_ATMEM ? kM * kKs : 256];  // A - tf32(A) in shared memory (3xTF32 without ATMEM; 1 KB keeps bhi 1024-aligned)
     float bhi[NB][kN * kKs];                        // im2col(X) tiles, same layout
     float blo[PASSES == 3 ? NB : 1][PASSES == 3 ? kN * kKs : 256];
     uint64_t a_full[NA], b_full[NB], b_empty[NB], acc_full[2], acc_empty[2];
@@ -117,6 +124,20 @@ __device__ __forceinline__ void wait_backoff(uint64_t *bar, uint32_t parity) {
     while (!mbar_test(bar, parity)) __nanosleep(64);
 #endif
 }
+
+#ifdef GIST_WG_TRACE
+// Timing experiment only: clock64 stamps of CTA 0 for its first kWgTrace stages: 0 MMA thread starts
+// waiting for b_full, 1 b_full observed, 2 the stage's MMAs issued, 3 builder warp 0 observed
+// b_empty, 4 builder warp 0 arrives b_full, 5 decoder warp 0 finished the K-tile (slab_full arrive)
+constexpr int kWgTrace = 256;
+__device__ long long *g_wg_trace = nullptr;
+#define WG_TRACE(g, ev)                                                                     \
+    do {                                                                                    \
+        if (g_wg_trace && blockIdx.x == 0 && (g) < kWgTrace) g_wg_trace[(g) * 8 + (ev)] = clock64(); \
+    } while (0)
+#else
+#define WG_TRACE(g, ev)
+#endif
 
 template <int PASSES, int NA, int NB, bool VEC>
 __global__ void __launch_bounds__(kThreads, 1)
@@ -215,10 +236,23 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                 if (first && gp >= 2) mbar_wait(&S.acc_empty[b], (uint32_t)((gp / 2) - 1) & 1u);
                 // one wait per stage: the builders arrive on b_full only after the stage's dY tile has
                 // landed (a_full), so b_full covers both operands
+                WG_TRACE(g, 0);
                 mbar_wait(&S.b_full[st], phb);
+                WG_TRACE(g, 1);
                 tc_fence_after();
                 const uint32_t d = tmem + (uint32_t)(b * kAccStride);
                 const uint32_t ab = smem_u32(S.a[sa]), bb = smem_u32(S.bhi[st]);
+                if constexpr (PASSES == 3 && GIST_WG_ATMEM) {
+                    static_assert(2 * kN + 64 * NB <= kTmemCols, "the A stages fit beside the accumulators");
+                    const uint32_t at = tmem + a_tmem_col(st);
+#pragma unroll
+                    for (int kk = 0; kk < kKs / 8; ++kk) {  // K = 8 tf32 per instruction = 8 TMEM columns
+                        const uint64_t db = umma_desc_sw128(bb + 32 * kk);
+                        umma_tf32_ts(d, at + 8 * kk, db, kIdesc, (!first || kk != 0) ? 1u : 0u);
+                        umma_tf32_ts(d, at + 8 * kk, umma_desc_sw128(smem_u32(S.blo[st]) + 32 * kk), kIdesc, 1u);
+                        umma_tf32_ts(d, at + 32 + 8 * kk, db, kIdesc, 1u);
+                    }
+                } else {
 #pragma unroll
                 for (int kk = 0; kk < kKs / 8; ++kk) {  // K = 8 tf32 (32 bytes) per instruction
                     const uint64_t da = umma_desc_sw128(ab + 32 * kk), db = umma_desc_sw128(bb + 32 * kk);
@@ -228,7 +262,9 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                         umma_tf32(d, umma_desc_sw128(smem_u32(S.alo[st]) + 32 * kk), db, kIdesc, 1u);
                     }
                 }
+                }
                 umma_commit(&S.b_empty[st]);  // the stage's smem (A and B) is free once these MMAs complete
+                WG_TRACE(g, 2);
                 if (last) {
                     umma_commit(&S.acc_full[b]);
                     ++gp;
@@ -406,6 +442,7 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
             pair_range(t + 1, cur_e0, cur_e1);
 #endif
             __syncwarp();
+            if (dp == 0) WG_TRACE(tl * a.spt, 5);
             if (lane == 0) mbar_arrive_1(&S.slab_full[sb]);
         }
     } else {
@@ -423,6 +460,7 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                 const int64_t g = tl * a.spt + j;
                 const int st = (int)(g % NB), sa = (int)(g % NA);
                 if (g >= NB) mbar_wait(&S.b_empty[st], (uint32_t)((g / NB) - 1) & 1u);
+                if (p == 0) WG_TRACE(g, 3);
                 const int pos = j * kKs + 4 * ch;  // the chunk's first position in the K-tile
                 uint32_t ohr = 0, ow = 0;
                 a.div_w.divmod((uint32_t)pos, ohr, ow);
@@ -485,7 +523,30 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                             *reinterpret_cast<float4 *>(bl + o) = make_float4(lo[0], lo[1], lo[2], lo[3]);
                     }
                 }
-                if (PASSES == 3 && !GIST_WG_SKIP_ASPLIT) {
+                if (PASSES == 3 && GIST_WG_ATMEM) {
+                    // A_hi = tf32_rn(A), A_lo = A - A_hi (exact) into tensor memory: builder thread = one row
+                    // (output channel) of the dY tile, its lane of the warp's TMEM lane quarter
+                    mbar_wait(&S.a_full[sa], (uint32_t)(g / NA) & 1u);
+                    const uint32_t r = 32u * (uint32_t)(warp & 3) + (uint32_t)lane;
+                    const unsigned char *arow = reinterpret_cast<const unsigned char *>(S.a[sa]);
+                    uint32_t hv[32], lv[32];
+#pragma unroll
+                    for (int c = 0; c < 8; ++c) {  // chunk c (k = 4c .. 4c+3) of row r, 128-byte swizzle
+                        const float4 x = *reinterpret_cast<const float4 *>(arow + sw128_offset(r, (uint32_t)c));
+                        const float xs[4] = {x.x, x.y, x.z, x.w};
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) {
+                            const float h = to_tf32(xs[e]);
+                            hv[4 * c + e] = __float_as_uint(h);
+                            lv[4 * c + e] = __float_as_uint(xs[e] - h);
+                        }
+                    }
+                    const uint32_t taddr = tmem + ((32u * (uint32_t)(warp & 3)) << 16) + a_tmem_col(st);
+                    tmem_st32(taddr, hv);
+                    tmem_st32(taddr + 32, lv);
+                    tmem_wait_st();
+                    tc_fence_before();
+                } else if (PASSES == 3 && !GIST_WG_SKIP_ASPLIT) {
                     // A_hi = tf32_rn(A) written back in place, A_lo = A - A_hi (exact in fp32); the layouts
                     // of a[] and alo[] are identical, so chunk by chunk
                     mbar_wait(&S.a_full[sa], (uint32_t)(g / NA) & 1u);
@@ -502,6 +563,7 @@ wgrad_ssdc_kernel(const __grid_constant__ CUtensorMap tmap_dy, const WgArgs a) {
                 if constexpr (PASSES == 1) mbar_wait(&S.a_full[sa], (uint32_t)(g / NA) & 1u);  // b_full implies A
                 fence_proxy_async_smem();  // generic smem writes -> visible to the tensor core (async proxy)
                 __syncwarp();
+                if (p == 0) WG_TRACE(g, 4);
                 if (lane == 0) mbar_arrive_1(&S.b_full[st]);
             }
             __syncwarp();
@@ -559,10 +621,13 @@ WgPlan wg_plan(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W, int32_t 
 
 int32_t slab_pitch(int32_t W) { return (W + 2 + 3) / 4 * 4; }
 
+#ifndef GIST_WG_NS3
+#define GIST_WG_NS3 2  // pipeline stages, 3xTF32 (3 with A in TMEM: no faster)
+#endif
 #ifndef GIST_WG_NS1
 #define GIST_WG_NS1 4  // pipeline stages, 1xTF32 (3xTF32: 2; a deeper dY-only ring measured slower)
 #endif
-constexpr int kNS1 = GIST_WG_NS1;
+constexpr int kNS1 = GIST_WG_NS1, kNS3 = GIST_WG_NS3;
 constexpr size_t kMaxSmemW = 227 * 1024;
 
 template <int PASSES, int NA, int NB>
@@ -595,6 +660,10 @@ cudaError_t launch_wg(const CUtensorMap &tm, const WgArgs &args, const WgPlan &P
 }
 
 }  // namespace
+
+#ifdef GIST_WG_TRACE
+extern "C" int gist_debug_wg_trace(void *buf) { return (int)cudaMemcpyToSymbol(g_wg_trace, &buf, sizeof(void *)); }
+#endif
 
 size_t wgrad_smem_bytes(int32_t N, int32_t Ci, int32_t Co, int32_t H, int32_t W, int32_t passes);
 constexpr size_t kMaxSmem = 227 * 1024;  // sm_100 opt-in dynamic shared memory per CTA
@@ -664,8 +733,10 @@ cudaError_t launch_wgrad_ssdc(const float *dy, const int32_t *row_end, const uin
     // the deeper dY ring when the slabs leave room for it
     const bool deep1 = wg_smem_bytes<1, kNS1, kNS1>(P, W) <= kMaxSmemW;
     cudaError_t e;
+    const bool deep3 = wg_smem_bytes<3, kNS3, kNS3>(P, W) <= kMaxSmemW;
     if (passes == 3) {
-        e = vec ? launch_wg<3, 2, 2, true>(tm, args, P, W, s) : launch_wg<3, 2, 2, false>(tm, args, P, W, s);
+        if (deep3) e = vec ? launch_wg<3, kNS3, kNS3, true>(tm, args, P, W, s) : launch_wg<3, kNS3, kNS3, false>(tm, args, P, W, s);
+        else e = vec ? launch_wg<3, 2, 2, true>(tm, args, P, W, s) : launch_wg<3, 2, 2, false>(tm, args, P, W, s);
     } else {
         if (deep1) e = vec ? launch_wg<1, kNS1, kNS1, true>(tm, args, P, W, s) : launch_wg<1, kNS1, kNS1, false>(tm, args, P, W, s);
         else e = vec ? launch_wg<1, 4, 4, true>(tm, args, P, W, s) : launch_wg<1, 4, 4, false>(tm, args, P, W, s);
