@@ -4,9 +4,9 @@ D=gpurun_out/r2final; mkdir -p $D
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,driver_version --format=csv,noheader > $D/gpu.txt
 timeout 1800 python -m pytest tests -q -m gpu -p no:cacheprovider > $D/pytest_gpu.log 2>&1; tail -2 $D/pytest_gpu.log
 python -c "import __graft_entry__ as g; g.smoke()" > $D/smoke.log 2>&1; tail -1 $D/smoke.log
-timeout 900 python bench.py --steps 20 --warmup 5 > $D/bench_C3.json 2> $D/bench_C3.err; cut -c1-300 $D/bench_C3.json
+timeout 900 python bench.py --steps 20 --warmup 5 --metrics-jsonl $D/metrics_C3.jsonl > $D/bench_C3.json 2> $D/bench_C3.err; cut -c1-300 $D/bench_C3.json
 for c in C2 C4 C5o C5n; do
-  timeout 600 python bench.py --config $c --steps 20 --warmup 5 --no-e2e --cpu-seconds 1 > $D/bench_$c.json 2>/dev/null
+  timeout 600 python bench.py --config $c --steps 20 --warmup 5 --no-e2e --cpu-seconds 1 --metrics-jsonl $D/metrics_$c.jsonl > $D/bench_$c.json 2>/dev/null
 done
 timeout 900 python scripts/kernel_bench.py --small --reps 20 --json $D/kernel_bench.json > $D/kernel_bench.log 2>&1; tail -1 $D/kernel_bench.log
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $D/bench_launches.csv \
