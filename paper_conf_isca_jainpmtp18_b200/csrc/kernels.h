@@ -65,7 +65,7 @@ cudaError_t launch_dpr_decode(const uint32_t *packed, int64_t n, int bits, float
 
 // pool3.cu: 3x3 windows (stride 1/2, pad 0/1, floor/ceil) through plane tiles in shared memory;
 // cudaErrorNotSupported when a plane does not fit (the caller falls back)
-bool pool3_ok(const gist_pool2d &p);
+bool pool3_ok(const gist_pool2d &p, bool fwd);
 cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p,
                              int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, uint32_t *mask, bool relu,
                              cudaStream_t s);

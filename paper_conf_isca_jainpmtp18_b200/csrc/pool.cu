@@ -759,7 +759,7 @@ cudaError_t launch_relu_maxpool_fwd(const float *x, int32_t N, int32_t C, int32_
     // geometries use the L1 forward with relu on load and the caller adds binarize(x).
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
     *mask_fused = false;
-    if (GIST_POOL3 && pool3_ok(p)) {
+    if (GIST_POOL3 && pool3_ok(p, true)) {
         const cudaError_t e = launch_pool3_fwd(x, N, C, H, W, p, Ho, Wo, out, argmax, mask, true, s);
         if (e != cudaErrorNotSupported) {
             *mask_fused = mask != nullptr;
@@ -797,7 +797,7 @@ cudaError_t launch_maxpool_fwd(const float *y, int32_t N, int32_t C, int32_t H, 
                                bool *mask_fused) {
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
     if (mask_fused) *mask_fused = false;
-    if (GIST_POOL3 && pool3_ok(p)) {
+    if (GIST_POOL3 && pool3_ok(p, true)) {
         const cudaError_t e = launch_pool3_fwd(y, N, C, H, W, p, Ho, Wo, out, argmax, mask_fused ? mask : nullptr,
                                                false, s);
         if (e != cudaErrorNotSupported) {
@@ -842,7 +842,7 @@ cudaError_t launch_pool_bwd(const float *dout, const uint32_t *argmax, const uin
                             int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo, float *dx,
                             cudaStream_t s) {
     const PoolArgs a = make_args(N, C, H, W, p, Ho, Wo);
-    if (GIST_POOL3 && pool3_ok(p)) {
+    if (GIST_POOL3 && pool3_ok(p, false)) {
         const cudaError_t e = launch_pool3_bwd(dout, argmax, mask, N, C, H, W, p, Ho, Wo, dx, s);
         if (e != cudaErrorNotSupported) return e;
     }

@@ -3,7 +3,7 @@
 //
 // Plane tiles through a TMA ring.  A tile is G whole planes; their input (forward) or their dY,
 // argmax words and mask words (backward) are contiguous ranges of the maps, so one persistent CTA
-// per (half) SM streams tile after tile into a kRS-deep shared-memory ring with 1-D bulk copies
+// per (half) SM streams tile after tile into a 2-4 stage shared-memory ring with 1-D bulk copies
 // (cp.async.bulk, issued by one thread) while its 256 threads compute the current tile from shared
 // memory: HBM sees each byte once, and the loads of the next tiles are in flight during compute.
 //   forward, stride 2: one thread per output (lanes = consecutive outputs); taps outside the input
@@ -26,6 +26,8 @@
 #include <math_constants.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "kernels.h"
@@ -45,12 +47,7 @@ constexpr int kRT = GIST_POOL3_THREADS;  // threads per CTA
 #ifndef GIST_POOL3_BWD_STRIP
 #define GIST_POOL3_BWD_STRIP 1  // stride-1 backward: column strips for tiles of >= kRT/2 columns (0: never)
 #endif
-constexpr int kRS = 3;    // ring stages
-#ifndef GIST_POOL3_STAGE_KB
-#define GIST_POOL3_STAGE_KB 32  // KB per ring stage (3 stages + extras < 113 KB: 2 CTAs per SM)
-#endif
-constexpr int kStageBytes = GIST_POOL3_STAGE_KB * 1024;
-constexpr int kStageFloats = kStageBytes / 4;
+constexpr int kMaxRS = 4;  // ring stages: a.rs <= kMaxRS stages of a.sf floats (host: ring_for)
 constexpr int kNbBytes = 12 * 1024;  // nibble bytes of one tile (stride-1 forward, backward)
 
 struct P3Args {
@@ -61,8 +58,10 @@ struct P3Args {
     int32_t hb, wb;  // stride-2 backward: 2x2 blocks per plane (rows, columns)
     int32_t PR, PC;  // backward: padded nibble-byte plane (rows, columns)
     int32_t a_off, m_off;  // backward stage layout (floats): dY at 0, argmax words, mask words
+    int32_t segs, segr;    // stride-2 forward: row segments per plane column, output rows per segment
+    int32_t rs, sf;        // ring: stages, floats per stage
     int64_t NC, tiles, n_in, n_out;
-    FastDiv div_hw, div_w, div_howo, div_wo, div_blk, div_wb;
+    FastDiv div_hw, div_w, div_howo, div_wo, div_blk, div_wb, div_seg;
 };
 
 __device__ __forceinline__ void take3(float v, int idx, float &best, int &bi) {
@@ -142,87 +141,159 @@ pool3_fwd_kernel(const float *__restrict__ y, P3Args a, float *__restrict__ out,
     pdl_enter();
     extern __shared__ __align__(128) unsigned char smp[];
     float *ring = reinterpret_cast<float *>(smp);
-    uint8_t *nbs = smp + kRS * kStageBytes;  // stride 1: nibble bytes of the tile
-    uint64_t *full = reinterpret_cast<uint64_t *>(smp + kRS * kStageBytes + (S == 1 ? kNbBytes : 0));
+    uint8_t *nbs = smp + (size_t)a.rs * a.sf * 4;  // nibble bytes of the tile (one per output)
+    uint64_t *full = reinterpret_cast<uint64_t *>(nbs + kNbBytes);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const float ninf = -CUDART_INF_F;
     if (tid == 0) {
-        for (int s = 0; s < kRS; ++s) mbar_init(&full[s], 1);
+        for (int s = 0; s < a.rs; ++s) mbar_init(&full[s], 1);
         fence_mbar_init();
     }
     __syncthreads();
+    FwdTile *desc = reinterpret_cast<FwdTile *>(full + kMaxRS);  // per stage: the tile it holds
     const int64_t mine = a.tiles > blockIdx.x ? (a.tiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
-    auto issue = [&](int64_t j) {
+    // one thread computes a tile's ranges when it issues the tile's copy and leaves them with the
+    // stage (the full barrier's arrive releases them to the consumers)
+    auto issue = [&](int64_t j, int st) {
         const FwdTile t = fwd_tile(a, blockIdx.x + j * gridDim.x);
-        const int st = (int)(j % kRS);
+        desc[st] = t;
         const uint32_t b = ring_bytes(t.lo, t.hi);
         mbar_arrive_expect_tx(&full[st], b);
-        if (b) ring_copy(ring + (size_t)st * kStageFloats, y + (t.lo & ~3ll), b, &full[st]);
+        if (b) ring_copy(ring + (size_t)st * a.sf, y + (t.lo & ~3ll), b, &full[st]);
     };
     if (tid == 0)
-        for (int64_t j = 0; j < kRS && j < mine; ++j) issue(j);
+        for (int64_t j = 0; j < a.rs && j < mine; ++j) issue(j, (int)j);
+    int st = 0;
+    uint32_t ph = 0;
     for (int64_t j = 0; j < mine; ++j) {
-        const int st = (int)(j % kRS);
-        float *R = ring + (size_t)st * kStageFloats;
-        const FwdTile t = fwd_tile(a, blockIdx.x + j * gridDim.x);
+        float *R = ring + (size_t)st * a.sf;
+        mbar_wait(&full[st], ph);
+        const FwdTile t = desc[st];
         const int64_t sb = t.lo & ~3ll;  // stage index of element e: e - sb
-        mbar_wait(&full[st], (uint32_t)(j / kRS) & 1u);
         if (tail_fill(R, y, t.lo, t.hi, 0)) fence_proxy_async_smem();
         __syncthreads();
-        // a1 mask words [ia/32, ib/32) (relu(y) > 0 iff y > 0): one staged float4 per lane, the 8
-        // lanes of a word OR their bits together (conflict-free 128-bit shared loads)
+        // a1 mask words [ia/32, ib/32) (relu(y) > 0 iff y > 0): lane l of a warp reads element
+        // 32 w + l of each of 4 words (conflict-free), one ballot per word; tile-local 32-bit indices
         if (MASK) {
-            const int64_t q0 = t.ia >> 2, q1 = ((t.ib + 31) >> 5) << 3;  // quads of the owned words
-            for (int64_t qb = q0; qb < q1; qb += kRT) {
-                const int64_t q = qb + tid;  // q0 % 8 == 0 and kRT % 8 == 0: lanes 8g..8g+7 = one word
-                uint32_t bits = 0;
-                if (q < q1) {
-                    const float4 f = *reinterpret_cast<const float4 *>(R + (4 * q - sb));
-                    const int64_t e = 4 * q;  // O1: y > 0 (NaN, -0.0 -> 0); elements past the map read 0
-                    bits = (f.x > 0.0f && e < t.hi ? 1u : 0u) | (f.y > 0.0f && e + 1 < t.hi ? 2u : 0u) |
-                           (f.z > 0.0f && e + 2 < t.hi ? 4u : 0u) | (f.w > 0.0f && e + 3 < t.hi ? 8u : 0u);
+            const int nw = (int)((t.ib - t.ia + 31) >> 5);
+            const int lim = (int)(t.hi - t.ia);  // staged elements from ia (the map ends there)
+            const float *E = R + (t.ia - sb);
+            uint32_t *mw = mask + (t.ia >> 5);
+            // every tile but the map's last: whole groups of 4 words without bounds tests
+            const int nw4 = lim >= 32 * nw ? (nw & ~3) : 0;
+            for (int w0 = warp * 4; w0 < nw4; w0 += kRT / 8) {
+                const float *e = E + 32 * w0 + lane;  // O1: y > 0 (NaN, -0.0 -> 0)
+                uint32_t word = 0;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const uint32_t b = __ballot_sync(kFull, e[32 * k] > 0.0f);
+                    word = lane == k ? b : word;
                 }
-                bits <<= 4 * (lane & 7);
-                bits |= __shfl_xor_sync(kFull, bits, 1);
-                bits |= __shfl_xor_sync(kFull, bits, 2);
-                bits |= __shfl_xor_sync(kFull, bits, 4);
-                if ((lane & 7) == 0 && q < q1) mask[q >> 3] = bits;
+                if (lane < 4) mw[w0 + lane] = word;
+            }
+            for (int w = nw4 + warp; w < nw; w += kRT / 32) {  // the rest, elements past the map read 0
+                const int e = 32 * w + lane;
+                const uint32_t b = __ballot_sync(kFull, e < lim && E[e] > 0.0f);
+                if (lane == 0) mw[w] = b;
             }
         }
         const int64_t olo = t.p0 * a.HoWo;
         if (S == 2) {
-            // one thread per owned output, 32 consecutive outputs per warp (oa % 8 == 0)
-            const int la = (int)(t.oa - olo), lb = (int)(t.ob - olo);
-            for (int c = la + warp * 32; c < lb; c += kRT) {
-                const int l = c + lane;
-                uint32_t nib = 0;
-                if (l < lb) {
-                    uint32_t pl, rem, oh, ow;
-                    a.div_howo.divmod((uint32_t)l, pl, rem);
-                    a.div_wo.divmod(rem, oh, ow);
-                    const int ih0 = (int)oh * 2 - a.P, iw0 = (int)ow * 2 - a.P;
-                    const float *pb = R + ((t.p0 + pl) * a.HW - sb);
-                    int bi = max(0, -ih0) * 3 + max(0, -iw0);
-                    float best = ninf;
-#pragma unroll
-                    for (int dy = 0; dy < 3; ++dy) {
-                        const int ih = ih0 + dy;
-                        const bool rok = !CHECK || (ih >= 0 && ih < a.H);
-#pragma unroll
-                        for (int dx = 0; dx < 3; ++dx) {
-                            const int iw = iw0 + dx;
-                            const bool ok = rok && (!CHECK || (iw >= 0 && iw < a.W));
-                            const float v = ok ? act3<RELU>(pb[ok ? ih * a.W + iw : 0]) : ninf;
-                            take3(v, 3 * dy + dx, best, bi);
-                        }
+            // one thread per (plane, output column, row segment) walks down the segment's output
+            // rows: input row 2 oh - P + 2 of one output is row 2 (oh + 1) - P of the next, so each
+            // step scans two new input rows (separable, as for stride 1).  Nibble bytes go to
+            // shared memory by output index - olo8 (word boundaries 8-byte aligned), then packed.
+            const int64_t olo8 = olo & ~7ll;
+            uint8_t *nb0 = nbs + (olo - olo8);
+            const float *P0 = R + (t.lo - sb);  // plane 0 of the tile
+            float *otile = out + olo;
+            const int items = t.np * a.segs * a.Wo;
+            for (int it = tid; it < items; it += kRT) {
+                uint32_t ps, ow, pl, sg;
+                a.div_wo.divmod((uint32_t)it, ps, ow);
+                a.div_seg.divmod(ps, pl, sg);
+                const int oh0 = (int)sg * a.segr, oh1 = min(a.Ho, oh0 + a.segr);
+                const float *pb = P0 + (int)pl * a.HW;
+                const int iw0 = 2 * (int)ow - a.P;
+                const int dx0 = max(0, -iw0);
+                int oo = (int)pl * a.HoWo + (int)ow;  // tile-local output index
+                if (!CHECK) {
+                    // every window inside the plane: the first tap of a row starts its scan, the
+                    // first row starts the window's (equal to the -inf start of R3's scan)
+                    const float *r = pb + 2 * oh0 * a.W + iw0;
+                    oo += oh0 * a.Wo;
+                    float hv0 = act3<RELU>(r[0]);
+                    int hx0 = 0;
+                    take3(act3<RELU>(r[1]), 1, hv0, hx0);
+                    take3(act3<RELU>(r[2]), 2, hv0, hx0);
+                    for (int oh = oh0; oh < oh1; ++oh) {
+                        r += a.W;
+                        float hv1 = act3<RELU>(r[0]), hv2 = act3<RELU>(r[a.W]);
+                        int hx1 = 0, hx2 = 0;
+                        take3(act3<RELU>(r[1]), 1, hv1, hx1);
+                        take3(act3<RELU>(r[a.W + 1]), 1, hv2, hx2);
+                        take3(act3<RELU>(r[2]), 2, hv1, hx1);
+                        take3(act3<RELU>(r[a.W + 2]), 2, hv2, hx2);
+                        float best = hv0;
+                        int bi = hx0;
+                        take3(hv1, 3 + hx1, best, bi);
+                        take3(hv2, 6 + hx2, best, bi);
+                        otile[oo] = best;
+                        nb0[oo] = (uint8_t)bi;
+                        oo += a.Wo;
+                        hv0 = hv2, hx0 = hx2;
+                        r += a.W;
                     }
-                    out[olo + l] = best;
-                    nib = (uint32_t)bi << (4 * (lane & 7));
+                    continue;
                 }
-                nib |= __shfl_xor_sync(kFull, nib, 1);
-                nib |= __shfl_xor_sync(kFull, nib, 2);
-                nib |= __shfl_xor_sync(kFull, nib, 4);
-                if ((lane & 7) == 0 && l < lb) arg[(olo + l) >> 3] = nib;
+                float hv0, hv1, hv2;
+                int hx0, hx1, hx2;
+                hscan<RELU>(pb + (2 * oh0 - a.P) * a.W, 2 * oh0 - a.P, iw0, a, hv0, hx0);
+                for (int oh = oh0; oh < oh1; ++oh) {
+                    const int ih1 = 2 * oh - a.P + 1;
+                    hscan<RELU>(pb + ih1 * a.W, ih1, iw0, a, hv1, hx1);
+                    hscan<RELU>(pb + (ih1 + 1) * a.W, ih1 + 1, iw0, a, hv2, hx2);
+                    float best = ninf;
+                    int bi = max(0, a.P - 2 * oh) * 3 + dx0;  // first in-bounds position (all -inf)
+                    take3(hv0, hx0, best, bi);
+                    take3(hv1, 3 + hx1, best, bi);
+                    take3(hv2, 6 + hx2, best, bi);
+                    otile[oo + oh * a.Wo] = best;
+                    nb0[oo + oh * a.Wo] = (uint8_t)bi;
+                    hv0 = hv2, hx0 = hx2;
+                }
+            }
+            // the outputs of plane p0 + np in this tile's last argmax word (<= 7, nibbles only)
+            const int ext = (int)(t.ob - (t.p0 + t.np) * a.HoWo);
+            if (tid < ext) {
+                uint32_t oh, ow;
+                a.div_wo.divmod((uint32_t)tid, oh, ow);
+                const int ih0 = (int)oh * 2 - a.P, iw0 = (int)ow * 2 - a.P;
+                const float *pb = P0 + t.np * a.HW;
+                int bi = max(0, -ih0) * 3 + max(0, -iw0);
+                float best = ninf;
+#pragma unroll
+                for (int dy = 0; dy < 3; ++dy)
+#pragma unroll
+                    for (int dx = 0; dx < 3; ++dx) {
+                        const int ih = ih0 + dy, iw = iw0 + dx;
+                        const bool ok = ih >= 0 && ih < a.H && iw >= 0 && iw < a.W;
+                        take3(ok ? act3<RELU>(pb[ok ? ih * a.W + iw : 0]) : ninf, 3 * dy + dx, best, bi);
+                    }
+                nb0[t.np * a.HoWo + tid] = (uint8_t)bi;
+            }
+            __syncthreads();
+            // pack the owned words [oa/8, ob/8): 8 nibble bytes each (one aligned 64-bit load);
+            // only the map's last word can be partial (its pad nibbles are 0)
+            const int w0 = (int)((t.oa - olo8) >> 3), w1 = (int)((t.ob - olo8 + 7) >> 3);
+            const int nvalid = (int)(t.ob - olo8);  // bytes written from olo8 on (last word of the map)
+            for (int w = w0 + tid; w < w1; w += kRT) {
+                const uint2 b = *reinterpret_cast<const uint2 *>(nbs + 8 * w);
+                const uint32_t lo4 = (b.x & 0xfu) | ((b.x >> 4) & 0xf0u) | ((b.x >> 8) & 0xf00u) | ((b.x >> 12) & 0xf000u);
+                const uint32_t hi4 = (b.y & 0xfu) | ((b.y >> 4) & 0xf0u) | ((b.y >> 8) & 0xf00u) | ((b.y >> 12) & 0xf000u);
+                const int valid = nvalid - 8 * w;
+                const uint32_t keep = valid >= 8 ? ~0u : ((1u << (4 * valid)) - 1u);
+                arg[(olo8 >> 3) + w] = (lo4 | (hi4 << 16)) & keep;
             }
         } else {
             // stride 1 (G * HoWo % 8 == 0: every word whole in the tile): one thread per output column
@@ -267,7 +338,8 @@ pool3_fwd_kernel(const float *__restrict__ y, P3Args a, float *__restrict__ out,
             }
         }
         __syncthreads();  // stage st (and the nibble bytes) consumed
-        if (tid == 0 && j + kRS < mine) issue(j + kRS);
+        if (tid == 0 && j + a.rs < mine) issue(j + a.rs, st);
+        if (++st == a.rs) st = 0, ph ^= 1u;
     }
 }
 
@@ -299,19 +371,19 @@ pool3_bwd_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ ar
     pdl_enter();
     extern __shared__ __align__(128) unsigned char smp[];
     float *ring = reinterpret_cast<float *>(smp);
-    uint8_t *nbb = smp + kRS * kStageBytes;  // padded nibble-byte planes of the tile
-    uint64_t *full = reinterpret_cast<uint64_t *>(smp + kRS * kStageBytes + kNbBytes);
+    uint8_t *nbb = smp + (size_t)a.rs * a.sf * 4;  // padded nibble-byte planes of the tile
+    uint64_t *full = reinterpret_cast<uint64_t *>(nbb + kNbBytes);
     const int tid = threadIdx.x;
     if (tid == 0) {
-        for (int s = 0; s < kRS; ++s) mbar_init(&full[s], 1);
+        for (int s = 0; s < a.rs; ++s) mbar_init(&full[s], 1);
         fence_mbar_init();
     }
     __syncthreads();
     const int64_t mine = a.tiles > blockIdx.x ? (a.tiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
     auto issue = [&](int64_t j) {
         const BwdTile t = bwd_tile(a, blockIdx.x + j * gridDim.x);
-        const int st = (int)(j % kRS);
-        float *R = ring + (size_t)st * kStageFloats;
+        const int st = (int)(j % a.rs);
+        float *R = ring + (size_t)st * a.sf;
         const uint32_t bd = ring_bytes(t.olo, t.ohi), ba = ring_bytes(t.aw_lo, t.aw_hi);
         const uint32_t bm = MASK ? ring_bytes(t.mw_lo, t.mw_hi) : 0u;
         mbar_arrive_expect_tx(&full[st], bd + ba + bm);
@@ -320,12 +392,12 @@ pool3_bwd_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ ar
         if (bm) ring_copy(R + a.m_off, mask + (t.mw_lo & ~3ll), bm, &full[st]);
     };
     if (tid == 0)
-        for (int64_t j = 0; j < kRS && j < mine; ++j) issue(j);
+        for (int64_t j = 0; j < a.rs && j < mine; ++j) issue(j);
     for (int64_t j = 0; j < mine; ++j) {
-        const int st = (int)(j % kRS);
-        float *R = ring + (size_t)st * kStageFloats;
+        const int st = (int)(j % a.rs);
+        float *R = ring + (size_t)st * a.sf;
         const BwdTile t = bwd_tile(a, blockIdx.x + j * gridDim.x);
-        mbar_wait(&full[st], (uint32_t)(j / kRS) & 1u);
+        mbar_wait(&full[st], (uint32_t)(j / a.rs) & 1u);
         {
             uint32_t *RA = reinterpret_cast<uint32_t *>(R + a.a_off), *RM = reinterpret_cast<uint32_t *>(R + a.m_off);
             bool wrote = tail_fill(R, dout, t.olo, t.ohi, 0);
@@ -483,7 +555,7 @@ pool3_bwd_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ ar
             }
         }
         __syncthreads();  // stage st consumed
-        if (tid == 0 && j + kRS < mine) issue(j + kRS);
+        if (tid == 0 && j + a.rs < mine) issue(j + a.rs);
     }
 }
 
@@ -518,26 +590,62 @@ P3Args p3_args(int32_t N, int32_t C, int32_t H, int32_t W, const gist_pool2d &p,
 
 // Planes per tile: as many as a stage holds (`per_plane` floats each, `fixed` floats of slack),
 // a multiple of `unit`, but no more than keeps ~4 tiles per CTA.  0: one unit does not fit.
-int32_t choose_g(int64_t NC, int64_t per_plane, int64_t fixed, int32_t unit, int64_t ctas) {
-    const int64_t fit = (kStageFloats - fixed) / per_plane;
+int32_t choose_g(int64_t NC, int64_t per_plane, int64_t fixed, int32_t unit, int64_t ctas, int64_t stage_floats) {
+    const int64_t fit = (stage_floats - fixed) / per_plane;
     if (fit < unit) return 0;
     int64_t g = std::min<int64_t>(fit, std::max<int64_t>(1, NC / (4 * ctas)));
     g = std::max<int64_t>(unit, g / unit * unit);
     return (int32_t)g;
 }
 
-size_t ring_smem(bool nibble_bytes) { return (size_t)kRS * kStageBytes + (nibble_bytes ? kNbBytes : 0) + 64; }
+// Ring per kernel kind (stages x KB per stage), measured on B200 (AlexNet / NiN / GoogLeNet maps):
+// stride-2 forward 2 x 48 KB (was 3 x 32: AlexNet relu1 62 -> 52 us, fewer per-tile overheads),
+// the others 3 x 32 KB.  GIST_POOL3_RING="f1=3x32,f2=2x48,b1=3x32,b2=3x32" overrides (tuning).
+struct Ring {
+    int rs, kb;
+};
+Ring ring_for(bool fwd, int S) {
+    static Ring cfg[2][2] = {{{3, 32}, {3, 32}}, {{3, 32}, {2, 48}}};  // [fwd][S - 1]
+    static const bool parsed = [] {
+        if (const char *e = getenv("GIST_POOL3_RING")) {
+            for (const char *q = e; *q;) {
+                char kind = 0;
+                int sd = 0, rs = 0, kb = 0, used = 0;
+                if (sscanf(q, "%c%d=%dx%d%n", &kind, &sd, &rs, &kb, &used) == 4 && (sd == 1 || sd == 2) &&
+                    rs >= 2 && rs <= kMaxRS && kb >= 8 && kb <= 96)
+                    cfg[kind == 'f'][sd - 1] = Ring{rs, kb};
+                q += used ? used : 1;
+                while (*q == ',') ++q;
+            }
+        }
+        return true;
+    }();
+    (void)parsed;
+    return cfg[fwd ? 1 : 0][S - 1];
+}
+size_t ring_smem(const Ring &r) {
+    return (size_t)r.rs * r.kb * 1024 + kNbBytes + 8 * kMaxRS + kMaxRS * sizeof(FwdTile);
+}
+int64_t resident_ctas(size_t smem) {
+    return std::max<int64_t>(1, std::min<int64_t>(2, (int64_t)(227 * 1024) / (int64_t)(smem + 1024))) * num_sms();
+}
 
 }  // namespace
 
 // Used for stride 1 (GoogLeNet's in-module pools): forward 16% -> 28% of HBM, backward 12% -> 21%
-// (inc3a b64, isolated).  The stride-2 path is kept for GIST_POOL3_S2=1 only: the L1 kernels of
-// pool.cu measured faster there (AlexNet relu1 b128 forward 52% vs 39%, backward 36% vs 30%).
+// (inc3a b64, isolated), and for the stride-2 forward (column walker, 2 x 48 KB ring): AlexNet relu1
+// b128 56 -> 52 us, with the a1 mask 72 (L1 kernel + binarize) -> 68 us; NiN relu_cccp2 b256
+// 144 -> 125 us.  The stride-2 backward stays on pool.cu's 2x2-block kernel (82 vs 100 us on
+// AlexNet relu1) unless GIST_POOL3_S2_BWD=1.
 #ifndef GIST_POOL3_S2
-#define GIST_POOL3_S2 0
+#define GIST_POOL3_S2 1
 #endif
-bool pool3_ok(const gist_pool2d &p) {
-    return p.kh == 3 && p.kw == 3 && p.sh == p.sw && (p.sh == 1 || (GIST_POOL3_S2 && p.sh == 2)) && p.ph == p.pw &&
+#ifndef GIST_POOL3_S2_BWD
+#define GIST_POOL3_S2_BWD 0
+#endif
+bool pool3_ok(const gist_pool2d &p, bool fwd) {
+    const bool s2 = fwd ? GIST_POOL3_S2 : GIST_POOL3_S2_BWD;
+    return p.kh == 3 && p.kw == 3 && p.sh == p.sw && (p.sh == 1 || (s2 && p.sh == 2)) && p.ph == p.pw &&
            p.ph <= 1;
 }
 
@@ -547,7 +655,11 @@ cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, in
                              int32_t Ho, int32_t Wo, float *out, uint32_t *argmax, uint32_t *mask, bool relu,
                              cudaStream_t s) {
     P3Args a = p3_args(N, C, H, W, p, Ho, Wo);
-    const int64_t ctas = 2 * (int64_t)num_sms();
+    const Ring ring = ring_for(true, a.S);
+    a.rs = ring.rs;
+    a.sf = ring.kb * 256;
+    const size_t smem = ring_smem(ring);
+    const int64_t ctas = resident_ctas(smem);
     if (a.S == 1) {
         // whole argmax (and mask) words per tile; the nibble bytes of a tile fit kNbBytes
         int32_t unit = 8 / gcd_i(a.HoWo, 8);
@@ -555,7 +667,7 @@ cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, in
             const int32_t mu = 32 / gcd_i(a.HW, 32);
             unit = unit * mu / gcd_i(unit, mu);
         }
-        a.G = choose_g(a.NC, a.HW, 64, unit, ctas);
+        a.G = choose_g(a.NC, a.HW, 64, unit, ctas, a.sf);
         while (a.G > unit && (int64_t)a.G * a.HoWo > kNbBytes) a.G -= unit;
         if (a.G == 0 || (int64_t)a.G * a.HoWo > kNbBytes) return cudaErrorNotSupported;
     } else {
@@ -565,13 +677,19 @@ cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, in
         if (a.HoWo % 8) xr = std::min(H, (std::min(6, a.HoWo - 1) / Wo) * a.S - a.P + 3);
         if (mask && a.HW % 32) xr = std::max(xr, std::min(H, (30 + W) / W));
         a.xrows = xr;
-        a.G = choose_g(a.NC, a.HW, 64 + (int64_t)xr * W + 32, 1, ctas);
-        if (a.G == 0) return cudaErrorNotSupported;
+        a.G = choose_g(a.NC, a.HW, 64 + (int64_t)xr * W + 32, 1, ctas, a.sf);
+        while (a.G > 1 && (int64_t)a.G * a.HoWo + 14 > kNbBytes) --a.G;
+        if (a.G == 0 || (int64_t)a.G * a.HoWo + 14 > kNbBytes) return cudaErrorNotSupported;
+        // row segments: about one (plane, column, segment) item per thread
+        const int64_t cols = (int64_t)a.G * Wo;
+        const int32_t want = (int32_t)std::max<int64_t>(1, std::min<int64_t>(Ho, kRT / cols));
+        a.segr = (Ho + want - 1) / want;
+        a.segs = (Ho + a.segr - 1) / a.segr;
+        a.div_seg = FastDiv::make((uint32_t)a.segs);
     }
     a.tiles = ceil_div(a.NC, a.G);
     // every window inside the input: no bounds tests (AlexNet's floor-mode 3x3/s2)
     const bool check = !(a.P == 0 && (Ho - 1) * a.S + 3 <= H && (Wo - 1) * a.S + 3 <= W);
-    const size_t smem = ring_smem(a.S == 1);
     const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(a.tiles, ctas));
 #define P3F(S_, M_, R_, C_)                                                                                 \
     do {                                                                                                    \
@@ -609,7 +727,11 @@ cudaError_t launch_pool3_bwd(const float *dout, const uint32_t *argmax, const ui
                              int32_t H, int32_t W, const gist_pool2d &p, int32_t Ho, int32_t Wo, float *dx,
                              cudaStream_t s) {
     P3Args a = p3_args(N, C, H, W, p, Ho, Wo);
-    const int64_t ctas = 2 * (int64_t)num_sms();
+    const Ring ring = ring_for(false, a.S);
+    a.rs = ring.rs;
+    a.sf = ring.kb * 256;
+    const size_t smem = ring_smem(ring);
+    const int64_t ctas = resident_ctas(smem);
     if (a.S == 2) {
         a.hb = (H + a.P + 1) / 2;
         a.wb = (W + a.P + 1) / 2;
@@ -624,14 +746,13 @@ cudaError_t launch_pool3_bwd(const float *dout, const uint32_t *argmax, const ui
     // stage floats per plane: dY (HoWo) + argmax words (HoWo/8) + mask words (HW/32), and the
     // phases / round-ups of the three ranges
     const int64_t per_plane = (int64_t)a.HoWo + (a.HoWo + 7) / 8 + (mask ? (a.HW + 31) / 32 : 0) + 1;
-    a.G = choose_g(a.NC, per_plane, 64, 1, ctas);
+    a.G = choose_g(a.NC, per_plane, 64, 1, ctas, a.sf);
     while (a.G > 1 && (int64_t)a.G * a.PR * a.PC > kNbBytes) --a.G;
     if (a.G == 0 || (int64_t)a.G * a.PR * a.PC > kNbBytes) return cudaErrorNotSupported;
     a.tiles = ceil_div(a.NC, a.G);
     const int64_t G = a.G;
     a.a_off = (int32_t)((G * a.HoWo + 8 + 3) & ~3ll);
     a.m_off = (int32_t)((a.a_off + (G * a.HoWo + 7) / 8 + 8 + 3) & ~3ll);
-    const size_t smem = ring_smem(true);
     const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(a.tiles, ctas));
 #define P3B(S_, M_)                                                                                          \
     do {                                                                                                     \

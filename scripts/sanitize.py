@@ -28,6 +28,11 @@ for shape in [(3, 5, 7, 7), (2, 9, 14, 14)]:
     y = WL.relu_map(shape, 0.5, 3, dev)
     out, arg, mask = gist.gist_maxpool_fwd_argmax(y, WL.P3S1P1, fuse_mask=True)
     gist.gist_pool_relu_bwd(torch.randn_like(out), arg, mask, shape, WL.P3S1P1)
+# 3x3/s2 plane-tile pools (pool3.cu when enabled): ragged tiles, words across planes, ceil, padding 1
+for g, shape in [(WL.P3S2, (3, 7, 27, 27)), (WL.P3S2C, (2, 5, 14, 14)), ((3, 3, 2, 2, 1, 1, 0), (2, 3, 15, 15))]:
+    y = WL.relu_map(shape, 0.5, 4, dev)
+    out, arg, mask = gist.gist_maxpool_fwd_argmax(y, g, fuse_mask=True)
+    gist.gist_pool_relu_bwd(torch.randn_like(out), arg, mask, shape, g)
 # f4: decode-in-GEMM weight gradient, both precisions, a vector (W % 4 == 0) and a scalar shape
 for N, Ci, Co, H, W in [(1, 16, 128, 8, 8), (1, 16, 128, 6, 10)]:
     x = WL.relu_map((N, Ci, H, W), 0.8, 5, dev)
