@@ -597,6 +597,9 @@ def main():
     ap.add_argument("--no-fuse-mask", dest="fuse_mask", action="store_false",
                     help="call a1 separately instead of passing the mask to the a2 call")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--eager", action="store_true",
+                    help="launch every timed step's C-ABI calls from Python (default: capture one step in a "
+                         "CUDA graph and replay it, so host launch overhead stays out of the device timing)")
     ap.add_argument("--nvtx", action="store_true", help="an NVTX range per call site (timed and instrumented steps)")
     ap.add_argument("--metrics-jsonl", default=None,
                     help="write per-(config, site, kernel, rank) device times and GB/s of the instrumented pass here")
@@ -657,16 +660,39 @@ def main():
     # breakdown and the roofline numbers.
     timer = KernelTimer(stream, nvtx=args.nvtx)
     nvtx_ranges = NvtxRanges() if args.nvtx else None
+    # One step captured as a CUDA graph (the C-ABI calls launch on the capturing stream; PDL edges
+    # are kept), replayed K times: the device executes exactly the eager step's kernels, without the
+    # per-call Python/ctypes gaps between them.  --eager (or --nvtx) times Python-launched steps.
+    graph, graph_note, per_step_launches = None, None, None
+    if not (args.eager or args.nvtx):
+        try:
+            c0 = gist.gist_launch_count()
+            g_ = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g_):
+                wl.step()
+            per_step_launches = gist.gist_launch_count() - c0
+            for _ in range(2):
+                g_.replay()
+            torch.cuda.synchronize()
+            graph = g_
+        except Exception as ex:  # noqa: BLE001  (reported in the line, timed eagerly instead)
+            graph_note = f"graph capture failed ({type(ex).__name__}: {str(ex)[:120]}); eager launches"
+            torch.cuda.synchronize()
     launches0 = gist.gist_launch_count()
     with ClockSampler(dev) as clocks:
         barrier()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev0.record(stream)
         for _ in range(args.steps):
-            wl.step(nvtx_ranges)
+            if graph is not None:
+                graph.replay()
+            else:
+                wl.step(nvtx_ranges)
         ev1.record(stream)
         barrier()
         launches = gist.gist_launch_count() - launches0
+        if graph is not None:
+            launches = per_step_launches * args.steps
         elapsed_ms = ev0.elapsed_time(ev1)
         ev2, ev3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev2.record(stream)
@@ -799,6 +825,8 @@ def main():
         "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": launches,
+        "launch": ("cuda_graph: one captured step replayed K times (%d libgist launches per step)" % per_step_launches
+                   if graph is not None else (graph_note or "eager: C-ABI calls from Python every step")),
         "clocks": clocks.summary(),
         "compression": wl.compression(nnz),
         "kernels": kernels,

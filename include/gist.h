@@ -114,10 +114,12 @@ gist_status gist_binarize_encode(const float *y, int64_t n, uint32_t *mask, cuda
  *          written too — in the same pass (one read of y) for 2x2/s2 unpadded pools with H and
  *          W even whose warp unit of BR whole row pairs fits 512 items: BR*W/V <= 512 with
  *          V = 4 if W % 4 == 0 else 2, a = 16/gcd(W,16), BR = a*max(1, floor(256/(a*W/V)))
- *          (every VGG16 and OverFeat map), and for 3x3 stride-1 windows with padding 0 or 1
- *          (GoogLeNet's in-module pools: whole-plane tiles staged in shared memory, when the
- *          planes of one tile, a multiple of 32/gcd(H*W,32) and of 8/gcd(Ho*Wo,8), fit a 32 KB
- *          stage); otherwise by a second kernel over y.
+ *          (every VGG16 and OverFeat map), and for 3x3 windows of stride 1 or 2 with padding
+ *          0 or 1 (AlexNet, NiN, GoogLeNet: whole-plane tiles staged in shared memory) when
+ *          the planes of one tile fit a ring stage: stride 1, a multiple of 32/gcd(H*W,32)
+ *          and of 8/gcd(Ho*Wo,8) planes in 32 KB with G*Ho*Wo <= 12288; stride 2, one plane
+ *          plus the <= 3 rows of the next in 48 KB (H*W up to ~12000: not GoogLeNet's
+ *          112x112 stem); otherwise by a second kernel over y.
  * TOO_LARGE if N*C*H*W >= 2^31. */
 gist_status gist_maxpool_fwd_argmax(const float *y, int32_t N, int32_t C, int32_t H, int32_t W,
                                     const gist_pool2d *p, float *out, uint32_t *argmax,
@@ -130,7 +132,7 @@ gist_status gist_maxpool_fwd_argmax(const float *y, int32_t N, int32_t C, int32_
  * (R21: torch's ReLU; -0.0 and NaN pass through), reading x once: out = the window max of
  * relu(x), argmax = its 4-bit in-window index, mask bit i = (x[i] > 0) (= relu(x)[i] > 0).
  * mask is required.  One kernel for 2x2/s2 with even H and W (VGG16, OverFeat) and for the 3x3
- * stride-1 pools that gist_maxpool_fwd_argmax fuses; other geometries run the forward with relu
+ * pools that gist_maxpool_fwd_argmax fuses; other geometries run the forward with relu
  * on load plus a binarize pass over x.  Errors as
  * gist_maxpool_fwd_argmax; mask == NULL -> INVALID_ARGUMENT. */
 gist_status gist_relu_maxpool_fwd_argmax(const float *x, int32_t N, int32_t C, int32_t H, int32_t W,

@@ -44,11 +44,16 @@ constexpr int kRT = GIST_POOL3_THREADS;  // threads per CTA
 #ifndef GIST_POOL3_BWD_SEG
 #define GIST_POOL3_BWD_SEG 0  // 1: row segments for tiles with few columns (measured slower in the C4 step)
 #endif
+#ifndef GIST_POOL3_BWD_HITS
+#define GIST_POOL3_BWD_HITS 1  // backward through hit masks (0: nibble planes + per-input tests)
+#endif
 #ifndef GIST_POOL3_BWD_STRIP
 #define GIST_POOL3_BWD_STRIP 1  // stride-1 backward: column strips for tiles of >= kRT/2 columns (0: never)
 #endif
 constexpr int kMaxRS = 4;  // ring stages: a.rs <= kMaxRS stages of a.sf floats (host: ring_for)
-constexpr int kNbBytes = 12 * 1024;  // nibble bytes of one tile (stride-1 forward, backward)
+constexpr int kNbBytes = 12 * 1024;   // nibble bytes of one tile (forward, nibble-plane backward)
+constexpr int kHitBytes = 16 * 1024;  // hit masks of one tile (backward): 16 bits (S = 1) or 4 bits per input
+constexpr int kAuxBytes = kHitBytes;  // the per-CTA area after the ring (>= kNbBytes)
 
 struct P3Args {
     int32_t H, W, Ho, Wo, S, P;
@@ -142,7 +147,7 @@ pool3_fwd_kernel(const float *__restrict__ y, P3Args a, float *__restrict__ out,
     extern __shared__ __align__(128) unsigned char smp[];
     float *ring = reinterpret_cast<float *>(smp);
     uint8_t *nbs = smp + (size_t)a.rs * a.sf * 4;  // nibble bytes of the tile (one per output)
-    uint64_t *full = reinterpret_cast<uint64_t *>(nbs + kNbBytes);
+    uint64_t *full = reinterpret_cast<uint64_t *>(nbs + kAuxBytes);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const float ninf = -CUDART_INF_F;
     if (tid == 0) {
@@ -296,31 +301,47 @@ pool3_fwd_kernel(const float *__restrict__ y, P3Args a, float *__restrict__ out,
                 arg[(olo8 >> 3) + w] = (lo4 | (hi4 << 16)) & keep;
             }
         } else {
-            // stride 1 (G * HoWo % 8 == 0: every word whole in the tile): one thread per output column
-            const int items = t.np * a.Wo;
+            // stride 1 (G * HoWo % 8 == 0: every word whole in the tile): one thread per (plane,
+            // output column, row segment) walks down the segment, one new input row per output.
+            // Border taps (padding) are masked with selects on clamped addresses, not branches.
+            float *otile = out + olo;
+            const int items = t.np * a.segs * a.Wo;
             for (int it = tid; it < items; it += kRT) {
-                uint32_t pl, ow;
-                a.div_wo.divmod((uint32_t)it, pl, ow);
+                uint32_t ps, ow, pl, sg;
+                a.div_wo.divmod((uint32_t)it, ps, ow);
+                a.div_seg.divmod(ps, pl, sg);
+                const int oh0 = (int)sg * a.segr, oh1 = min(a.Ho, oh0 + a.segr);
                 const float *pb = R + ((t.p0 + pl) * a.HW - sb);
                 const int iw0 = (int)ow - a.P;
-                float hv[3];
-                int hx[3];
-                hscan<RELU>(pb - a.P * a.W, -a.P, iw0, a, hv[0], hx[0]);
-                hscan<RELU>(pb + (1 - a.P) * a.W, 1 - a.P, iw0, a, hv[1], hx[1]);
-                const int dx0 = max(0, -iw0);
-                float *op = out + olo + (int64_t)pl * a.HoWo + ow;
-                uint8_t *nb = nbs + pl * a.HoWo + ow;
-                for (int oh = 0; oh < a.Ho; ++oh) {
-                    const int ih2 = oh - a.P + 2;
-                    hscan<RELU>(pb + ih2 * a.W, ih2, iw0, a, hv[2], hx[2]);
-                    float best = ninf;
-                    int bi = max(0, a.P - oh) * 3 + dx0;
-#pragma unroll
-                    for (int dy = 0; dy < 3; ++dy) take3(hv[dy], 3 * dy + hx[dy], best, bi);
-                    op[(int64_t)oh * a.Wo] = best;
-                    nb[oh * a.Wo] = (uint8_t)bi;
-                    hv[0] = hv[1], hx[0] = hx[1];
-                    hv[1] = hv[2], hx[1] = hx[2];
+                const bool okL = iw0 >= 0, okR = iw0 + 2 < a.W;
+                const int cM = iw0 + 1, cL = okL ? iw0 : cM, cR = okR ? iw0 + 2 : cM;
+                const int dx0 = okL ? 0 : 1;  // first in-bounds column of the window (P <= 1)
+                // row scan of input row ih: (max, column) in R3's order; an absent row: (-inf, dx0)
+                auto hrow = [&](int ih, float &v, int &x) {
+                    const float *rp = pb + min(max(ih, 0), a.H - 1) * a.W;
+                    const float l = act3<RELU>(rp[cL]), m = act3<RELU>(rp[cM]), r = act3<RELU>(rp[cR]);
+                    v = okL ? l : ninf;
+                    x = dx0;
+                    take3(m, 1, v, x);
+                    take3(okR ? r : ninf, 2, v, x);
+                    if ((unsigned)ih >= (unsigned)a.H) v = ninf, x = dx0;
+                };
+                float hv0, hv1, hv2;
+                int hx0, hx1, hx2;
+                hrow(oh0 - a.P, hv0, hx0);
+                hrow(oh0 - a.P + 1, hv1, hx1);
+                int oo = (int)pl * a.HoWo + oh0 * a.Wo + (int)ow;  // tile-local output index
+                for (int oh = oh0; oh < oh1; ++oh) {
+                    hrow(oh - a.P + 2, hv2, hx2);
+                    float best = hv0;  // the window's first row (an absent first row: -inf, bi = 3 + dx0)
+                    int bi = hx0 + (oh - a.P >= 0 ? 0 : 3);
+                    take3(hv1, 3 + hx1, best, bi);
+                    take3(hv2, 6 + hx2, best, bi);
+                    otile[oo] = best;
+                    nbs[oo] = (uint8_t)bi;
+                    oo += a.Wo;
+                    hv0 = hv1, hx0 = hx1;
+                    hv1 = hv2, hx1 = hx2;
                 }
             }
             __syncthreads();
@@ -372,7 +393,7 @@ pool3_bwd_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ ar
     extern __shared__ __align__(128) unsigned char smp[];
     float *ring = reinterpret_cast<float *>(smp);
     uint8_t *nbb = smp + (size_t)a.rs * a.sf * 4;  // padded nibble-byte planes of the tile
-    uint64_t *full = reinterpret_cast<uint64_t *>(nbb + kNbBytes);
+    uint64_t *full = reinterpret_cast<uint64_t *>(nbb + kAuxBytes);
     const int tid = threadIdx.x;
     if (tid == 0) {
         for (int s = 0; s < a.rs; ++s) mbar_init(&full[s], 1);
@@ -559,6 +580,158 @@ pool3_bwd_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ ar
     }
 }
 
+// Backward through hit masks.  Pass 1 (one thread per argmax word): every window ORs one bit into
+// the hit mask of the input its argmax selects -- bit 3 (2 - dy) + (2 - dx) for stride 1 (9 bits,
+// 16 per input), bit 2 r + c for stride 2 (4 bits per input; r = 0 for the upper of two covering
+// window rows, c likewise) -- so that a mask's bits in ascending order are its windows in ascending
+// output order.  Pass 2 (one thread per input element): +0.0f, then dY of each set bit in that
+// order (R6), selected by the a1 mask bit (R7).  OR is order-free, so the result does not depend
+// on the atomics' order; the work is one atomic per window and one step per hit instead of 9 (4)
+// nibble tests per input.
+template <int S, bool MASK, bool SAME>
+__global__ void __launch_bounds__(kRT)
+pool3_bwd_hits_kernel(const float *__restrict__ dout, const uint32_t *__restrict__ arg,
+                      const uint32_t *__restrict__ mask, P3Args a, float *__restrict__ dx) {
+    pdl_enter();
+    extern __shared__ __align__(128) unsigned char smp[];
+    float *ring = reinterpret_cast<float *>(smp);
+    uint32_t *hits = reinterpret_cast<uint32_t *>(smp + (size_t)a.rs * a.sf * 4);
+    uint64_t *full = reinterpret_cast<uint64_t *>(smp + (size_t)a.rs * a.sf * 4 + kAuxBytes);
+    constexpr int kHB = S == 1 ? 16 : 4;  // hit bits per input
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        for (int s = 0; s < a.rs; ++s) mbar_init(&full[s], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const int64_t mine = a.tiles > blockIdx.x ? (a.tiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+    auto issue = [&](int64_t j, int st) {
+        const BwdTile t = bwd_tile(a, blockIdx.x + j * gridDim.x);
+        float *R = ring + (size_t)st * a.sf;
+        const uint32_t bd = ring_bytes(t.olo, t.ohi), ba = ring_bytes(t.aw_lo, t.aw_hi);
+        const uint32_t bm = MASK ? ring_bytes(t.mw_lo, t.mw_hi) : 0u;
+        mbar_arrive_expect_tx(&full[st], bd + ba + bm);
+        if (bd) ring_copy(R, dout + (t.olo & ~3ll), bd, &full[st]);
+        if (ba) ring_copy(R + a.a_off, arg + (t.aw_lo & ~3ll), ba, &full[st]);
+        if (bm) ring_copy(R + a.m_off, mask + (t.mw_lo & ~3ll), bm, &full[st]);
+    };
+    if (tid == 0)
+        for (int64_t j = 0; j < a.rs && j < mine; ++j) issue(j, (int)j);
+    int st = 0;
+    uint32_t ph = 0;
+    for (int64_t j = 0; j < mine; ++j) {
+        float *R = ring + (size_t)st * a.sf;
+        const BwdTile t = bwd_tile(a, blockIdx.x + j * gridDim.x);
+        const int cnt = t.np * a.HW;
+        {  // clear the tile's hit masks (the previous tile's gather has finished: end-of-tile barrier)
+            uint4 *h4 = reinterpret_cast<uint4 *>(hits);
+            const int n16 = (cnt * kHB / 8 + 15) >> 4;
+            for (int i = tid; i < n16; i += kRT) h4[i] = make_uint4(0u, 0u, 0u, 0u);
+        }
+        mbar_wait(&full[st], ph);
+        {
+            uint32_t *RA = reinterpret_cast<uint32_t *>(R + a.a_off), *RM = reinterpret_cast<uint32_t *>(R + a.m_off);
+            bool wrote = tail_fill(R, dout, t.olo, t.ohi, 0);
+            wrote |= tail_fill(RA, arg, t.aw_lo, t.aw_hi, 4);
+            if (MASK) wrote |= tail_fill(RM, mask, t.mw_lo, t.mw_hi, 8);
+            if (wrote) fence_proxy_async_smem();
+        }
+        __syncthreads();
+        const float *D = R + (t.olo - (t.olo & ~3ll));  // dY by tile-local output index
+        const uint32_t *Aw = reinterpret_cast<const uint32_t *>(R + a.a_off) + (t.aw_lo - (t.aw_lo & ~3ll));
+        const uint32_t *Mw = reinterpret_cast<const uint32_t *>(R + a.m_off) + (t.mw_lo - (t.mw_lo & ~3ll));
+        const int aph = (int)(t.olo & 7), mph = (int)(t.ilo & 31);
+        {  // pass 1: scatter one hit bit per window
+            const int no = t.np * a.HoWo;
+            const int nw = (aph + no + 7) >> 3;
+            for (int w = tid; w < nw; w += kRT) {
+                const uint32_t word = Aw[w];
+                const int l0 = 8 * w - aph;  // tile-local output of nibble 0
+                if (SAME) {  // 3x3/s1/p1 with Ho = H, Wo = W: window l is centred on input l
+#pragma unroll
+                    for (int k = 0; k < 8; ++k) {
+                        const int l = l0 + k;
+                        const int jn = (int)((word >> (4 * k)) & 0xfu);
+                        const int dy = (jn * 11) >> 5, dxx = jn - 3 * dy;
+                        const int tt = l + (dy - 1) * a.W + dxx - 1;
+                        if (l >= 0 && l < no && jn <= 8 && (unsigned)tt < (unsigned)cnt)
+                            atomicOr(&hits[tt >> 1], (1u << (8 - jn)) << (16 * (tt & 1)));
+                    }
+                    continue;
+                }
+                uint32_t pl, rem, oh, ow;
+                a.div_howo.divmod((uint32_t)(l0 > 0 ? l0 : 0), pl, rem);
+                a.div_wo.divmod(rem, oh, ow);
+                int base = (int)pl * a.HW + ((int)oh * S - a.P) * a.W + (int)ow * S - a.P;  // window's (0, 0) tap
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    const int l = l0 + k;
+                    if (l >= 0 && l < no) {
+                        const int jn = (int)((word >> (4 * k)) & 0xfu);
+                        const int dy = (jn * 11) >> 5, dxx = jn - 3 * dy;  // jn / 3, jn % 3 (jn <= 8)
+                        const int tt = base + dy * a.W + dxx;               // the selected input
+                        if (jn <= 8 && (unsigned)tt < (unsigned)cnt) {      // (a malformed map cannot write outside)
+                            if (S == 1) {
+                                atomicOr(&hits[tt >> 1], (1u << (8 - jn)) << (16 * (tt & 1)));
+                            } else {
+                                const int bit = (dy == 2 ? 0 : 2) + (dxx == 2 ? 0 : 1);
+                                atomicOr(&hits[tt >> 3], 1u << (4 * (tt & 7) + bit));
+                            }
+                        }
+                        base += S;
+                        if (++ow == (uint32_t)a.Wo) {
+                            ow = 0;
+                            base += S * a.W - a.Wo * S;
+                            if (++oh == (uint32_t)a.Ho) {
+                                oh = 0;
+                                base += a.HW - a.Ho * S * a.W;
+                            }
+                        }
+                    }
+                }
+            }
+        }
+        __syncthreads();
+        {  // pass 2: gather per input element
+            float *dxt = dx + t.ilo;
+            for (int l = tid; l < cnt; l += kRT) {
+                uint32_t h = (hits[l * kHB / 32] >> ((l * kHB) & 31)) & ((1u << kHB) - 1u);
+                const bool on = !MASK || ((Mw[(l + mph) >> 5] >> ((l + mph) & 31)) & 1u);
+                float acc = 0.0f;  // R6: +0.0f, then ascending output order
+                if (SAME && on && h) {  // window l - W - 1 is (th - 2, tw - 2)
+                    const float *Dp = D + l - a.W - 1;
+#pragma unroll
+                    for (int k = 0; k < 9; ++k)
+                        if (h & (1u << k)) acc = acc + Dp[(k / 3) * a.W + k % 3];
+                } else if (on && h) {
+                    uint32_t pl, rem, ih, iw;
+                    a.div_hw.divmod((uint32_t)l, pl, rem);
+                    a.div_w.divmod(rem, ih, iw);
+                    const int th = (int)ih + a.P, tw = (int)iw + a.P;
+                    // a fixed, predicated walk over the bits (a loop over set bits diverges: the
+                    // warp would run as many steps as its most-hit lane)
+                    if (S == 1) {
+                        const float *Dp = D + (int)pl * a.HoWo + (th - 2) * a.Wo + (tw - 2);  // window (th-2, tw-2)
+#pragma unroll
+                        for (int k = 0; k < 9; ++k)
+                            if (h & (1u << k)) acc = acc + Dp[(k / 3) * a.Wo + k % 3];
+                    } else {
+                        const float *Dp = D + (int)pl * a.HoWo + ((th >> 1) - 1) * a.Wo + ((tw >> 1) - 1);
+                        if (h & 1u) acc = acc + Dp[0];
+                        if (h & 2u) acc = acc + Dp[1];
+                        if (h & 4u) acc = acc + Dp[a.Wo];
+                        if (h & 8u) acc = acc + Dp[a.Wo + 1];
+                    }
+                }
+                dxt[l] = acc;
+            }
+        }
+        __syncthreads();  // stage st and the hit masks consumed
+        if (tid == 0 && j + a.rs < mine) issue(j + a.rs, st);
+        if (++st == a.rs) st = 0, ph ^= 1u;
+    }
+}
+
 int gcd_i(int a, int b) {
     while (b) {
         const int t = a % b;
@@ -624,7 +797,7 @@ Ring ring_for(bool fwd, int S) {
     return cfg[fwd ? 1 : 0][S - 1];
 }
 size_t ring_smem(const Ring &r) {
-    return (size_t)r.rs * r.kb * 1024 + kNbBytes + 8 * kMaxRS + kMaxRS * sizeof(FwdTile);
+    return (size_t)r.rs * r.kb * 1024 + kAuxBytes + 8 * kMaxRS + kMaxRS * sizeof(FwdTile);
 }
 int64_t resident_ctas(size_t smem) {
     return std::max<int64_t>(1, std::min<int64_t>(2, (int64_t)(227 * 1024) / (int64_t)(smem + 1024))) * num_sms();
@@ -670,6 +843,11 @@ cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, in
         a.G = choose_g(a.NC, a.HW, 64, unit, ctas, a.sf);
         while (a.G > unit && (int64_t)a.G * a.HoWo > kNbBytes) a.G -= unit;
         if (a.G == 0 || (int64_t)a.G * a.HoWo > kNbBytes) return cudaErrorNotSupported;
+        const int64_t cols = (int64_t)a.G * Wo;  // row segments: about one item per thread
+        const int32_t want = (int32_t)std::max<int64_t>(1, std::min<int64_t>(Ho, kRT / cols));
+        a.segr = (Ho + want - 1) / want;
+        a.segs = (Ho + a.segr - 1) / a.segr;
+        a.div_seg = FastDiv::make((uint32_t)a.segs);
     } else {
         // rows of the next plane a tile may need: the windows of its last argmax word's (<= 7)
         // outputs there, and the (<= 31) elements of its last mask word
@@ -732,6 +910,7 @@ cudaError_t launch_pool3_bwd(const float *dout, const uint32_t *argmax, const ui
     a.sf = ring.kb * 256;
     const size_t smem = ring_smem(ring);
     const int64_t ctas = resident_ctas(smem);
+    const bool hitk = GIST_POOL3_BWD_HITS != 0;
     if (a.S == 2) {
         a.hb = (H + a.P + 1) / 2;
         a.wb = (W + a.P + 1) / 2;
@@ -747,13 +926,38 @@ cudaError_t launch_pool3_bwd(const float *dout, const uint32_t *argmax, const ui
     // phases / round-ups of the three ranges
     const int64_t per_plane = (int64_t)a.HoWo + (a.HoWo + 7) / 8 + (mask ? (a.HW + 31) / 32 : 0) + 1;
     a.G = choose_g(a.NC, per_plane, 64, 1, ctas, a.sf);
-    while (a.G > 1 && (int64_t)a.G * a.PR * a.PC > kNbBytes) --a.G;
-    if (a.G == 0 || (int64_t)a.G * a.PR * a.PC > kNbBytes) return cudaErrorNotSupported;
+    // the tile's hit masks (hits kernel) or padded nibble planes must fit the area after the ring
+    const int64_t aux_plane = hitk ? (int64_t)a.HW * (a.S == 1 ? 2 : 1) / 1 : (int64_t)a.PR * a.PC;
+    const int64_t aux_cap = hitk ? (a.S == 1 ? kHitBytes : 2 * (int64_t)kHitBytes) : kNbBytes;  // S = 2: half bytes
+    while (a.G > 1 && (int64_t)a.G * aux_plane + 32 > aux_cap) --a.G;
+    if (a.G == 0 || (int64_t)a.G * aux_plane + 32 > aux_cap) return cudaErrorNotSupported;
     a.tiles = ceil_div(a.NC, a.G);
     const int64_t G = a.G;
     a.a_off = (int32_t)((G * a.HoWo + 8 + 3) & ~3ll);
     a.m_off = (int32_t)((a.a_off + (G * a.HoWo + 7) / 8 + 8 + 3) & ~3ll);
     const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(a.tiles, ctas));
+    if (hitk) {
+#define P3H(S_, M_, SM_)                                                                                     \
+    do {                                                                                                     \
+        static PerDeviceAttr attr;                                                                           \
+        const cudaError_t e =                                                                                \
+            attr.ensure(reinterpret_cast<const void *>(pool3_bwd_hits_kernel<S_, M_, SM_>), (int)smem);     \
+        if (e != cudaSuccess) return e;                                                                      \
+        launch_k(pool3_bwd_hits_kernel<S_, M_, SM_>, grid, kRT, smem, s, dout, argmax, mask, a, dx);         \
+    } while (0)
+        const bool same = a.S == 1 && a.P == 1 && Ho == H && Wo == W;
+        if (a.S == 1) {
+            if (same) {
+                if (mask) P3H(1, true, true); else P3H(1, false, true);
+            } else {
+                if (mask) P3H(1, true, false); else P3H(1, false, false);
+            }
+        } else {
+            if (mask) P3H(2, true, false); else P3H(2, false, false);
+        }
+#undef P3H
+        return cudaPeekAtLastError();
+    }
 #define P3B(S_, M_)                                                                                          \
     do {                                                                                                     \
         static PerDeviceAttr attr;                                                                           \
