@@ -68,17 +68,18 @@ maxpool_fwd_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ 
     pdl_enter();
     const int kh = KH ? KH : a.kh, kw = KW ? KW : a.kw;
     const int lane = threadIdx.x & 31;
-    const int64_t chunks = ((int64_t)a.n_out + 31) / 32;
-    const int64_t nwarps = ((int64_t)gridDim.x * kPoolThreads) >> 5;
-    for (int64_t c = ((int64_t)blockIdx.x * kPoolThreads + threadIdx.x) >> 5; c < chunks; c += nwarps) {
-        const int64_t o = c * 32 + lane;
+    // 32-bit output indices (the API rejects maps of 2^31 elements or more)
+    const uint32_t chunks = ((uint32_t)a.n_out + 31) / 32;
+    const uint32_t nwarps = (gridDim.x * kPoolThreads) >> 5;
+    for (uint32_t c = (blockIdx.x * kPoolThreads + threadIdx.x) >> 5; c < chunks; c += nwarps) {
+        const uint32_t o = c * 32 + lane;
         uint32_t nib = 0;
-        if (o < a.n_out) {
+        if (o < (uint32_t)a.n_out) {
             uint32_t q, ow, nc, oh;
-            a.div_wo.divmod((uint32_t)o, q, ow);
+            a.div_wo.divmod(o, q, ow);
             a.div_ho.divmod(q, nc, oh);
             const int h0 = (int)oh * a.sh - a.ph, w0 = (int)ow * a.sw - a.pw;
-            const float *plane = y + (int64_t)nc * a.H * a.W;
+            const float *plane = y + nc * (uint32_t)(a.H * a.W);
             float best = -CUDART_INF_F;
             int bi = -1;
             if (KH && KW) {
@@ -128,7 +129,7 @@ maxpool_fwd_kernel(const float *__restrict__ y, PoolArgs a, float *__restrict__ 
         nib |= __shfl_xor_sync(kFull, nib, 1);
         nib |= __shfl_xor_sync(kFull, nib, 2);
         nib |= __shfl_xor_sync(kFull, nib, 4);
-        if ((lane & 7) == 0 && o < a.n_out) arg[o >> 3] = nib;
+        if ((lane & 7) == 0 && o < (uint32_t)a.n_out) arg[o >> 3] = nib;
     }
 }
 
@@ -627,26 +628,33 @@ pool_bwd_k3s2_block_kernel(const float *__restrict__ dout, const uint32_t *__res
                            const uint32_t *__restrict__ mask, PoolArgs a, FastDiv div_wb, FastDiv div_hb,
                            int64_t nblk, float *__restrict__ dx) {
     pdl_enter();
-    const int64_t HW = (int64_t)a.H * a.W, HoWo = (int64_t)a.Ho * a.Wo;
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < nblk; t += stride) {
+    // 32-bit element indices (the API rejects maps of 2^31 elements or more): one 64-bit address per
+    // row of loads or stores, the rest immediate offsets
+    const uint32_t HW = (uint32_t)a.H * (uint32_t)a.W, HoWo = (uint32_t)a.Ho * (uint32_t)a.Wo;
+    const uint32_t stride = gridDim.x * blockDim.x, nb = (uint32_t)nblk;
+    for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < nb; t += stride) {
         uint32_t q, b, plane, A;
-        div_wb.divmod((uint32_t)t, q, b);
+        div_wb.divmod(t, q, b);
         div_hb.divmod(q, plane, A);
-        const bool up = A >= 1, left = b >= 1;             // windows (A-1, .) / (., b-1) exist
+        const bool up = A >= 1, left = b >= 1;                      // windows (A-1, .) / (., b-1) exist
         const bool here_r = (int)A < a.Ho, here_c = (int)b < a.Wo;  // windows (A, .) / (., b) exist
-        const int64_t o11 = (int64_t)plane * HoWo + (int64_t)A * a.Wo + b;  // window (A, b)
+        // signed offsets: o00 (and o11 - 1) are negative at the map's first windows, where the
+        // loads they address are not made
+        const int o11 = (int)(plane * HoWo + A * (uint32_t)a.Wo + b);  // window (A, b)
+        const int o00 = o11 - a.Wo - 1;                                 // window (A-1, b-1)
+        const float *g0 = dout + o00, *g1 = dout + (o11 - 1);          // rows A-1 and A of dY
         float g[4] = {0.f, 0.f, 0.f, 0.f};
-        uint32_t nb[4] = {15u, 15u, 15u, 15u};  // 15: no window / no hit
+        uint32_t nbv[4] = {15u, 15u, 15u, 15u};  // 15: no window / no hit
         const bool ok[4] = {up && left, up && here_c, here_r && left, here_r && here_c};
-        const int64_t os[4] = {o11 - a.Wo - 1, o11 - a.Wo, o11 - 1, o11};
+        const int os[4] = {o00, o00 + 1, o11 - 1, o11};
+        if (ok[0]) g[0] = ld_ro(g0);
+        if (ok[1]) g[1] = ld_ro(g0 + 1);
+        if (ok[2]) g[2] = ld_ro(g1);
+        if (ok[3]) g[3] = ld_ro(g1 + 1);
 #pragma unroll
         for (int k = 0; k < 4; ++k)
-            if (ok[k]) {
-                g[k] = ld_ro(dout + os[k]);
-                nb[k] = (ld_ro(arg + (os[k] >> 3)) >> (4 * (os[k] & 7))) & 0xfu;
-            }
-        const int64_t i00 = (int64_t)plane * HW + (int64_t)(2 * A) * a.W + 2 * (int)b;
+            if (ok[k]) nbv[k] = (ld_ro(arg + (os[k] >> 3)) >> (4 * (os[k] & 7))) & 0xfu;
+        const uint32_t i00 = plane * HW + (2 * A) * (uint32_t)a.W + 2 * b;
         const bool r1 = 2 * (int)A + 1 < a.H, c1 = 2 * (int)b + 1 < a.W;
         uint32_t m0 = 3u, m1 = 3u;
         if (mask) {
@@ -655,26 +663,27 @@ pool_bwd_k3s2_block_kernel(const float *__restrict__ dout, const uint32_t *__res
             const uint32_t w0 = ld_ro(mask + (i00 >> 5)), w0b = c1 ? ld_ro(mask + ((i00 + 1) >> 5)) : 0u;
             m0 = ((w0 >> (i00 & 31)) & 1u) | (((w0b >> ((i00 + 1) & 31)) & 1u) << 1);
             if (r1) {
-                const int64_t i10 = i00 + a.W;
+                const uint32_t i10 = i00 + (uint32_t)a.W;
                 const uint32_t w1 = ld_ro(mask + (i10 >> 5)), w1b = c1 ? ld_ro(mask + ((i10 + 1) >> 5)) : 0u;
                 m1 = ((w1 >> (i10 & 31)) & 1u) | (((w1b >> ((i10 + 1) & 31)) & 1u) << 1);
             }
         }
         float a00 = 0.0f, a01 = 0.0f, a10 = 0.0f, a11 = 0.0f;  // +0.0f, then ascending o
-        if (nb[0] == 8u) a00 = a00 + g[0];
-        if (nb[1] == 6u) a00 = a00 + g[1];
-        if (nb[1] == 7u) a01 = a01 + g[1];
-        if (nb[2] == 2u) a00 = a00 + g[2];
-        if (nb[2] == 5u) a10 = a10 + g[2];
-        if (nb[3] == 0u) a00 = a00 + g[3];
-        if (nb[3] == 1u) a01 = a01 + g[3];
-        if (nb[3] == 3u) a10 = a10 + g[3];
-        if (nb[3] == 4u) a11 = a11 + g[3];
-        dx[i00] = (m0 & 1u) ? a00 : 0.0f;
-        if (c1) dx[i00 + 1] = (m0 & 2u) ? a01 : 0.0f;
+        if (nbv[0] == 8u) a00 = a00 + g[0];
+        if (nbv[1] == 6u) a00 = a00 + g[1];
+        if (nbv[1] == 7u) a01 = a01 + g[1];
+        if (nbv[2] == 2u) a00 = a00 + g[2];
+        if (nbv[2] == 5u) a10 = a10 + g[2];
+        if (nbv[3] == 0u) a00 = a00 + g[3];
+        if (nbv[3] == 1u) a01 = a01 + g[3];
+        if (nbv[3] == 3u) a10 = a10 + g[3];
+        if (nbv[3] == 4u) a11 = a11 + g[3];
+        float *d0 = dx + i00, *d1 = d0 + a.W;
+        d0[0] = (m0 & 1u) ? a00 : 0.0f;
+        if (c1) d0[1] = (m0 & 2u) ? a01 : 0.0f;
         if (r1) {
-            dx[i00 + a.W] = (m1 & 1u) ? a10 : 0.0f;
-            if (c1) dx[i00 + a.W + 1] = (m1 & 2u) ? a11 : 0.0f;
+            d1[0] = (m1 & 1u) ? a10 : 0.0f;
+            if (c1) d1[1] = (m1 & 2u) ? a11 : 0.0f;
         }
     }
 }
