@@ -1,7 +1,11 @@
 """compute-sanitizer as a test target: memcheck and synccheck over every kernel on
 small ragged shapes (scripts/sanitize.py), including the odd-W / n % 32 == 0 pool shapes where
 a mask read one word past the buffer was possible.  racecheck is run by scripts/gpu_sanitize.sh;
-its only reports are the SSDC encoder's mbarrier-ordered role hand-offs."""
+its only reports are the SSDC encoder's mbarrier-ordered role hand-offs.
+
+Opt-in (GIST_SANITIZE=1): the GPU pool has closed compute-sanitizer (its wrapper exits 86) because
+runs under it left GPUs needing a reset, so the default -m gpu run does not start it.  The logs
+under profiles/r2_sanitize_*.log are from the runs made before it was closed."""
 import os
 import shutil
 import subprocess
@@ -16,11 +20,15 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 @pytest.mark.parametrize("tool", ["memcheck", "synccheck"])
 def test_compute_sanitizer_clean(gist, cuda, tool):
     cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+    if os.environ.get("GIST_SANITIZE") != "1":
+        pytest.skip("compute-sanitizer runs are opt-in (GIST_SANITIZE=1)")
     if not os.path.exists(cs):
         pytest.skip("compute-sanitizer not installed")
     r = subprocess.run([cs, "--tool", tool, "--error-exitcode", "9", sys.executable,
                         os.path.join(ROOT, "scripts", "sanitize.py")],
                        capture_output=True, text=True, timeout=900, cwd=ROOT)
     tail = (r.stdout + r.stderr)[-3000:]
+    if r.returncode == 86 and "closed" in tail:
+        pytest.skip("compute-sanitizer is closed on this GPU pool")
     assert r.returncode == 0, tail
     assert "ERROR SUMMARY: 0 errors" in r.stdout + r.stderr, tail
