@@ -18,9 +18,9 @@
 //   * publisher warp: tile-local row scan -> rinc[], tile total published (epoch tag | count
 //     in one word) to tot[tile];
 //   * gatherer warp: running prefix over tot[] -> the tile's global offset, and row_end;
-//   * 16 writer warps (2 rows each): once the tile is published, load their rows from the ring
+//   * 8 writer warps (4 rows each): once the tile is published, load their rows from the ring
 //     into registers (one tile ahead) and release the stage; rank nonzeros (lane l owns columns
-//     [8l, 8l+8); lane prefix: one shuffle scan of both rows' lane counts), stage them in
+//     l + 32k; one ballot per 32 columns, row starts from the publisher's row scan), stage them in
 //     shared memory congruent to the output mod 16, and store the whole 16-entry groups of
 //     val/col with two 1-D bulk copies (shared -> global) once the offset is resolved.
 // HBM sees the algorithmic traffic: 4n read once, 5*nnz + 4*rows written.
@@ -56,12 +56,20 @@ constexpr int kRow = 256;
 #define GIST_SSDC_DEC_CTAS 3  // decode CTAs per SM (grid cap); 4-6 measured slower in isolation
 #endif
 #ifndef GIST_SSDC_LPRE
-#define GIST_SSDC_LPRE 0  // 1: the counters also scan the writers' lane counts (writers skip count + scan): 0.228 -> 0.265 ms, the counters then pace the prefix chain
+#define GIST_SSDC_LPRE 0  // 1 (with GIST_SSDC_BALLOT=0): the counters also scan the writers' lane counts (writers skip count + scan): 0.228 -> 0.265 ms, the counters then pace the prefix chain
+#endif
+#ifndef GIST_SSDC_BALLOT
+// 1: writer lane l holds columns l + 32k of its rows and one ballot per 32 columns ranks the nonzeros
+// (row starts from rinc: no lane counts, no shuffle scan).  With 4 rows per writer (8 writer warps),
+// relu1_1 b64 s = .5 / .8 / .9: 0.246 / 0.228 / 0.228 -> 0.226 / 0.224 / 0.222 ms, C3 step a4 70% -> 73%.
+// 0: lane l holds columns [8l, 8l+8) and a shuffle scan of the lane counts ranks them (2 rows per writer).
+#define GIST_SSDC_BALLOT 1
 #endif
 #ifndef GIST_SSDC_WROWS
-#define GIST_SSDC_WROWS 2
+#define GIST_SSDC_WROWS (GIST_SSDC_BALLOT ? 4 : 2)
 #endif
 constexpr int kWRows = GIST_SSDC_WROWS;        // rows per writer warp per tile
+static_assert(!(GIST_SSDC_LPRE && GIST_SSDC_BALLOT), "lane prefixes are for the scan path");
 constexpr int kTileRows = 32;                         // rows per tile = 8192 elements = 32 KB
 static_assert(kTileRows == 32, "the gatherer writes row_end with one lane per row");
 constexpr int kWriters = kTileRows / kWRows;
@@ -76,7 +84,7 @@ constexpr int kPartElems = kPartRows * kRow;           // 8 KB per TMA stage (4 
 constexpr int kStages = GIST_SSDC_STAGES;
 constexpr int kQ = GIST_SSDC_Q;
 constexpr int kProd = 0, kCount = 1, kPub = kCount + kParts, kGather = kPub + 1, kWriter0 = kGather + 1;
-constexpr int kEncThreads = 32 * (kWriter0 + kWriters);  // 23 warps = 736 threads
+constexpr int kEncThreads = 32 * (kWriter0 + kWriters);  // 15 warps = 480 threads (8 writers)
 constexpr int kStage = kTileRows * kRow + 16;  // staged entries per tile (+ 16-entry phase)
 constexpr int kWriterThreads = 32 * kWriters;
 constexpr int kGatherPer = 8;                     // totals per lane per gather round (256 per warp)
@@ -170,6 +178,30 @@ __device__ __forceinline__ void stage_rows(EncSmem &S, int q, int sb, int w, int
     const uint32_t w_excl = rw ? S.rinc[q][rw - 1] : 0u;
     if (S.rinc[q][rw + kWRows - 1] == w_excl) return;  // no nonzeros in these rows
     const uint32_t p = (uint32_t)(S.base[q] & 15) + w_excl;  // staging index of the writer's first entry
+#if GIST_SSDC_BALLOT
+    // lane l holds columns l + 32k of each row (k = 0..7: lo.x..w, hi.x..w).  Row r's entries start
+    // at rinc[rw + r - 1] (tile-local), so no lane counts or scans: one ballot per 32 columns gives
+    // each nonzero its rank, and the entries of columns [32k, 32k + 32) follow those of lower k
+    // (ascending column order, O4).
+    const uint32_t lt = (1u << lane) - 1u;
+    uint32_t *vs = S.vst[sb];
+    uint8_t *cs = S.cst[sb];
+#pragma unroll
+    for (int r = 0; r < kWRows; ++r) {
+        const uint32_t v[8] = {lo[r].x, lo[r].y, lo[r].z, lo[r].w, hi[r].x, hi[r].y, hi[r].z, hi[r].w};
+        uint32_t base = p + ((r ? S.rinc[q][rw + r - 1] : w_excl) - w_excl);
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const uint32_t b = __ballot_sync(kFull, v[k] != 0u);  // R8: nonzero bit patterns
+            if (v[k] != 0u) {
+                const uint32_t i = base + __popc(b & lt);
+                vs[i] = v[k];
+                cs[i] = (uint8_t)(32 * k + lane);
+            }
+            base += __popc(b);
+        }
+    }
+#else
     static_assert(kWRows == 2, "the packed scan carries two rows");
 #if GIST_SSDC_LPRE
     // the counters scanned this writer's lane counts (published with the tile, ordered by published[q])
@@ -207,6 +239,7 @@ __device__ __forceinline__ void stage_rows(EncSmem &S, int q, int sb, int w, int
                 : "memory");
         }
     }
+#endif  // GIST_SSDC_BALLOT
 }
 
 // Writer warp 0, once every writer has staged the tile: the whole 16-entry groups leave as two
@@ -319,7 +352,7 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
 #endif
             int64_t t = first_ticket;
             int jc = 0;  // job cursor: tickets rise, so jobs only move forward
-            for (int64_t j = 0;; ++j) {
+            for (uint32_t j = 0;; ++j) {
                 const int q = (int)(j % kQ);
                 if (j >= kQ) mbar_wait_sleep(&S.freed[q], (uint32_t)(j / kQ - 1) & 1u);
                 if (t < tiles)
@@ -330,7 +363,7 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
                 const EncJob &jb = J.j[jc];
                 const int64_t e_tile = (t - jb.tile0) * (int64_t)(kTileRows * kRow);
                 for (int h = 0; h < kParts; ++h) {
-                    const int64_t js = kParts * j + h;
+                    const uint32_t js = kParts * j + h;
                     const int s = (int)(js % kStages);
                     if (js >= kStages) mbar_wait_sleep(&S.empty[s], (uint32_t)(js / kStages - 1) & 1u);
                     const int64_t e0 = e_tile + h * kPartElems;
@@ -349,8 +382,8 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
     } else if (warp >= kCount && warp < kCount + kParts) {
         // ---- counters: part h of every tile; lane r ends up with row r's count
         const int h = warp - kCount;
-        for (int64_t j = 0;; ++j) {
-            const int64_t js = kParts * j + h;
+        for (uint32_t j = 0;; ++j) {
+            const uint32_t js = kParts * j + h;
             const int s = (int)(js % kStages);
             const int q = (int)(j % kQ);
             mbar_wait_sleep(&S.full[s], (uint32_t)(js / kStages) & 1u);
@@ -412,7 +445,7 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
         }
     } else if (warp == kPub) {
         // ---- publisher: tile-local row scan, tile total -> tot[tile]
-        for (int64_t j = 0;; ++j) {
+        for (uint32_t j = 0;; ++j) {
             const int q = (int)(j % kQ);
             mbar_wait_sleep(&S.counted[q], (uint32_t)(j / kQ) & 1u);
             const int64_t t = S.tile[q];
@@ -441,7 +474,7 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
         // until all are published), base(t) = sum.
         int64_t pos = 0, sum = 0;
         int cur = -1;  // chain head of the running prefix
-        for (int64_t j = 0;; ++j) {
+        for (uint32_t j = 0;; ++j) {
             const int q = (int)(j % kQ);
             mbar_wait_sleep(&S.published[q], (uint32_t)(j / kQ) & 1u);
             const int64_t t = S.tile[q];
@@ -500,7 +533,7 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
         // the tile of local slot jj once published (its count is in rinc[]; its rows still in
         // the ring); lane l gets the 8 consecutive columns [8l, 8l+8) of each of its rows, so a
         // lane's nonzeros are contiguous in the output (elements past n were zero-filled)
-        auto fetch = [&](int64_t jj, uint4 (&l)[kWRows], uint4 (&h)[kWRows]) -> int64_t {
+        auto fetch = [&](uint32_t jj, uint4 (&l)[kWRows], uint4 (&h)[kWRows]) -> int64_t {
             const int q = (int)(jj % kQ);
             mbar_wait_sleep(&S.published[q], (uint32_t)(jj / kQ) & 1u);
             const int64_t t = S.tile[q];
@@ -508,14 +541,21 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
             // from shared memory, then release the stage (the part's kPartRows / kWRows writers)
             if (t < tiles) {
                 const int part = (w * kWRows) / kPartRows;
-                const int64_t js = kParts * jj + part;
+                const uint32_t js = kParts * jj + part;
                 const int st = (int)(js % kStages);
                 const float *rowp = S.raw[st] + (w * kWRows - part * kPartRows) * kRow;
 #pragma unroll
                 for (int r = 0; r < kWRows; ++r) {
+#if GIST_SSDC_BALLOT
+                    // columns lane + 32k (conflict-free 32-bit loads)
+                    const uint32_t *p1 = reinterpret_cast<const uint32_t *>(rowp + r * kRow) + lane;
+                    l[r] = make_uint4(p1[0], p1[32], p1[64], p1[96]);
+                    h[r] = make_uint4(p1[128], p1[160], p1[192], p1[224]);
+#else
                     const uint4 *p4 = reinterpret_cast<const uint4 *>(rowp + r * kRow);
                     l[r] = p4[2 * lane];
                     h[r] = p4[2 * lane + 1];
+#endif
                 }
                 __syncwarp();
                 if (lane == 0) mbar_arrive1(&S.empty[st]);
@@ -526,7 +566,7 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
         // it, the tile is fully staged (writer 0 then stores it), and writer 0's bulk copies of the
         // previous tile, which it waited on just before, have read buffer (jj - 1) & 1, so tile
         // jj + 1 may overwrite it.
-        auto retire = [&](int64_t jj, int64_t t, const uint4 (&l)[kWRows], const uint4 (&h)[kWRows]) {
+        auto retire = [&](uint32_t jj, int64_t t, const uint4 (&l)[kWRows], const uint4 (&h)[kWRows]) {
             const int q = (int)(jj % kQ);
             const int sb = (int)(jj & 1);
             mbar_wait_sleep(&S.resolved[q], (uint32_t)(jj / kQ) & 1u);
@@ -545,7 +585,7 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
         };
 #pragma unroll
         for (int d = 0; d < kDepth - 1; ++d) tt[d] = (d == 0 || tt[d - 1] < tiles) ? fetch(d, lo[d], hi[d]) : tiles;
-        for (int64_t j = 0;; j += kDepth) {
+        for (uint32_t j = 0;; j += kDepth) {
 #pragma unroll
             for (int d = 0; d < kDepth; ++d) {
                 // set d holds tile j+d; prefetch j+d+kDepth-1 into set (d + kDepth - 1) % kDepth
