@@ -65,6 +65,11 @@ constexpr int kRow = 256;
 // 0: lane l holds columns [8l, 8l+8) and a shuffle scan of the lane counts ranks them (2 rows per writer).
 #define GIST_SSDC_BALLOT 1
 #endif
+#ifndef GIST_SSDC_SPIN_NS
+// producer (ring space), counters (data) and publisher (counts) poll with test_wait + __nanosleep:
+// their try_wait loops took ~24% of the kernel's issue slots (ncu), which the writers need
+#define GIST_SSDC_SPIN_NS 256  // relu1_1 s = .8: 0.2257 (try_wait) vs 0.2298 / 0.2277 / 0.2257 / 0.2245 ms at 32 / 64 / 128 / 256 ns
+#endif
 #ifndef GIST_SSDC_WROWS
 #define GIST_SSDC_WROWS (GIST_SSDC_BALLOT ? 4 : 2)
 #endif
@@ -365,7 +370,7 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
                 for (int h = 0; h < kParts; ++h) {
                     const uint32_t js = kParts * j + h;
                     const int s = (int)(js % kStages);
-                    if (js >= kStages) mbar_wait_sleep(&S.empty[s], (uint32_t)(js / kStages - 1) & 1u);
+                    if (js >= kStages) mbar_wait_backoff(&S.empty[s], (uint32_t)(js / kStages - 1) & 1u, GIST_SSDC_SPIN_NS);
                     const int64_t e0 = e_tile + h * kPartElems;
                     const int64_t avail = t < tiles ? jb.n - e0 : 0;
                     const uint32_t bytes =
@@ -386,7 +391,7 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
             const uint32_t js = kParts * j + h;
             const int s = (int)(js % kStages);
             const int q = (int)(j % kQ);
-            mbar_wait_sleep(&S.full[s], (uint32_t)(js / kStages) & 1u);
+            mbar_wait_backoff(&S.full[s], (uint32_t)(js / kStages) & 1u, GIST_SSDC_SPIN_NS);
             const int64_t t = S.tile[q];
             if (t < tiles) {
                 float *T = S.raw[s];
@@ -447,7 +452,7 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
         // ---- publisher: tile-local row scan, tile total -> tot[tile]
         for (uint32_t j = 0;; ++j) {
             const int q = (int)(j % kQ);
-            mbar_wait_sleep(&S.counted[q], (uint32_t)(j / kQ) & 1u);
+            mbar_wait_backoff(&S.counted[q], (uint32_t)(j / kQ) & 1u, GIST_SSDC_SPIN_NS);
             const int64_t t = S.tile[q];
             if (t < tiles) {
                 uint32_t inc = S.rcnt[q][lane];
