@@ -51,7 +51,8 @@ constexpr int kRT = GIST_POOL3_THREADS;  // threads per CTA
 #define GIST_POOL3_BWD_STRIP 1  // stride-1 backward: column strips for tiles of >= kRT/2 columns (0: never)
 #endif
 constexpr int kMaxRS = 4;  // ring stages: a.rs <= kMaxRS stages of a.sf floats (host: ring_for)
-constexpr int kNbBytes = 12 * 1024;   // nibble bytes of one tile (forward, nibble-plane backward)
+constexpr int kNbBytes = 12 * 1024;   // nibble bytes of one tile (nibble-plane backward)
+constexpr int kNbFwd = 8 * 1024;      // forward: nibble bytes of one tile, two tiles' worth in the aux area
 constexpr int kHitBytes = 16 * 1024;  // hit masks of one tile (backward): 16 bits (S = 1) or 4 bits per input
 constexpr int kAuxBytes = kHitBytes;  // the per-CTA area after the ring (>= kNbBytes)
 
@@ -108,6 +109,7 @@ __device__ __forceinline__ bool tail_fill(T *dst, const T *__restrict__ src, int
 
 struct FwdTile {
     int64_t p0, lo, hi, oa, ob, ia, ib;
+    int64_t ce;  // end of the bulk-copied range (>= hi except at the map's ragged end)
     int np;
 };
 
@@ -123,6 +125,11 @@ __device__ __forceinline__ FwdTile fwd_tile(const P3Args &a, int64_t k) {
     t.lo = t.p0 * a.HW;
     const int64_t end = t.lo + (int64_t)t.np * a.HW;
     t.hi = last ? end : min(a.n_in, end + max((int64_t)a.xrows * a.W, t.ib - end));
+    // the copy ends on a 16-byte boundary past hi when the map has the elements (<= 3 more floats,
+    // within the stage's slack), so only the map's last tile needs threads to load a ragged tail
+    const int64_t up = (t.hi + 3) & ~3ll;
+    t.ce = up <= a.n_in ? up : (t.hi & ~3ll);
+    if (t.ce < (t.lo & ~3ll)) t.ce = t.lo & ~3ll;
     return t;
 }
 
@@ -146,8 +153,8 @@ pool3_fwd_kernel(const float *__restrict__ y, P3Args a, float *__restrict__ out,
     pdl_enter();
     extern __shared__ __align__(128) unsigned char smp[];
     float *ring = reinterpret_cast<float *>(smp);
-    uint8_t *nbs = smp + (size_t)a.rs * a.sf * 4;  // nibble bytes of the tile (one per output)
-    uint64_t *full = reinterpret_cast<uint64_t *>(nbs + kAuxBytes);
+    uint8_t *nbs0 = smp + (size_t)a.rs * a.sf * 4;  // nibble bytes of two tiles (one per output), kNbFwd each
+    uint64_t *full = reinterpret_cast<uint64_t *>(nbs0 + kAuxBytes);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const float ninf = -CUDART_INF_F;
     if (tid == 0) {
@@ -162,21 +169,47 @@ pool3_fwd_kernel(const float *__restrict__ y, P3Args a, float *__restrict__ out,
     auto issue = [&](int64_t j, int st) {
         const FwdTile t = fwd_tile(a, blockIdx.x + j * gridDim.x);
         desc[st] = t;
-        const uint32_t b = ring_bytes(t.lo, t.hi);
+        const uint32_t b = (uint32_t)((t.ce - (t.lo & ~3ll)) * 4);
         mbar_arrive_expect_tx(&full[st], b);
         if (b) ring_copy(ring + (size_t)st * a.sf, y + (t.lo & ~3ll), b, &full[st]);
+    };
+    // argmax words of a finished tile from its nibble bytes (8 per word, one aligned 64-bit load);
+    // only the map's last word can be partial (its pad nibbles are 0).  Run one tile later, between
+    // the next tile's walk and the barrier that ends it (the bytes are double-buffered).
+    auto pack = [&](const FwdTile &t, const uint8_t *nbs) {
+        const int64_t olo = t.p0 * a.HoWo;
+        const int64_t olo8 = S == 2 ? (olo & ~7ll) : olo;  // stride 1: tiles hold whole words
+        const int w0 = S == 2 ? (int)((t.oa - olo8) >> 3) : 0;
+        const int64_t oend = S == 2 ? t.ob : olo + (int64_t)t.np * a.HoWo;
+        const int w1 = (int)((oend - olo8 + 7) >> 3);
+        const int nvalid = (int)(oend - olo8);  // nibble bytes from olo8 on
+        for (int w = w0 + tid; w < w1; w += kRT) {
+            const uint2 b = *reinterpret_cast<const uint2 *>(nbs + 8 * w);
+            const uint32_t lo4 = (b.x & 0xfu) | ((b.x >> 4) & 0xf0u) | ((b.x >> 8) & 0xf00u) | ((b.x >> 12) & 0xf000u);
+            const uint32_t hi4 = (b.y & 0xfu) | ((b.y >> 4) & 0xf0u) | ((b.y >> 8) & 0xf00u) | ((b.y >> 12) & 0xf000u);
+            const int valid = nvalid - 8 * w;
+            const uint32_t keep = valid >= 8 ? ~0u : ((1u << (4 * valid)) - 1u);
+            arg[(olo8 >> 3) + w] = (lo4 | (hi4 << 16)) & keep;
+        }
     };
     if (tid == 0)
         for (int64_t j = 0; j < a.rs && j < mine; ++j) issue(j, (int)j);
     int st = 0;
     uint32_t ph = 0;
+    FwdTile prev{};
     for (int64_t j = 0; j < mine; ++j) {
         float *R = ring + (size_t)st * a.sf;
+        uint8_t *nbs = nbs0 + (j & 1) * kNbFwd;
         mbar_wait(&full[st], ph);
         const FwdTile t = desc[st];
         const int64_t sb = t.lo & ~3ll;  // stage index of element e: e - sb
-        if (tail_fill(R, y, t.lo, t.hi, 0)) fence_proxy_async_smem();
-        __syncthreads();
+        if (t.ce < t.hi) {  // the map's ragged end (tile-uniform): threads load the last <= 3 elements
+            if (tid < t.hi - t.ce) {
+                R[t.ce - sb + tid] = y[t.ce + tid];
+                fence_proxy_async_smem();  // generic writes into a TMA stage
+            }
+            __syncthreads();
+        }
         // a1 mask words [ia/32, ib/32) (relu(y) > 0 iff y > 0): lane l of a warp reads element
         // 32 w + l of each of 4 words (conflict-free), one ballot per word; tile-local 32-bit indices
         if (MASK) {
@@ -207,7 +240,7 @@ pool3_fwd_kernel(const float *__restrict__ y, P3Args a, float *__restrict__ out,
             // one thread per (plane, output column, row segment) walks down the segment's output
             // rows: input row 2 oh - P + 2 of one output is row 2 (oh + 1) - P of the next, so each
             // step scans two new input rows (separable, as for stride 1).  Nibble bytes go to
-            // shared memory by output index - olo8 (word boundaries 8-byte aligned), then packed.
+            // shared memory by output index - olo8 (word boundaries 8-byte aligned).
             const int64_t olo8 = olo & ~7ll;
             uint8_t *nb0 = nbs + (olo - olo8);
             const float *P0 = R + (t.lo - sb);  // plane 0 of the tile
@@ -287,19 +320,6 @@ pool3_fwd_kernel(const float *__restrict__ y, P3Args a, float *__restrict__ out,
                     }
                 nb0[t.np * a.HoWo + tid] = (uint8_t)bi;
             }
-            __syncthreads();
-            // pack the owned words [oa/8, ob/8): 8 nibble bytes each (one aligned 64-bit load);
-            // only the map's last word can be partial (its pad nibbles are 0)
-            const int w0 = (int)((t.oa - olo8) >> 3), w1 = (int)((t.ob - olo8 + 7) >> 3);
-            const int nvalid = (int)(t.ob - olo8);  // bytes written from olo8 on (last word of the map)
-            for (int w = w0 + tid; w < w1; w += kRT) {
-                const uint2 b = *reinterpret_cast<const uint2 *>(nbs + 8 * w);
-                const uint32_t lo4 = (b.x & 0xfu) | ((b.x >> 4) & 0xf0u) | ((b.x >> 8) & 0xf00u) | ((b.x >> 12) & 0xf000u);
-                const uint32_t hi4 = (b.y & 0xfu) | ((b.y >> 4) & 0xf0u) | ((b.y >> 8) & 0xf00u) | ((b.y >> 12) & 0xf000u);
-                const int valid = nvalid - 8 * w;
-                const uint32_t keep = valid >= 8 ? ~0u : ((1u << (4 * valid)) - 1u);
-                arg[(olo8 >> 3) + w] = (lo4 | (hi4 << 16)) & keep;
-            }
         } else {
             // stride 1 (G * HoWo % 8 == 0: every word whole in the tile): one thread per (plane,
             // output column, row segment) walks down the segment, one new input row per output.
@@ -344,24 +364,17 @@ pool3_fwd_kernel(const float *__restrict__ y, P3Args a, float *__restrict__ out,
                     hv1 = hv2, hx1 = hx2;
                 }
             }
-            __syncthreads();
-            // pack: one argmax word per thread (8 nibble bytes, one aligned 64-bit load); only the
-            // map's last word can be partial (its pad nibbles are 0)
-            const int no = t.np * a.HoWo;
-            const int nw = (no + 7) >> 3;
-            for (int w = tid; w < nw; w += kRT) {
-                const uint2 b = *reinterpret_cast<const uint2 *>(nbs + 8 * w);
-                const uint32_t lo4 = (b.x & 0xfu) | ((b.x >> 4) & 0xf0u) | ((b.x >> 8) & 0xf00u) | ((b.x >> 12) & 0xf000u);
-                const uint32_t hi4 = (b.y & 0xfu) | ((b.y >> 4) & 0xf0u) | ((b.y >> 8) & 0xf00u) | ((b.y >> 12) & 0xf000u);
-                const int valid = no - 8 * w;  // nibbles of this word inside the map
-                const uint32_t keep = valid >= 8 ? ~0u : ((1u << (4 * valid)) - 1u);
-                arg[(olo >> 3) + w] = (lo4 | (hi4 << 16)) & keep;
-            }
         }
-        __syncthreads();  // stage st (and the nibble bytes) consumed
+        // the previous tile's words, from the other nibble buffer (complete since the last barrier)
+        if (j > 0) pack(prev, nbs0 + ((j - 1) & 1) * kNbFwd);
+        prev = t;
+        // one barrier per tile: stage st and the previous tile's nibble bytes are consumed, this
+        // tile's nibble bytes are complete (packed during the next tile's walk)
+        __syncthreads();
         if (tid == 0 && j + a.rs < mine) issue(j + a.rs, st);
         if (++st == a.rs) st = 0, ph ^= 1u;
     }
+    if (mine > 0) pack(prev, nbs0 + ((mine - 1) & 1) * kNbFwd);
 }
 
 // ---------------------------------------------------------------- backward
@@ -841,8 +854,8 @@ cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, in
             unit = unit * mu / gcd_i(unit, mu);
         }
         a.G = choose_g(a.NC, a.HW, 64, unit, ctas, a.sf);
-        while (a.G > unit && (int64_t)a.G * a.HoWo > kNbBytes) a.G -= unit;
-        if (a.G == 0 || (int64_t)a.G * a.HoWo > kNbBytes) return cudaErrorNotSupported;
+        while (a.G > unit && (int64_t)a.G * a.HoWo > kNbFwd) a.G -= unit;
+        if (a.G == 0 || (int64_t)a.G * a.HoWo > kNbFwd) return cudaErrorNotSupported;
         const int64_t cols = (int64_t)a.G * Wo;  // row segments: about one item per thread
         const int32_t want = (int32_t)std::max<int64_t>(1, std::min<int64_t>(Ho, kRT / cols));
         a.segr = (Ho + want - 1) / want;
@@ -856,8 +869,8 @@ cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, in
         if (mask && a.HW % 32) xr = std::max(xr, std::min(H, (30 + W) / W));
         a.xrows = xr;
         a.G = choose_g(a.NC, a.HW, 64 + (int64_t)xr * W + 32, 1, ctas, a.sf);
-        while (a.G > 1 && (int64_t)a.G * a.HoWo + 14 > kNbBytes) --a.G;
-        if (a.G == 0 || (int64_t)a.G * a.HoWo + 14 > kNbBytes) return cudaErrorNotSupported;
+        while (a.G > 1 && (int64_t)a.G * a.HoWo + 14 > kNbFwd) --a.G;
+        if (a.G == 0 || (int64_t)a.G * a.HoWo + 14 > kNbFwd) return cudaErrorNotSupported;
         // row segments: about one (plane, column, segment) item per thread
         const int64_t cols = (int64_t)a.G * Wo;
         const int32_t want = (int32_t)std::max<int64_t>(1, std::min<int64_t>(Ho, kRT / cols));
