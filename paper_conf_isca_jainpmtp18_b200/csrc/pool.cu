@@ -647,27 +647,30 @@ pool_bwd_k3s2_block_kernel(const float *__restrict__ dout, const uint32_t *__res
         uint32_t nbv[4] = {15u, 15u, 15u, 15u};  // 15: no window / no hit
         const bool ok[4] = {up && left, up && here_c, here_r && left, here_r && here_c};
         const int os[4] = {o00, o00 + 1, o11 - 1, o11};
+        const uint32_t i00 = plane * HW + (2 * A) * (uint32_t)a.W + 2 * b;
+        const bool r1 = 2 * (int)A + 1 < a.H, c1 = 2 * (int)b + 1 < a.W;
+        // every load is issued before any is used (the mask words' latency overlaps the dY and
+        // argmax loads'; with the mask read after the nibbles were decoded it was a second round trip)
+        const bool hm = mask != nullptr;
+        const uint32_t i10 = i00 + (uint32_t)a.W;
+        // the right-hand bit is read only when that column exists (c1): in the last column of an
+        // odd-W map, element i00 + 1 may be element n, one word past the mask buffer
+        const uint32_t w0 = hm ? ld_ro(mask + (i00 >> 5)) : ~0u;
+        const uint32_t w0b = hm && c1 ? ld_ro(mask + ((i00 + 1) >> 5)) : ~0u;
+        const uint32_t w1 = hm && r1 ? ld_ro(mask + (i10 >> 5)) : ~0u;
+        const uint32_t w1b = hm && r1 && c1 ? ld_ro(mask + ((i10 + 1) >> 5)) : ~0u;
+        uint32_t aw[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) aw[k] = ok[k] ? ld_ro(arg + (os[k] >> 3)) : 0u;
         if (ok[0]) g[0] = ld_ro(g0);
         if (ok[1]) g[1] = ld_ro(g0 + 1);
         if (ok[2]) g[2] = ld_ro(g1);
         if (ok[3]) g[3] = ld_ro(g1 + 1);
 #pragma unroll
         for (int k = 0; k < 4; ++k)
-            if (ok[k]) nbv[k] = (ld_ro(arg + (os[k] >> 3)) >> (4 * (os[k] & 7))) & 0xfu;
-        const uint32_t i00 = plane * HW + (2 * A) * (uint32_t)a.W + 2 * b;
-        const bool r1 = 2 * (int)A + 1 < a.H, c1 = 2 * (int)b + 1 < a.W;
-        uint32_t m0 = 3u, m1 = 3u;
-        if (mask) {
-            // the right-hand bit is read only when that column exists (c1): in the last column of
-            // an odd-W map, element i00 + 1 may be element n, one word past the mask buffer
-            const uint32_t w0 = ld_ro(mask + (i00 >> 5)), w0b = c1 ? ld_ro(mask + ((i00 + 1) >> 5)) : 0u;
-            m0 = ((w0 >> (i00 & 31)) & 1u) | (((w0b >> ((i00 + 1) & 31)) & 1u) << 1);
-            if (r1) {
-                const uint32_t i10 = i00 + (uint32_t)a.W;
-                const uint32_t w1 = ld_ro(mask + (i10 >> 5)), w1b = c1 ? ld_ro(mask + ((i10 + 1) >> 5)) : 0u;
-                m1 = ((w1 >> (i10 & 31)) & 1u) | (((w1b >> ((i10 + 1) & 31)) & 1u) << 1);
-            }
-        }
+            if (ok[k]) nbv[k] = (aw[k] >> (4 * (os[k] & 7))) & 0xfu;
+        const uint32_t m0 = ((w0 >> (i00 & 31)) & 1u) | (((w0b >> ((i00 + 1) & 31)) & 1u) << 1);
+        const uint32_t m1 = ((w1 >> (i10 & 31)) & 1u) | (((w1b >> ((i10 + 1) & 31)) & 1u) << 1);
         float a00 = 0.0f, a01 = 0.0f, a10 = 0.0f, a11 = 0.0f;  // +0.0f, then ascending o
         if (nbv[0] == 8u) a00 = a00 + g[0];
         if (nbv[1] == 6u) a00 = a00 + g[1];
