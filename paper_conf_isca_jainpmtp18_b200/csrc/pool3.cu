@@ -784,6 +784,35 @@ int32_t choose_g(int64_t NC, int64_t per_plane, int64_t fixed, int32_t unit, int
     return (int32_t)g;
 }
 
+// Forward tile plan: planes per tile G (a multiple of `unit`, at most gmax) and output rows per
+// walker segment, chosen to minimise the busiest CTA's walk time: tiles per CTA x (rounds of kRT
+// items x (segment rows + the item's setup) + a per-tile overhead), in row steps.  (The earlier
+// rule -- G for ~4 tiles per CTA, then about one item per thread -- left e.g. 336 of 512 threads
+// busy on GoogLeNet's 14x14 planes.)
+#ifndef GIST_POOL3_PLAN
+#define GIST_POOL3_PLAN 1
+#endif
+struct FwdPlan {
+    int32_t G, segr, segs;
+};
+FwdPlan plan_fwd(int64_t NC, int32_t Ho, int32_t Wo, int32_t unit, int32_t gmax, int64_t ctas) {
+    FwdPlan best{0, 0, 0};
+    double best_cost = 1e300;
+    for (int32_t g = unit; g <= gmax; g += unit) {
+        const int64_t tiles = (NC + g - 1) / g;
+        const int64_t per_cta = (tiles + ctas - 1) / ctas;
+        for (int32_t segr = 1; segr <= Ho; ++segr) {
+            const int32_t segs = (Ho + segr - 1) / segr;
+            if (segr > 1 && (Ho + segr - 2) / (segr - 1) == segs) continue;  // same segments, longer rows
+            const int64_t items = (int64_t)g * Wo * segs;
+            const int64_t rounds = (items + kRT - 1) / kRT;
+            const double cost = (double)per_cta * ((double)rounds * (segr + 0.6) + 4.0);
+            if (cost < best_cost - 1e-9) best_cost = cost, best = FwdPlan{g, segr, segs};
+        }
+    }
+    return best;
+}
+
 // Ring per kernel kind (stages x KB per stage), measured on B200 (AlexNet / NiN / GoogLeNet maps):
 // stride-2 forward 2 x 48 KB (was 3 x 32: AlexNet relu1 62 -> 52 us, fewer per-tile overheads),
 // the others 3 x 32 KB.  GIST_POOL3_RING="f1=3x32,f2=2x48,b1=3x32,b2=3x32" overrides (tuning).
@@ -860,6 +889,12 @@ cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, in
         const int32_t want = (int32_t)std::max<int64_t>(1, std::min<int64_t>(Ho, kRT / cols));
         a.segr = (Ho + want - 1) / want;
         a.segs = (Ho + a.segr - 1) / a.segr;
+        if (GIST_POOL3_PLAN) {
+            int32_t gmax = (int32_t)std::min<int64_t>((a.sf - 64) / a.HW, kNbFwd / a.HoWo);
+            gmax = gmax / unit * unit;
+            const FwdPlan pl = plan_fwd(a.NC, Ho, Wo, unit, gmax, ctas);
+            if (pl.G > 0) a.G = pl.G, a.segr = pl.segr, a.segs = pl.segs;
+        }
         a.div_seg = FastDiv::make((uint32_t)a.segs);
     } else {
         // rows of the next plane a tile may need: the windows of its last argmax word's (<= 7)
@@ -876,6 +911,11 @@ cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, in
         const int32_t want = (int32_t)std::max<int64_t>(1, std::min<int64_t>(Ho, kRT / cols));
         a.segr = (Ho + want - 1) / want;
         a.segs = (Ho + a.segr - 1) / a.segr;
+        if (GIST_POOL3_PLAN) {
+            int32_t gmax = (int32_t)std::min<int64_t>((a.sf - 64 - (int64_t)xr * W - 32) / a.HW, (kNbFwd - 14) / a.HoWo);
+            const FwdPlan pl = plan_fwd(a.NC, Ho, Wo, 1, gmax, ctas);
+            if (pl.G > 0) a.G = pl.G, a.segr = pl.segr, a.segs = pl.segs;
+        }
         a.div_seg = FastDiv::make((uint32_t)a.segs);
     }
     a.tiles = ceil_div(a.NC, a.G);
