@@ -786,7 +786,8 @@ int32_t choose_g(int64_t NC, int64_t per_plane, int64_t fixed, int32_t unit, int
 
 // Forward tile plan: planes per tile G (a multiple of `unit`, at most gmax) and output rows per
 // walker segment, chosen to minimise the busiest CTA's walk time: tiles per CTA x (rounds of kRT
-// items x (segment rows + the item's setup) + a per-tile overhead), in row steps.  (The earlier
+// items x (segment rows + the item's setup and first rows, `warm`) + a per-tile overhead), in row
+// steps.  (The earlier
 // rule -- G for ~4 tiles per CTA, then about one item per thread -- left e.g. 336 of 512 threads
 // busy on GoogLeNet's 14x14 planes.)
 #ifndef GIST_POOL3_PLAN
@@ -795,20 +796,37 @@ int32_t choose_g(int64_t NC, int64_t per_plane, int64_t fixed, int32_t unit, int
 struct FwdPlan {
     int32_t G, segr, segs;
 };
-FwdPlan plan_fwd(int64_t NC, int32_t Ho, int32_t Wo, int32_t unit, int32_t gmax, int64_t ctas) {
+FwdPlan plan_fwd(int64_t NC, int32_t Ho, int32_t Wo, int32_t unit, int32_t gmax, int64_t ctas, double warm) {
     FwdPlan best{0, 0, 0};
     double best_cost = 1e300;
     for (int32_t g = unit; g <= gmax; g += unit) {
-        const int64_t tiles = (NC + g - 1) / g;
-        const int64_t per_cta = (tiles + ctas - 1) / ctas;
+        const int64_t per_cta = ((NC + g - 1) / g + ctas - 1) / ctas;
         for (int32_t segr = 1; segr <= Ho; ++segr) {
             const int32_t segs = (Ho + segr - 1) / segr;
             if (segr > 1 && (Ho + segr - 2) / (segr - 1) == segs) continue;  // same segments, longer rows
-            const int64_t items = (int64_t)g * Wo * segs;
-            const int64_t rounds = (items + kRT - 1) / kRT;
-            const double cost = (double)per_cta * ((double)rounds * (segr + 0.6) + 4.0);
-            if (cost < best_cost - 1e-9) best_cost = cost, best = FwdPlan{g, segr, segs};
+            const int64_t rounds = ((int64_t)g * Wo * segs + kRT - 1) / kRT;
+            const double cost = (double)per_cta * ((double)rounds * (segr + warm) + 4.0);
+            // ties go to the larger G (fewer tiles: GoogLeNet inc4b 14x14, G = 28 vs 36 at equal cost
+            // measured 27.4 vs 20.0 us)
+            if (cost < best_cost - 1e-9 || (cost < best_cost + 1e-9 && g > best.G))
+                best_cost = cost, best = FwdPlan{g, segr, segs};
         }
+    }
+    return best;
+}
+
+// Backward (hit masks) tile plan: planes per tile chosen to minimise the busiest CTA's time, tiles
+// per CTA x (rounds of kRT argmax words x 3 + rounds of kRT inputs + a per-tile overhead of 4).
+// The caller keeps the earlier G when it is larger (GoogLeNet inc3a: the model's pick, 7 planes
+// instead of 8, measured 6% slower).
+int32_t plan_bwd_hits(int64_t NC, int64_t HoWo, int64_t HW, int32_t gmax, int64_t ctas) {
+    int32_t best = 0;
+    double best_cost = 1e300;
+    for (int32_t g = 1; g <= gmax; ++g) {
+        const int64_t per_cta = ((NC + g - 1) / g + ctas - 1) / ctas;
+        const int64_t r1 = ((g * HoWo + 7) / 8 + kRT - 1) / kRT, r2 = (g * HW + kRT - 1) / kRT;
+        const double cost = (double)per_cta * (3.0 * r1 + r2 + 4.0);
+        if (cost < best_cost + 1e-9) best_cost = std::min(best_cost, cost), best = g;  // ties: the larger G
     }
     return best;
 }
@@ -892,7 +910,9 @@ cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, in
         if (GIST_POOL3_PLAN) {
             int32_t gmax = (int32_t)std::min<int64_t>((a.sf - 64) / a.HW, kNbFwd / a.HoWo);
             gmax = gmax / unit * unit;
-            const FwdPlan pl = plan_fwd(a.NC, Ho, Wo, unit, gmax, ctas);
+            const char *fg = getenv("GIST_POOL3_FWD_G");  // tuning only: a fixed G (its segments planned)
+            const int32_t gf = fg ? atoi(fg) / unit * unit : 0;
+            const FwdPlan pl = gf > 0 && gf <= gmax ? plan_fwd(a.NC, Ho, Wo, gf, gf, ctas, 1.6) : plan_fwd(a.NC, Ho, Wo, unit, gmax, ctas, 1.6);
             if (pl.G > 0) a.G = pl.G, a.segr = pl.segr, a.segs = pl.segs;
         }
         a.div_seg = FastDiv::make((uint32_t)a.segs);
@@ -913,7 +933,7 @@ cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, in
         a.segs = (Ho + a.segr - 1) / a.segr;
         if (GIST_POOL3_PLAN) {
             int32_t gmax = (int32_t)std::min<int64_t>((a.sf - 64 - (int64_t)xr * W - 32) / a.HW, (kNbFwd - 14) / a.HoWo);
-            const FwdPlan pl = plan_fwd(a.NC, Ho, Wo, 1, gmax, ctas);
+            const FwdPlan pl = plan_fwd(a.NC, Ho, Wo, 1, gmax, ctas, 1.0);
             if (pl.G > 0) a.G = pl.G, a.segr = pl.segr, a.segs = pl.segs;
         }
         a.div_seg = FastDiv::make((uint32_t)a.segs);
@@ -984,6 +1004,11 @@ cudaError_t launch_pool3_bwd(const float *dout, const uint32_t *argmax, const ui
     const int64_t aux_cap = hitk ? (a.S == 1 ? kHitBytes : 2 * (int64_t)kHitBytes) : kNbBytes;  // S = 2: half bytes
     while (a.G > 1 && (int64_t)a.G * aux_plane + 32 > aux_cap) --a.G;
     if (a.G == 0 || (int64_t)a.G * aux_plane + 32 > aux_cap) return cudaErrorNotSupported;
+    if (hitk && GIST_POOL3_PLAN) {
+        const int64_t gfit = std::min<int64_t>((a.sf - 64) / per_plane, (aux_cap - 32) / aux_plane);
+        const int32_t g = plan_bwd_hits(a.NC, a.HoWo, a.HW, (int32_t)gfit, ctas);
+        if (g > a.G) a.G = g;
+    }
     a.tiles = ceil_div(a.NC, a.G);
     const int64_t G = a.G;
     a.a_off = (int32_t)((G * a.HoWo + 8 + 3) & ~3ll);

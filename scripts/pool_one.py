@@ -27,6 +27,8 @@ CASES = {
     "googlenet1": ((64, 64, 112, 112), WL.P3S2C),
     "inc3a": ((64, 192, 28, 28), WL.P3S1P1),
     "inc4a": ((64, 480, 14, 14), WL.P3S1P1),
+    "inc4b": ((64, 512, 14, 14), WL.P3S1P1),
+    "inc3b": ((64, 256, 28, 28), WL.P3S1P1),
     "inc5a": ((64, 832, 7, 7), WL.P3S1P1),
 }
 
