@@ -66,6 +66,7 @@ struct P3Args {
     int32_t a_off, m_off;  // backward stage layout (floats): dY at 0, argmax words, mask words
     int32_t segs, segr;    // stride-2 forward: row segments per plane column, output rows per segment
     int32_t rs, sf;        // ring: stages, floats per stage
+    int32_t bands, br;     // stride-2 forward of planes larger than a stage: bands per plane, output rows per band
     int64_t NC, tiles, n_in, n_out;
     FastDiv div_hw, div_w, div_howo, div_wo, div_blk, div_wb, div_seg;
 };
@@ -109,12 +110,39 @@ __device__ __forceinline__ bool tail_fill(T *dst, const T *__restrict__ src, int
 
 struct FwdTile {
     int64_t p0, lo, hi, oa, ob, ia, ib;
-    int64_t ce;  // end of the bulk-copied range (>= hi except at the map's ragged end)
+    int64_t ce;   // end of the bulk-copied range (>= hi except at the map's ragged end)
+    int64_t olo;  // first output of the tile (plane p0, output row oh0)
     int np;
+    int oh0, oh1;  // output rows of the tile's planes ([0, Ho) unless banded)
 };
 
 __device__ __forceinline__ FwdTile fwd_tile(const P3Args &a, int64_t k) {
     FwdTile t;
+    if (a.bands > 1) {
+        // one band of output rows [oh0, oh1) of plane p0 (stride 2, P = 0, Wo % 8 == 0 and 2W % 32 ==
+        // 0, so a band owns whole argmax words and the mask words of its input rows [2 oh0, 2 oh1),
+        // the last band up to H); it stages input rows [2 oh0, min(H, 2 oh1 + 1))
+        t.p0 = k / a.bands;
+        const int b = (int)(k - t.p0 * a.bands);
+        t.np = 1;
+        t.oh0 = b * a.br;
+        t.oh1 = min(a.Ho, t.oh0 + a.br);
+        const int64_t pb = t.p0 * a.HW;
+        const int ih_own1 = t.oh1 == a.Ho ? a.H : 2 * t.oh1;
+        t.olo = t.p0 * a.HoWo + (int64_t)t.oh0 * a.Wo;
+        t.oa = t.olo;
+        t.ob = t.p0 * a.HoWo + (int64_t)t.oh1 * a.Wo;
+        t.ia = pb + (int64_t)(2 * t.oh0) * a.W;
+        t.ib = pb + (int64_t)ih_own1 * a.W;
+        t.lo = t.ia;
+        t.hi = pb + (int64_t)min(a.H, 2 * t.oh1 + 1) * a.W;
+        const int64_t up = (t.hi + 3) & ~3ll;
+        t.ce = up <= a.n_in ? up : (t.hi & ~3ll);
+        if (t.ce < (t.lo & ~3ll)) t.ce = t.lo & ~3ll;
+        return t;
+    }
+    t.oh0 = 0;
+    t.oh1 = a.Ho;
     t.p0 = k * a.G;
     t.np = (int)min((int64_t)a.G, a.NC - t.p0);
     const bool last = t.p0 + t.np == a.NC;
@@ -122,6 +150,7 @@ __device__ __forceinline__ FwdTile fwd_tile(const P3Args &a, int64_t k) {
     t.ob = last ? a.n_out : (((t.p0 + t.np) * a.HoWo + 7) & ~7ll);
     t.ia = (t.p0 * a.HW + 31) & ~31ll;
     t.ib = last ? a.n_in : (((t.p0 + t.np) * a.HW + 31) & ~31ll);
+    t.olo = t.p0 * a.HoWo;
     t.lo = t.p0 * a.HW;
     const int64_t end = t.lo + (int64_t)t.np * a.HW;
     t.hi = last ? end : min(a.n_in, end + max((int64_t)a.xrows * a.W, t.ib - end));
@@ -177,7 +206,7 @@ pool3_fwd_kernel(const float *__restrict__ y, P3Args a, float *__restrict__ out,
     // only the map's last word can be partial (its pad nibbles are 0).  Run one tile later, between
     // the next tile's walk and the barrier that ends it (the bytes are double-buffered).
     auto pack = [&](const FwdTile &t, const uint8_t *nbs) {
-        const int64_t olo = t.p0 * a.HoWo;
+        const int64_t olo = t.olo;
         const int64_t olo8 = S == 2 ? (olo & ~7ll) : olo;  // stride 1: tiles hold whole words
         const int w0 = S == 2 ? (int)((t.oa - olo8) >> 3) : 0;
         const int64_t oend = S == 2 ? t.ob : olo + (int64_t)t.np * a.HoWo;
@@ -235,22 +264,24 @@ pool3_fwd_kernel(const float *__restrict__ y, P3Args a, float *__restrict__ out,
                 if (lane == 0) mw[w] = b;
             }
         }
-        const int64_t olo = t.p0 * a.HoWo;
+        const int64_t olo = t.olo;
         if (S == 2) {
             // one thread per (plane, output column, row segment) walks down the segment's output
             // rows: input row 2 oh - P + 2 of one output is row 2 (oh + 1) - P of the next, so each
             // step scans two new input rows (separable, as for stride 1).  Nibble bytes go to
             // shared memory by output index - olo8 (word boundaries 8-byte aligned).
             const int64_t olo8 = olo & ~7ll;
-            uint8_t *nb0 = nbs + (olo - olo8);
-            const float *P0 = R + (t.lo - sb);  // plane 0 of the tile
-            float *otile = out + olo;
+            // banded tiles: the tile's output rows [t.oh0, t.oh1) of plane p0; P0 addresses row 0 of
+            // that plane (rows above the band are not staged and not read)
+            uint8_t *nb0 = nbs + (olo - olo8) - (int64_t)t.oh0 * a.Wo;
+            const float *P0 = R + (t.p0 * a.HW - sb);  // plane 0 of the tile
+            float *otile = out + olo - (int64_t)t.oh0 * a.Wo;
             const int items = t.np * a.segs * a.Wo;
             for (int it = tid; it < items; it += kRT) {
                 uint32_t ps, ow, pl, sg;
                 a.div_wo.divmod((uint32_t)it, ps, ow);
                 a.div_seg.divmod(ps, pl, sg);
-                const int oh0 = (int)sg * a.segr, oh1 = min(a.Ho, oh0 + a.segr);
+                const int oh0 = t.oh0 + (int)sg * a.segr, oh1 = min(t.oh1, oh0 + a.segr);
                 const float *pb = P0 + (int)pl * a.HW;
                 const int iw0 = 2 * (int)ow - a.P;
                 const int dx0 = max(0, -iw0);
@@ -873,6 +904,9 @@ int64_t resident_ctas(size_t smem) {
 #ifndef GIST_POOL3_S2
 #define GIST_POOL3_S2 1
 #endif
+#ifndef GIST_POOL3_BAND
+#define GIST_POOL3_BAND 1  // stride-2 forward of planes larger than a stage in bands of output rows
+#endif
 #ifndef GIST_POOL3_S2_BWD
 #define GIST_POOL3_S2_BWD 0
 #endif
@@ -925,7 +959,28 @@ cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, in
         a.xrows = xr;
         a.G = choose_g(a.NC, a.HW, 64 + (int64_t)xr * W + 32, 1, ctas, a.sf);
         while (a.G > 1 && (int64_t)a.G * a.HoWo + 14 > kNbFwd) --a.G;
-        if (a.G == 0 || (int64_t)a.G * a.HoWo + 14 > kNbFwd) return cudaErrorNotSupported;
+        const bool fits = a.G > 0 && (int64_t)a.G * a.HoWo + 14 <= kNbFwd;
+        // a plane larger than a stage (GoogLeNet's 112x112 stem): bands of output rows, when every
+        // band owns whole argmax and mask words (P = 0, Wo % 8 == 0, W % 16 == 0, HW % 32 == 0)
+        const char *fb = getenv("GIST_POOL3_BANDS");  // testing: force this many bands per plane
+        const int32_t force = fb ? atoi(fb) : 0;
+        if ((!fits || force > 1) && GIST_POOL3_BAND && a.P == 0 && Wo % 8 == 0 && W % 16 == 0 && a.HW % 32 == 0) {
+            const int32_t br_max = (int32_t)std::min<int64_t>((((int64_t)a.sf - 64) / W - 1) / 2, kNbFwd / Wo);
+            if (br_max < 1) return cudaErrorNotSupported;
+            a.bands = force > 1 ? std::min(force, Ho) : (Ho + br_max - 1) / br_max;
+            a.br = (Ho + a.bands - 1) / a.bands;
+            a.bands = (Ho + a.br - 1) / a.br;
+            if (a.br > br_max) return cudaErrorNotSupported;
+            a.G = 1;
+            a.xrows = 0;
+            const int32_t want = (int32_t)std::max<int64_t>(1, std::min<int64_t>(a.br, kRT / Wo));
+            a.segr = (a.br + want - 1) / want;
+            a.segs = (a.br + a.segr - 1) / a.segr;
+            a.div_seg = FastDiv::make((uint32_t)a.segs);
+            a.tiles = a.NC * a.bands;
+            goto launch;
+        }
+        if (!fits) return cudaErrorNotSupported;
         // row segments: about one (plane, column, segment) item per thread
         const int64_t cols = (int64_t)a.G * Wo;
         const int32_t want = (int32_t)std::max<int64_t>(1, std::min<int64_t>(Ho, kRT / cols));
@@ -939,6 +994,7 @@ cudaError_t launch_pool3_fwd(const float *y, int32_t N, int32_t C, int32_t H, in
         a.div_seg = FastDiv::make((uint32_t)a.segs);
     }
     a.tiles = ceil_div(a.NC, a.G);
+launch:
     // every window inside the input: no bounds tests (AlexNet's floor-mode 3x3/s2)
     const bool check = !(a.P == 0 && (Ho - 1) * a.S + 3 <= H && (Wo - 1) * a.S + 3 <= W);
     const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(a.tiles, ctas));

@@ -144,6 +144,33 @@ def test_relu_maxpool_fwd_in_place_relu(gist, ref, cuda, g, shape):
     assert_bits_equal(host(mask), ref.binarize_encode(y), "mask")
 
 
+@pytest.mark.parametrize("bands", [2, 3, 5])
+@pytest.mark.parametrize("shape,g", [((2, 5, 48, 48), (3, 3, 2, 2, 0, 0, 1)), ((3, 4, 32, 32), (3, 3, 2, 2, 0, 0, 1)),
+                                     ((1, 6, 80, 80), (3, 3, 2, 2, 0, 0, 1))],
+                         ids=["48x48ceil", "32x32ceil", "80x80ceil"])
+def test_pool3_banded_stride2_forward(gist, ref, cuda, monkeypatch, bands, shape, g):
+    """The stride-2 forward in bands of output rows (the path of planes larger than a stage, e.g.
+    GoogLeNet's 112x112 stem), forced on small planes with GIST_POOL3_BANDS: out, argmax and the
+    fused mask (with and without the in-place ReLU) equal the oracle's, including a ragged last band."""
+    monkeypatch.setenv("GIST_POOL3_BANDS", str(bands))
+    y = pool_case(shape, g, sum(shape) + bands, cuda)
+    out, arg, mask = gist.gist_maxpool_fwd_argmax(y, g, fuse_mask=True)
+    r_out, r_arg = ref.maxpool_fwd_argmax(host(y), g)
+    assert_bits_equal(host(out), r_out, "out")
+    assert_bits_equal(host(arg), r_arg, "argmax")
+    assert_bits_equal(host(mask), ref.binarize_encode(host(y)), "mask")
+    out2, arg2, _ = gist.gist_maxpool_fwd_argmax(y, g)
+    assert_bits_equal(host(out2), r_out, "out (no mask)")
+    assert_bits_equal(host(arg2), r_arg, "argmax (no mask)")
+    x = WL.grad_map(shape, sum(shape), cuda)
+    xr = torch.relu(x.cpu()).numpy()
+    out3, arg3, mask3 = gist.gist_relu_maxpool_fwd_argmax(x, g)
+    r_out3, r_arg3 = ref.maxpool_fwd_argmax(xr, g)
+    assert_bits_equal(host(out3), r_out3, "out (relu on load)")
+    assert_bits_equal(host(arg3), r_arg3, "argmax (relu on load)")
+    assert_bits_equal(host(mask3), ref.binarize_encode(xr), "mask (relu on load)")
+
+
 def test_fused_bwd_equals_torch_autograd_on_gpu_inputs(gist, cuda):
     # Same chain as the CPU pin, but on the GPU kernels: relu -> max_pool2d (AlexNet 3x3/s2).
     g = (3, 3, 2, 2, 0, 0, 0)
