@@ -88,8 +88,12 @@ constexpr int kPartRows = kTileRows / kParts;
 constexpr int kPartElems = kPartRows * kRow;           // 8 KB per TMA stage (4 parts)
 constexpr int kStages = GIST_SSDC_STAGES;
 constexpr int kQ = GIST_SSDC_Q;
+#ifndef GIST_SSDC_STORER
+#define GIST_SSDC_STORER 1  // a store warp issues each tile's bulk copies (the writers never wait on each other)
+#endif
 constexpr int kProd = 0, kCount = 1, kPub = kCount + kParts, kGather = kPub + 1, kWriter0 = kGather + 1;
-constexpr int kEncThreads = 32 * (kWriter0 + kWriters);  // 15 warps = 480 threads (8 writers)
+constexpr int kStorer = kWriter0 + kWriters;
+constexpr int kEncThreads = 32 * (kWriter0 + kWriters + GIST_SSDC_STORER);  // 16 warps = 512 threads (8 writers)
 constexpr int kStage = kTileRows * kRow + 16;  // staged entries per tile (+ 16-entry phase)
 constexpr int kWriterThreads = 32 * kWriters;
 constexpr int kGatherPer = 8;                     // totals per lane per gather round (256 per warp)
@@ -146,6 +150,7 @@ struct __align__(128) EncSmem {
     int32_t job[kQ];                 // job of that tile
     uint64_t full[kStages], empty[kStages];
     uint64_t counted[kQ], published[kQ], resolved[kQ], freed[kQ];
+    uint64_t staged[kQ], sfree[2];  // writers -> store warp (tile staged), store warp -> writers (buffer read)
 };
 
 // The tile totals are self-contained words (tag | count) and nothing else is published with
@@ -323,8 +328,10 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
             mbar_init(&S.counted[q], kParts);
             mbar_init(&S.published[q], 1);
             mbar_init(&S.resolved[q], 1);
-            mbar_init(&S.freed[q], kWriters);
+            mbar_init(&S.freed[q], GIST_SSDC_STORER ? 1 : kWriters);
+            mbar_init(&S.staged[q], kWriters);
         }
+        for (int b = 0; b < 2; ++b) mbar_init(&S.sfree[b], 1);
         fence_mbar_init();
     }
 #if GIST_PDL
@@ -473,6 +480,26 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
             }
             if (t >= tiles) break;
         }
+    } else if (GIST_SSDC_STORER && warp == kStorer) {
+        // ---- store warp: once the writers have staged tile jj, its whole 16-entry groups leave as two
+        // bulk copies (and the ragged head and tail as plain stores); when the copies have read the
+        // staging buffer, the buffer goes back to the writers and the slot to the producer
+        for (uint32_t jj = 0;; ++jj) {
+            const int q = (int)(jj % kQ);
+            const int sb = (int)(jj & 1);
+            mbar_wait_sleep(&S.published[q], (uint32_t)(jj / kQ) & 1u);
+            if (S.tile[q] >= tiles) break;
+            mbar_wait_sleep(&S.staged[q], (uint32_t)(jj / kQ) & 1u);
+            store_tile(S, q, sb, lane, J);
+            if (lane == 0) bulk_wait_read();
+            __syncwarp();
+            if (lane == 0) {
+                TRACE(jj, 3);
+                mbar_arrive1(&S.sfree[sb]);
+                mbar_arrive1(&S.freed[q]);
+            }
+        }
+        if (lane == 0) bulk_wait_all();
     } else if (warp == kGather) {
         // ---- gatherer: running prefix over all tile totals, in tile order.  For each of this
         // CTA's tiles t: sum tot[pos .. t) (up to 256 totals per coalesced round trip; re-poll
@@ -575,6 +602,15 @@ ssdc_encode_kernel(const __grid_constant__ EncJobs J, uint32_t *__restrict__ ws)
             const int q = (int)(jj % kQ);
             const int sb = (int)(jj & 1);
             mbar_wait_sleep(&S.resolved[q], (uint32_t)(jj / kQ) & 1u);
+#if GIST_SSDC_STORER
+            // buffer sb was last staged for tile jj - 2: wait until the store warp's copies have read it
+            if (jj >= 2) mbar_wait_sleep(&S.sfree[sb], (uint32_t)((jj - 2) / 2) & 1u);
+            stage_rows(S, q, sb, w, lane, l, h);
+            fence_proxy_async_smem();  // generic staging writes -> async-proxy bulk reads
+            __syncwarp();
+            if (lane == 0) mbar_arrive1(&S.staged[q]);
+            return;
+#endif
             stage_rows(S, q, sb, w, lane, l, h);
             fence_proxy_async_smem();  // generic staging writes -> async-proxy bulk reads
             if (w == 0 && lane == 0) bulk_wait_read();
