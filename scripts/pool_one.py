@@ -26,6 +26,10 @@ CASES = {
     "nin4": ((256, 256, 27, 27), WL.P3S2C),
     "googlenet1": ((64, 64, 112, 112), WL.P3S2C),
     "inc3a": ((64, 192, 28, 28), WL.P3S1P1),
+    "vgg1": ((64, 64, 224, 224), WL.P2S2),
+    "vgg3": ((64, 256, 56, 56), WL.P2S2),
+    "vgg4": ((64, 512, 28, 28), WL.P2S2),
+    "vgg5": ((64, 512, 14, 14), WL.P2S2),
     "inc4a": ((64, 480, 14, 14), WL.P3S1P1),
     "inc4b": ((64, 512, 14, 14), WL.P3S1P1),
     "inc3b": ((64, 256, 28, 28), WL.P3S1P1),
