@@ -306,9 +306,10 @@ class KernelTimer:
     """CUDA events around every launch, on the stream the kernels are launched on (and an NVTX range
     per call site when nvtx is set)."""
 
-    def __init__(self, stream, nvtx=False):
-        self.stream = stream
+    def __init__(self, stream, nvtx=False, external=False):
+        self.stream = stream  # None: the current stream (inside a graph capture, the capturing one)
         self.nvtx = nvtx
+        self.external = external  # events recorded as graph nodes (cudaEventRecordExternal)
         self.records = []  # (kind, site dict, start, end)
 
     def __call__(self, kind, d):
@@ -318,13 +319,14 @@ class KernelTimer:
             def __enter__(self_inner):
                 if timer.nvtx:
                     torch.cuda.nvtx.range_push(site_label(kind, d))
-                self_inner.s = torch.cuda.Event(enable_timing=True)
-                self_inner.e = torch.cuda.Event(enable_timing=True)
-                self_inner.s.record(timer.stream)
+                self_inner.s = torch.cuda.Event(enable_timing=True, external=timer.external)
+                self_inner.e = torch.cuda.Event(enable_timing=True, external=timer.external)
+                self_inner.st = timer.stream if timer.stream is not None else torch.cuda.current_stream()
+                self_inner.s.record(self_inner.st)
                 return self_inner
 
             def __exit__(self_inner, *a):
-                self_inner.e.record(timer.stream)
+                self_inner.e.record(self_inner.st)
                 if timer.nvtx:
                     torch.cuda.nvtx.range_pop()
                 timer.records.append((kind, d, self_inner.s, self_inner.e))
@@ -694,12 +696,39 @@ def main():
         if graph is not None:
             launches = per_step_launches * args.steps
         elapsed_ms = ev0.elapsed_time(ev1)
+        # the instrumented step, also as a graph when the timed step was one: the event pairs are graph
+        # nodes, so a small kernel's time does not include the host's per-call gap before it
+        g_inst, inst_note = None, "eager launches"
+        if graph is not None:
+            try:
+                timer_g = KernelTimer(None, external=True)
+                g_i = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g_i):
+                    wl.step(timer_g)
+                g_i.replay()
+                torch.cuda.synchronize()
+                g_inst, inst_note = g_i, "graph replays (event pairs as graph nodes)"
+            except Exception as ex:  # noqa: BLE001  (the eager instrumented pass below)
+                inst_note = f"eager launches (instrumented graph failed: {type(ex).__name__})"
+                torch.cuda.synchronize()
         ev2, ev3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev2.record(stream)
         for _ in range(args.steps):
-            wl.step(timer)
+            if g_inst is not None:
+                g_inst.replay()
+            else:
+                wl.step(timer)
         ev3.record(stream)
         barrier()
+        if g_inst is not None:
+            # per-launch times: one replay at a time (each replay re-records the same events)
+            timer.records = []
+            for _ in range(args.steps):
+                g_inst.replay()
+                torch.cuda.synchronize()
+                timer.records += [(k_, d_, s_.elapsed_time(e_)) for (k_, d_, s_, e_) in timer_g.records]
+        else:
+            timer.records = [(k_, d_, s_.elapsed_time(e_)) for (k_, d_, s_, e_) in timer.records]
     instrumented_ms = ev2.elapsed_time(ev3) / args.steps
     nnz = wl.nnz_host().tolist()
 
@@ -712,9 +741,8 @@ def main():
             nnz_of[id(d)] = int(nnz[k])
             k += 1
     per_site = {}  # (kind, site label) -> [ms, launches, algorithmic bytes]
-    for kind, d, s, e in timer.records:
+    for kind, d, ms in timer.records:
         r = per.setdefault(kind, {"ms": 0.0, "launches": 0, "algo_bytes": 0})
-        ms = s.elapsed_time(e)
         b = wl.algo_bytes(kind, d, nnz_of if isinstance(d, list) else nnz_of.get(id(d)))
         r["ms"] += ms
         r["launches"] += 1
@@ -830,7 +858,8 @@ def main():
         "clocks": clocks.summary(),
         "compression": wl.compression(nnz),
         "kernels": kernels,
-        "kernels_pass": {"note": "per-kernel times from K further steps with an event pair around every launch",
+        "kernels_pass": {"note": "per-kernel times from K further steps with an event pair around every launch, "
+                                 + inst_note,
                          "ms_per_step": round(instrumented_ms, 4)},
         "stash_bytes_per_gpu": 4 * wl.stash_elems,
     }
