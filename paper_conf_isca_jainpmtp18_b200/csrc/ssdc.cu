@@ -20,9 +20,11 @@
 //   * gatherer warp: running prefix over tot[] -> the tile's global offset, and row_end;
 //   * 8 writer warps (4 rows each): once the tile is published, load their rows from the ring
 //     into registers (one tile ahead) and release the stage; rank nonzeros (lane l owns columns
-//     l + 32k; one ballot per 32 columns, row starts from the publisher's row scan), stage them in
-//     shared memory congruent to the output mod 16, and store the whole 16-entry groups of
-//     val/col with two 1-D bulk copies (shared -> global) once the offset is resolved.
+//     l + 32k; one ballot per 32 columns, row starts from the publisher's row scan) and, once the
+//     offset is resolved, stage them in shared memory congruent to the output mod 16;
+//   * store warp: the whole 16-entry groups of val/col leave with two 1-D bulk copies (shared ->
+//     global) per tile, the ragged head and tail with plain stores; the staging buffer then goes
+//     back to the writers and the tile slot to the producer.
 // HBM sees the algorithmic traffic: 4n read once, 5*nnz + 4*rows written.
 // DESIGN.md §6 has the measured history of the alternatives (decoupled look-back, chunked
 // all-to-all prefix, single-pass compaction into a pending ring, L2 re-read writers).
